@@ -1,0 +1,272 @@
+"""CPU oracle for the retarded-potential step (Arumugam et al., ICPP'17).
+
+TEST INFRASTRUCTURE ONLY.  Only ``tests/``, ``__graft_entry__.smoke()`` and the
+``cpu_baseline`` / ``--impl reference`` legs of ``bench.py`` may import this
+module.  The product package never imports it and it imports nothing from the
+product package.
+
+This module is argument marshalling (ctypes) around ``rp_oracle.c``; every
+arithmetic step of the method lives in that C file, which cites PAPER.md
+(``/root/reference/PAPER.md``) line by line.  ``build()`` compiles it with
+``gcc -O2 -ffp-contract=off -fopenmp`` (no FMA contraction, plain IEEE FP64).
+"""
+from __future__ import annotations
+
+import ctypes as C
+import os
+import subprocess
+
+import numpy as np
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+_SRC = os.path.join(_HERE, "rp_oracle.c")
+_LIB = os.path.join(_HERE, "liboracle.so")
+
+SRC_GRID, SRC_GAUSS, SRC_DISK = 0, 1, 2
+
+
+def build(force: bool = False) -> str:
+    """Compile rp_oracle.c into liboracle.so (in-tree)."""
+    if force or not os.path.exists(_LIB) or os.path.getmtime(_LIB) < os.path.getmtime(_SRC):
+        tmp = _LIB + f".tmp{os.getpid()}"
+        subprocess.check_call(["gcc", "-O2", "-ffp-contract=off", "-fno-fast-math", "-fopenmp",
+                               "-std=c11", "-shared", "-fPIC", "-Wall", "-o", tmp, _SRC, "-lm"])
+        os.replace(tmp, _LIB)
+    return _LIB
+
+
+class Frame(C.Structure):
+    _fields_ = [("ox", C.c_double), ("oy", C.c_double), ("c", C.c_double), ("s", C.c_double)]
+
+
+class Params(C.Structure):
+    _fields_ = [("nx", C.c_int32), ("ny", C.c_int32), ("hx", C.c_double), ("hy", C.c_double),
+                ("c", C.c_double), ("dt", C.c_double), ("tau", C.c_double),
+                ("n_theta", C.c_int32), ("max_depth", C.c_int32), ("n_root", C.c_int32),
+                ("kappa_max", C.c_int32)]
+
+
+class Hist(C.Structure):
+    _fields_ = [("ring", C.POINTER(C.c_double)), ("frames", C.POINTER(Frame)),
+                ("H", C.c_int32), ("k", C.c_int32), ("n_pre", C.c_int32)]
+
+
+class Source(C.Structure):
+    _fields_ = [("kind", C.c_int32), ("x0", C.c_double), ("y0", C.c_double),
+                ("width", C.c_double), ("q", C.c_double), ("bx", C.c_double),
+                ("by", C.c_double), ("amp", C.POINTER(C.c_double))]
+
+
+class Result(C.Structure):
+    _fields_ = [("phi", C.c_double), ("ax", C.c_double), ("ay", C.c_double), ("err", C.c_double),
+                ("nseg", C.c_int32), ("nleaf", C.c_int32), ("capped", C.c_int32),
+                ("ties", C.c_int32), ("max_level", C.c_int32), ("pad", C.c_int32),
+                ("evals", C.c_int64), ("nodes", C.c_int64), ("min_margin", C.c_double)]
+
+
+_lib = None
+
+
+def lib():
+    global _lib
+    if _lib is None:
+        _lib = C.CDLL(build())
+        P = C.POINTER
+        d, i32, i64 = C.c_double, C.c_int32, C.c_int64
+        pd, pi32 = P(d), P(i32)
+        sig = {
+            "orc_gk15_constants": (None, [pd, pd, pd]),
+            "orc_tsc_weights": (None, [d, pd]),
+            "orc_lagrange3_weights": (None, [d, pd]),
+            "orc_bin_of": (i32, [d, d, P(Frame), d, d, i32, i32, pi32, pi32, pd, pd]),
+            "orc_deposit": (d, [i64, pd, pd, pd, pd, d, P(Frame), i32, i32, d, d, pd, pi32]),
+            "orc_arcs_rect": (i32, [d, d, d, d, d, d, d, pd]),
+            "orc_arcs_disk": (i32, [d, d, d, d, d, d, pd]),
+            "orc_kappa": (i32, [P(Params), P(Hist)]),
+            "orc_mesh_point": (None, [P(Params), P(Frame), i32, i32, pd, pd]),
+            "orc_point_lab": (None, [P(Params), P(Hist), P(Source), d, d, P(Result)]),
+            "orc_potentials": (None, [P(Params), P(Hist), P(Source), pi32, i32, P(Result)]),
+            "orc_clip_at": (i32, [P(Params), P(Hist), P(Source), d, d, i32, pd, pd]),
+            "orc_dists_at": (None, [P(Params), P(Hist), P(Source), d, d, i32, d, pd, pd]),
+            "orc_inner_at": (i64, [P(Params), P(Hist), P(Source), d, d, i32, d, pd]),
+            "orc_integrand_at": (None, [P(Params), P(Hist), P(Source), i32, d, d, d, pd]),
+            "orc_gk15_at": (None, [P(Params), P(Hist), P(Source), d, d, i32, d, d, pd, pd, pd]),
+            "orc_fields": (None, [P(Params), P(Frame), P(Frame), pd, pd, pd, pd, pd, pd, pd, pd]),
+            "orc_push": (None, [P(Params), P(Frame), i64, pd, pd, pd, pd, d, d, pd, pd, pd]),
+        }
+        for name, (res, args) in sig.items():
+            fn = getattr(_lib, name)
+            fn.restype = res
+            fn.argtypes = args
+    return _lib
+
+
+# ---------------------------------------------------------------- helpers
+def _pd(a):
+    if a is None:
+        return None
+    assert a.dtype == np.float64 and a.flags.c_contiguous
+    return a.ctypes.data_as(C.POINTER(C.c_double))
+
+
+def _pi(a):
+    assert a.dtype == np.int32 and a.flags.c_contiguous
+    return a.ctypes.data_as(C.POINTER(C.c_int32))
+
+
+def frame(f) -> Frame:
+    return Frame(*[float(v) for v in f])
+
+
+class Problem:
+    """Bundles (params, history, source) with the numpy buffers kept alive.
+
+    ``ring``: float64 [H, ny, nx, 4]; ``frames``: float64 [H, 4] (ox, oy, c, s);
+    ``amp``: optional float64 [H] amplitudes for analytic sources.
+    """
+
+    def __init__(self, *, nx, ny, hx, hy, c, dt, tau, kappa_max, k, n_pre,
+                 ring=None, frames=None, n_theta=64, max_depth=30, n_root=2,
+                 source=SRC_GRID, x0=0.0, y0=0.0, width=1.0, q=1.0, bx=0.0, by=0.0, amp=None):
+        H = kappa_max + 2
+        self.params = Params(nx, ny, hx, hy, c, dt, tau, n_theta, max_depth, n_root, kappa_max)
+        self.ring = None if ring is None else np.ascontiguousarray(ring, dtype=np.float64)
+        if self.ring is not None:
+            assert self.ring.shape == (H, ny, nx, 4), self.ring.shape
+        fr = np.zeros((H, 4)) if frames is None else np.asarray(frames, dtype=np.float64)
+        if frames is None:
+            fr[:, 2] = 1.0
+        self.frames_np = np.ascontiguousarray(fr)
+        assert self.frames_np.shape == (H, 4)
+        self.frames = (Frame * H)(*[Frame(*row) for row in self.frames_np])
+        self.amp = None if amp is None else np.ascontiguousarray(amp, dtype=np.float64)
+        self.hist = Hist(_pd(self.ring) if self.ring is not None else None,
+                         C.cast(self.frames, C.POINTER(Frame)), H, k, n_pre)
+        self.source = Source(source, x0, y0, width, q, bx, by,
+                             _pd(self.amp) if self.amp is not None else None)
+
+    # -------------------------------------------------------------- calls
+    def kappa(self) -> int:
+        return lib().orc_kappa(C.byref(self.params), C.byref(self.hist))
+
+    def mesh_point(self, ix, iy):
+        px, py = C.c_double(), C.c_double()
+        H = self.hist.H
+        lib().orc_mesh_point(C.byref(self.params), C.byref(self.frames[self.hist.k % H]),
+                             ix, iy, C.byref(px), C.byref(py))
+        return px.value, py.value
+
+    def point_lab(self, px, py) -> Result:
+        r = Result()
+        lib().orc_point_lab(C.byref(self.params), C.byref(self.hist), C.byref(self.source),
+                            px, py, C.byref(r))
+        return r
+
+    def potentials(self, pts) -> np.ndarray:
+        """Potentials at flattened mesh points; returns a structured array."""
+        pts = np.ascontiguousarray(pts, dtype=np.int32)
+        out = (Result * len(pts))()
+        lib().orc_potentials(C.byref(self.params), C.byref(self.hist), C.byref(self.source),
+                             _pi(pts), len(pts), out)
+        return np.ctypeslib.as_array(out).copy() if len(pts) else np.zeros(0)
+
+    def clip(self, px, py, j):
+        A, B = C.c_double(), C.c_double()
+        ok = lib().orc_clip_at(C.byref(self.params), C.byref(self.hist), C.byref(self.source),
+                               px, py, j, C.byref(A), C.byref(B))
+        return (A.value, B.value) if ok else None
+
+    def dists(self, px, py, j, r):
+        a, b = C.c_double(), C.c_double()
+        lib().orc_dists_at(C.byref(self.params), C.byref(self.hist), C.byref(self.source),
+                           px, py, j, r, C.byref(a), C.byref(b))
+        return a.value, b.value
+
+    def inner(self, px, py, j, r):
+        out = np.zeros(3)
+        n = lib().orc_inner_at(C.byref(self.params), C.byref(self.hist), C.byref(self.source),
+                               px, py, j, r, _pd(out))
+        return out, n
+
+    def integrand(self, j, u, v, tau_t):
+        out = np.zeros(3)
+        lib().orc_integrand_at(C.byref(self.params), C.byref(self.hist), C.byref(self.source),
+                               j, u, v, tau_t, _pd(out))
+        return out
+
+    def gk15(self, px, py, j, a, b):
+        K, G, e = np.zeros(3), np.zeros(3), C.c_double()
+        lib().orc_gk15_at(C.byref(self.params), C.byref(self.hist), C.byref(self.source),
+                          px, py, j, a, b, _pd(K), _pd(G), C.byref(e))
+        return K, G, e.value
+
+
+# ---------------------------------------------------------------- free functions
+def gk15_constants():
+    x, wk, wg = np.zeros(8), np.zeros(8), np.zeros(4)
+    lib().orc_gk15_constants(_pd(x), _pd(wk), _pd(wg))
+    return x, wk, wg
+
+
+def tsc_weights(d):
+    w = np.zeros(3)
+    lib().orc_tsc_weights(float(d), _pd(w))
+    return w
+
+
+def lagrange3_weights(t):
+    w = np.zeros(3)
+    lib().orc_lagrange3_weights(float(t), _pd(w))
+    return w
+
+
+def bin_of(x, y, fr, hx, hy, nx, ny):
+    ix, iy, dx, dy = C.c_int32(), C.c_int32(), C.c_double(), C.c_double()
+    b = lib().orc_bin_of(x, y, C.byref(frame(fr)), hx, hy, nx, ny, C.byref(ix), C.byref(iy),
+                         C.byref(dx), C.byref(dy))
+    return b, ix.value, iy.value, dx.value, dy.value
+
+
+def deposit(x, y, ux, uy, q, fr, nx, ny, hx, hy):
+    """Returns (M [ny,nx,4], bins int32[n], q_lost)."""
+    x, y, ux, uy = (np.ascontiguousarray(a, dtype=np.float64) for a in (x, y, ux, uy))
+    M = np.zeros((ny, nx, 4))
+    bins = np.zeros(len(x), dtype=np.int32)
+    ql = lib().orc_deposit(len(x), _pd(x), _pd(y), _pd(ux), _pd(uy), q, C.byref(frame(fr)),
+                           nx, ny, hx, hy, _pd(M), _pi(bins))
+    return M, bins, ql
+
+
+def arcs_rect(cu, cv, r, U0, U1, V0, V1):
+    out = np.zeros(16)
+    n = lib().orc_arcs_rect(cu, cv, r, U0, U1, V0, V1, _pd(out))
+    return n, out[: 2 * max(n, 0)].reshape(-1, 2)
+
+
+def arcs_disk(cu, cv, r, x0, y0, a):
+    out = np.zeros(16)
+    n = lib().orc_arcs_disk(cu, cv, r, x0, y0, a, _pd(out))
+    return n, out[: 2 * max(n, 0)].reshape(-1, 2)
+
+
+def fields(nx, ny, hx, hy, c, dt, fk, fkm1, phi, ax, ay, ax_prev=None, ay_prev=None):
+    P = Params(nx, ny, hx, hy, c, dt, 1.0, 64, 30, 2, 1)
+    phi, ax, ay = (np.ascontiguousarray(a, dtype=np.float64) for a in (phi, ax, ay))
+    if ax_prev is not None:
+        ax_prev = np.ascontiguousarray(ax_prev, dtype=np.float64)
+        ay_prev = np.ascontiguousarray(ay_prev, dtype=np.float64)
+    ex, ey, bz = np.zeros_like(phi), np.zeros_like(phi), np.zeros_like(phi)
+    fm = C.byref(frame(fkm1)) if fkm1 is not None else None
+    lib().orc_fields(C.byref(P), C.byref(frame(fk)), fm, _pd(phi), _pd(ax), _pd(ay),
+                     _pd(ax_prev), _pd(ay_prev), _pd(ex), _pd(ey), _pd(bz))
+    return ex, ey, bz
+
+
+def push(nx, ny, hx, hy, c, dt, fk, x, y, ux, uy, q_over_mc, bz_ext, ex, ey, bz):
+    """In-place Boris push on copies; returns (x, y, ux, uy)."""
+    P = Params(nx, ny, hx, hy, c, dt, 1.0, 64, 30, 2, 1)
+    x, y, ux, uy = (np.array(a, dtype=np.float64, copy=True) for a in (x, y, ux, uy))
+    ex, ey, bz = (np.ascontiguousarray(a, dtype=np.float64) for a in (ex, ey, bz))
+    lib().orc_push(C.byref(P), C.byref(frame(fk)), len(x), _pd(x), _pd(y), _pd(ux), _pd(uy),
+                   q_over_mc, bz_ext, _pd(ex), _pd(ey), _pd(bz))
+    return x, y, ux, uy

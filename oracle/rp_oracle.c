@@ -1,0 +1,727 @@
+/*
+ * rp_oracle.c -- CPU ORACLE for the retarded-potential step of
+ *   Arumugam, Godunov, Islam, Ranjan, Terzic, Zubair,
+ *   "A Machine Learning Approach for Efficient Parallel Simulation of Beam
+ *    Dynamics on GPUs", ICPP'17  (PAPER.md = /root/reference/PAPER.md).
+ *
+ * TEST INFRASTRUCTURE ONLY.  Only tests/, __graft_entry__.smoke() and the
+ * cpu_baseline / --impl reference legs of bench.py may load this library.
+ * The product path (paper_conf_icpp_arumugamrztgi17_b200/) never links,
+ * imports or calls it, and this file includes nothing from the product.
+ *
+ * Plain, slow, obviously-correct FP64.  Compiled with -O2 -ffp-contract=off
+ * (no FMA contraction), one OpenMP "parallel for schedule(dynamic)" over mesh
+ * points and nothing else clever.  Every function cites the PAPER.md line
+ * (P:NN) it follows, or the DESIGN.md "reading" (R-n) that fills a gap in the
+ * paper (the paper's integral limits, inner rule and stencil live in its
+ * absent references [9], [14]).
+ *
+ * Pins (tests/test_oracle_*.py, -m "not gpu"): GK15 monomial exactness,
+ * TSC / Lagrange weight identities, arcs vs dense theta sampling, clip vs a
+ * brute r' scan, Gaussian and uniform-disk closed forms (static and with a
+ * quadratic-in-time amplitude), brute-force Gauss-Legendre outer integral,
+ * Cartesian fine-cell sum, deposit charge conservation and J = rho*beta,
+ * (M, tau) -> (2M, 2tau) scaling, J = 0 => A = 0, FD exactness on
+ * quadratics, Boris |u| conservation and gyration radius, steady-state
+ * stationarity in the bend.
+ * "parity unpinned": none of the exported functions.
+ */
+#include <math.h>
+#include <stdint.h>
+#include <stdlib.h>
+#include <string.h>
+
+#ifndef M_PI
+#define M_PI 3.14159265358979323846
+#endif
+
+/* ------------------------------------------------------------------ */
+/* Types (mirrored by oracle/__init__.py with ctypes)                  */
+/* ------------------------------------------------------------------ */
+typedef struct { double ox, oy, c, s; } orc_frame; /* lab = O + u(c,s) + v(-s,c) */
+
+typedef struct {
+  int32_t nx, ny;
+  double hx, hy;
+  double c, dt;      /* subregion width c*dt                         */
+  double tau;        /* absolute tolerance per component (1e-6)      */
+  int32_t n_theta;   /* inner panels per arc (R-11)                          */
+  int32_t max_depth; /* bisection cap (R-12)                                 */
+  int32_t n_root;    /* 2: start from both halves of [A,B]; 1: from [A,B]   */
+  int32_t kappa_max; /* history depth (R-4)                                  */
+} orc_params;
+
+typedef struct {
+  const double* ring;      /* [H][ny][nx][4]: rho, rho*beta_x, rho*beta_y, 0 */
+  const orc_frame* frames; /* [H]                                            */
+  int32_t H;               /* ring slots = kappa_max + 2                      */
+  int32_t k;               /* current step                                    */
+  int32_t n_pre;           /* number of pre-history levels l = -1..-n_pre     */
+} orc_hist;
+
+enum { ORC_SRC_GRID = 0, ORC_SRC_GAUSS = 1, ORC_SRC_DISK = 2 };
+typedef struct {
+  int32_t kind;       /* ORC_SRC_*                                                */
+  double x0, y0;      /* analytic source centre, frame-local coordinates          */
+  double width;       /* gauss: sigma ; disk: radius a                           */
+  double q;           /* gauss: total charge Q ; disk: surface density sigma_s   */
+  double bx, by;      /* analytic source: beta (current = rho * beta)            */
+  const double* amp;  /* analytic source: amplitude per ring slot [H] (NULL = 1)  */
+} orc_source;
+
+typedef struct {
+  double phi, ax, ay, err;      /* I_rho, I_{rho bx}, I_{rho by}, sum of leaf errors */
+  int32_t nseg, nleaf, capped, ties, max_level, pad;
+  int64_t evals;                /* integrand evaluations (flop census)                */
+  int64_t nodes;                /* r' nodes evaluated (15 per segment)                */
+  double min_margin;            /* min |err - tol| / tol over all decisions           */
+} orc_result;
+
+/* ------------------------------------------------------------------ */
+/* GK15 constants (QUADPACK qk15), the outer rule of R-8               */
+/* ------------------------------------------------------------------ */
+static const double XGK[8] = {
+    0.991455371120812639206854697526329, 0.949107912342758524526189684047851,
+    0.864864423359769072789712788640926, 0.741531185599394439863864773280788,
+    0.586087235467691130294144845693013, 0.405845151377397166906606412076961,
+    0.207784955007898467600689403773245, 0.000000000000000000000000000000000};
+static const double WGK[8] = {
+    0.022935322010529224963732008058970, 0.063092092629978553290700663189204,
+    0.104790010322250183839876322541518, 0.140653259715525918745189590510238,
+    0.169004726639267902826583426598550, 0.190350578064785409913256402421014,
+    0.204432940075298892414161999234649, 0.209482141084727828012999174891714};
+/* Gauss-7 weights on XGK[1], XGK[3], XGK[5], XGK[7] */
+static const double WG[4] = {
+    0.129484966168869693270611432679082, 0.279705391489276667901467771423780,
+    0.381830050505118944950369775488975, 0.417959183673469387755102040816327};
+
+void orc_gk15_constants(double* xgk, double* wgk, double* wg) {
+  for (int i = 0; i < 8; ++i) { xgk[i] = XGK[i]; wgk[i] = WGK[i]; }
+  for (int i = 0; i < 4; ++i) wg[i] = WG[i];
+}
+
+/* ------------------------------------------------------------------ */
+/* Weights                                                              */
+/* ------------------------------------------------------------------ */
+/* TSC (quadratic B-spline) weights for nodes -1, 0, +1 about the nearest
+ * node at offset delta in [-1/2, 1/2] (R-6: the "27 neighbouring points" of
+ * P:45 are 3x3 spatial TSC nodes x 3 time levels). */
+void orc_tsc_weights(double d, double* w) {
+  double a = 0.5 - d, b = 0.5 + d;
+  w[0] = 0.5 * (a * a);
+  w[1] = 0.75 - d * d;
+  w[2] = 0.5 * (b * b);
+}
+
+/* Quadratic Lagrange weights in time for levels (l0,l1,l2) = (k-j-2,k-j-1,k-j)
+ * at nodes tau = -1, 0, +1 (R-2). */
+void orc_lagrange3_weights(double t, double* w) {
+  w[0] = 0.5 * t * (t - 1.0);
+  w[1] = 1.0 - t * t;
+  w[2] = 0.5 * t * (t + 1.0);
+}
+
+/* ------------------------------------------------------------------ */
+/* Binning and deposition (step 1 of the 4-step loop; R-14)       */
+/* ------------------------------------------------------------------ */
+static void to_local(const orc_frame* F, double x, double y, double* u, double* v) {
+  double dx = x - F->ox, dy = y - F->oy;
+  *u = F->c * dx + F->s * dy;
+  *v = F->c * dy - F->s * dx;
+}
+
+/* Nearest-node bin (R-13: round half up).  Returns iy*nx+ix, or -1 when the
+ * 3x3 stencil would leave the grid (particle lost). */
+int32_t orc_bin_of(double x, double y, const orc_frame* F, double hx, double hy,
+                   int32_t nx, int32_t ny, int32_t* ix_out, int32_t* iy_out,
+                   double* dx_out, double* dy_out) {
+  double u, v;
+  to_local(F, x, y, &u, &v);
+  double tx = u / hx, ty = v / hy;
+  double fx = floor(tx + 0.5), fy = floor(ty + 0.5);
+  double dx = tx - fx, dy = ty - fy;
+  int32_t ok = (fx >= 1.0 && fx <= (double)(nx - 2) && fy >= 1.0 && fy <= (double)(ny - 2));
+  int32_t ix = ok ? (int32_t)fx : -1, iy = ok ? (int32_t)fy : -1;
+  if (ix_out) *ix_out = ix;
+  if (iy_out) *iy_out = iy;
+  if (dx_out) *dx_out = dx;
+  if (dy_out) *dy_out = dy;
+  return ok ? iy * nx + ix : -1;
+}
+
+/* TSC deposit of n particles (x, y, ux, uy with u = gamma*beta) of charge q
+ * each onto M[ny][nx][4] (accumulated; caller zeroes).  Particle loop in
+ * index order.  Returns the lost charge. */
+double orc_deposit(int64_t n, const double* x, const double* y, const double* ux,
+                   const double* uy, double q, const orc_frame* F, int32_t nx,
+                   int32_t ny, double hx, double hy, double* M, int32_t* bins) {
+  double q_lost = 0.0;
+  for (int64_t i = 0; i < n; ++i) {
+    int32_t ix, iy;
+    double dx, dy;
+    int32_t b = orc_bin_of(x[i], y[i], F, hx, hy, nx, ny, &ix, &iy, &dx, &dy);
+    if (bins) bins[i] = b;
+    if (b < 0) { q_lost += q; continue; }
+    double g = sqrt(1.0 + ux[i] * ux[i] + uy[i] * uy[i]);
+    double bx = ux[i] / g, by = uy[i] / g;
+    double wx[3], wy[3];
+    orc_tsc_weights(dx, wx);
+    orc_tsc_weights(dy, wy);
+    for (int bb = 0; bb < 3; ++bb)
+      for (int aa = 0; aa < 3; ++aa) {
+        double w = q * wx[aa] * wy[bb] / (hx * hy);
+        double* m = M + 4 * ((int64_t)(iy + bb - 1) * nx + (ix + aa - 1));
+        m[0] += w;
+        m[1] += w * bx;
+        m[2] += w * by;
+      }
+  }
+  return q_lost;
+}
+
+/* ------------------------------------------------------------------ */
+/* History access ("stored linearly"; ring of H slots)            */
+/* ------------------------------------------------------------------ */
+static int32_t slot_of(int32_t level, int32_t H) { return ((level % H) + H) % H; }
+
+/* Frame at retarded time: quadratic Lagrange in time through the frames of
+ * levels l0,l1,l2 (R-7), written as X1 + w0 (X0-X1) + w2 (X2-X1) so that a
+ * static frame is returned exactly.  No renormalisation of (c, s). */
+static orc_frame frame_at(const orc_frame* F0, const orc_frame* F1, const orc_frame* F2,
+                          const double* w) {
+  orc_frame r;
+  r.ox = F1->ox + w[0] * (F0->ox - F1->ox) + w[2] * (F2->ox - F1->ox);
+  r.oy = F1->oy + w[0] * (F0->oy - F1->oy) + w[2] * (F2->oy - F1->oy);
+  r.c = F1->c + w[0] * (F0->c - F1->c) + w[2] * (F2->c - F1->c);
+  r.s = F1->s + w[0] * (F0->s - F1->s) + w[2] * (F2->s - F1->s);
+  return r;
+}
+
+/* ------------------------------------------------------------------ */
+/* Per-subregion context                                                */
+/* ------------------------------------------------------------------ */
+typedef struct {
+  const orc_params* P;
+  const orc_hist* Hh;
+  const orc_source* S;
+  double px, py;          /* mesh point, lab                                  */
+  int32_t j;              /* subregion index (S_j = [j c dt, (j+1) c dt])      */
+  const orc_frame* F[3];  /* frames of levels l0, l1, l2                       */
+  const double* G[3];     /* grids of levels l0, l1, l2                        */
+  double amp[3];          /* analytic amplitudes of the 3 levels               */
+  double U0, U1, V0, V1;  /* support rectangle (frame-local)                   */
+  int64_t evals;
+} subctx;
+
+/* tau_t(r') = (j+1) - r'/(c dt) in [0,1] on S_j (t' = k dt - r'/c). */
+static double tau_of(const subctx* X, double r) {
+  return (double)(X->j + 1) - r / (X->P->c * X->P->dt);
+}
+
+/* Local centre (c_u, c_v) of the circle about p at retarded time t'(r). */
+static void centre_at(const subctx* X, double r, double* cu, double* cv, double* w) {
+  orc_lagrange3_weights(tau_of(X, r), w);
+  orc_frame f = frame_at(X->F[0], X->F[1], X->F[2], w);
+  double dx = X->px - f.ox, dy = X->py - f.oy;
+  *cu = f.c * dx + f.s * dy;
+  *cv = -f.s * dx + f.c * dy;
+}
+
+/* squared distance from (cu,cv) to the support (0 inside), and squared
+ * distance to its farthest point (R-5: the limits of P:43). */
+static void support_dist2(const subctx* X, double cu, double cv, double* dmin2, double* dmax2) {
+  if (X->S->kind == ORC_SRC_DISK) {
+    double ex = cu - X->S->x0, ey = cv - X->S->y0;
+    double s = sqrt(ex * ex + ey * ey), a = X->S->width;
+    double lo = s - a > 0.0 ? s - a : 0.0, hi = s + a;
+    *dmin2 = lo * lo;
+    *dmax2 = hi * hi;
+    return;
+  }
+  double ex = 0.0, ey = 0.0;
+  if (cu < X->U0) ex = X->U0 - cu; else if (cu > X->U1) ex = cu - X->U1;
+  if (cv < X->V0) ey = X->V0 - cv; else if (cv > X->V1) ey = cv - X->V1;
+  *dmin2 = ex * ex + ey * ey;
+  double fx = fabs(cu - X->U0) > fabs(cu - X->U1) ? fabs(cu - X->U0) : fabs(cu - X->U1);
+  double fy = fabs(cv - X->V0) > fabs(cv - X->V1) ? fabs(cv - X->V0) : fabs(cv - X->V1);
+  *dmax2 = fx * fx + fy * fy;
+}
+
+static void dists_at(const subctx* X, double r, double* dmin2, double* dmax2) {
+  double cu, cv, w[3];
+  centre_at(X, r, &cu, &cv, w);
+  support_dist2(X, cu, cv, dmin2, dmax2);
+}
+
+/* Support clip of S_j (R-5): [A,B] = {r in S_j :
+ * d_min(r) <= r <= d_max(r)}, by 64-step bisection on squares.  Returns 0
+ * when the subregion has no support. */
+int32_t orc_clip(const subctx* X, double a, double b, double* A, double* B) {
+  double dmn, dmx;
+  dists_at(X, b, &dmn, &dmx);
+  if (dmn > b * b) return 0;
+  dists_at(X, a, &dmn, &dmx);
+  if (dmx < a * a) return 0;
+  /* lower end */
+  dists_at(X, a, &dmn, &dmx);
+  if (dmn <= a * a) {
+    *A = a;
+  } else {
+    double lo = a, hi = b;
+    for (int it = 0; it < 64; ++it) {
+      double m = 0.5 * (lo + hi);
+      dists_at(X, m, &dmn, &dmx);
+      if (dmn <= m * m) hi = m; else lo = m;
+    }
+    *A = hi;
+  }
+  /* upper end */
+  dists_at(X, b, &dmn, &dmx);
+  if (dmx >= b * b) {
+    *B = b;
+  } else {
+    double lo = a, hi = b;
+    for (int it = 0; it < 64; ++it) {
+      double m = 0.5 * (lo + hi);
+      dists_at(X, m, &dmn, &dmx);
+      if (dmx >= m * m) lo = m; else hi = m;
+    }
+    *B = lo;
+  }
+  return (*A < *B) ? 1 : 0;
+}
+
+/* ------------------------------------------------------------------ */
+/* Arcs of circle (cu,cv; r) inside a rectangle (R-5, C.3e)             */
+/* ------------------------------------------------------------------ */
+static int inside_rect(double u, double v, double U0, double U1, double V0, double V1) {
+  return u >= U0 && u <= U1 && v >= V0 && v <= V1;
+}
+
+static int cmp_double(const void* a, const void* b) {
+  double x = *(const double*)a, y = *(const double*)b;
+  return (x > y) - (x < y);
+}
+
+/* Writes up to 8 arcs as pairs (t1, t2) with t1 < t2 (t2 may exceed 2 pi for
+ * the wrap-around arc).  Returns the number of arcs, or -1 for the full
+ * circle. */
+int32_t orc_arcs_rect(double cu, double cv, double r, double U0, double U1, double V0,
+                      double V1, double* arcs) {
+  double t[8];
+  int n = 0;
+  const double twopi = 2.0 * M_PI;
+  double E[2] = {U0, U1};
+  for (int e = 0; e < 2; ++e) { /* vertical edges u = E[e] */
+    double d = (E[e] - cu) / r;
+    if (fabs(d) < 1.0) {
+      double al = acos(d);
+      double c1 = al, c2 = twopi - al;
+      double v1 = cv + r * sin(c1), v2 = cv + r * sin(c2);
+      if (v1 >= V0 && v1 <= V1) t[n++] = c1;
+      if (v2 >= V0 && v2 <= V1) t[n++] = c2;
+    }
+  }
+  double Fv[2] = {V0, V1};
+  for (int e = 0; e < 2; ++e) { /* horizontal edges v = Fv[e] */
+    double d = (Fv[e] - cv) / r;
+    if (fabs(d) < 1.0) {
+      double be = asin(d);
+      double c1 = be < 0.0 ? be + twopi : be, c2 = M_PI - be;
+      double u1 = cu + r * cos(c1), u2 = cu + r * cos(c2);
+      if (u1 >= U0 && u1 <= U1) t[n++] = c1;
+      if (u2 >= U0 && u2 <= U1) t[n++] = c2;
+    }
+  }
+  if (n == 0) return inside_rect(cu + r, cv, U0, U1, V0, V1) ? -1 : 0;
+  qsort(t, (size_t)n, sizeof(double), cmp_double);
+  int m = 0; /* merge exact duplicates */
+  for (int i = 0; i < n; ++i)
+    if (m == 0 || t[i] != t[m - 1]) t[m++] = t[i];
+  int na = 0;
+  for (int i = 0; i < m; ++i) {
+    double t1 = t[i], t2 = (i + 1 < m) ? t[i + 1] : t[0] + twopi;
+    double mid = 0.5 * (t1 + t2);
+    if (inside_rect(cu + r * cos(mid), cv + r * sin(mid), U0, U1, V0, V1)) {
+      arcs[2 * na] = t1;
+      arcs[2 * na + 1] = t2;
+      ++na;
+    }
+  }
+  return na;
+}
+
+/* Arc of circle (cu,cv; r) inside the disk (x0,y0; a).  Same return
+ * convention as orc_arcs_rect (test-only analytic source, C.4). */
+int32_t orc_arcs_disk(double cu, double cv, double r, double x0, double y0, double a,
+                      double* arcs) {
+  double ex = x0 - cu, ey = y0 - cv;
+  double s = sqrt(ex * ex + ey * ey);
+  if (s + r <= a) return -1;
+  if (r >= s + a || s >= r + a) return 0;
+  double ph = atan2(ey, ex);
+  double al = acos((r * r + s * s - a * a) / (2.0 * r * s));
+  arcs[0] = ph - al;
+  arcs[1] = ph + al;
+  return 1;
+}
+
+/* ------------------------------------------------------------------ */
+/* Integrand f^(p)(r', theta', t') (R-1, R-6, R-7)                 */
+/* ------------------------------------------------------------------ */
+/* TSC interpolation of one level at frame-local (u,v); out-of-range nodes 0. */
+static void grid_interp(const orc_params* P, const double* G, int32_t ix, int32_t iy,
+                        const double* wx, const double* wy, double* out) {
+  out[0] = out[1] = out[2] = 0.0;
+  for (int b = 0; b < 3; ++b) {
+    int32_t yy = iy + b - 1;
+    if (yy < 0 || yy >= P->ny) continue;
+    for (int a = 0; a < 3; ++a) {
+      int32_t xx = ix + a - 1;
+      if (xx < 0 || xx >= P->nx) continue;
+      const double* m = G + 4 * ((int64_t)yy * P->nx + xx);
+      double w = wx[a] * wy[b];
+      out[0] += w * m[0];
+      out[1] += w * m[1];
+      out[2] += w * m[2];
+    }
+  }
+}
+
+/* f at frame-local (u, v) and time weights wt[3] of levels (l0,l1,l2). */
+static void integrand(const subctx* X, double u, double v, const double* wt, double* f) {
+  const orc_source* S = X->S;
+  if (S->kind == ORC_SRC_GRID) {
+    const orc_params* P = X->P;
+    double tx = u / P->hx, ty = v / P->hy;
+    double fx = floor(tx + 0.5), fy = floor(ty + 0.5);
+    double wx[3], wy[3];
+    orc_tsc_weights(tx - fx, wx);
+    orc_tsc_weights(ty - fy, wy);
+    /* clamp far-out indices before the int conversion (values are 0 there) */
+    if (fx < -4.0 || fx > P->nx + 4.0 || fy < -4.0 || fy > P->ny + 4.0) {
+      f[0] = f[1] = f[2] = 0.0;
+      return;
+    }
+    int32_t ix = (int32_t)fx, iy = (int32_t)fy;
+    double g[3][3];
+    for (int l = 0; l < 3; ++l) grid_interp(P, X->G[l], ix, iy, wx, wy, g[l]);
+    for (int c = 0; c < 3; ++c) f[c] = wt[0] * g[0][c] + wt[1] * g[1][c] + wt[2] * g[2][c];
+    return;
+  }
+  double a = wt[0] * X->amp[0] + wt[1] * X->amp[1] + wt[2] * X->amp[2];
+  double rho;
+  if (S->kind == ORC_SRC_GAUSS) {
+    double ex = u - S->x0, ey = v - S->y0, sg = S->width;
+    rho = S->q / (2.0 * M_PI * sg * sg) * exp(-(ex * ex + ey * ey) / (2.0 * sg * sg));
+  } else {
+    rho = S->q; /* uniform disk, the arc lies inside it */
+  }
+  rho = a * rho;
+  f[0] = rho;
+  f[1] = rho * S->bx;
+  f[2] = rho * S->by;
+}
+
+/* Inner theta integral at radius r ("Newton-Cotes"; R-11): periodic
+ * trapezoid on a full circle, composite Simpson with n_theta panels per arc. */
+void orc_inner_ctx(subctx* X, double r, double* out) {
+  double cu, cv, wt[3];
+  centre_at(X, r, &cu, &cv, wt);
+  double arcs[16];
+  int32_t na;
+  if (X->S->kind == ORC_SRC_DISK)
+    na = orc_arcs_disk(cu, cv, r, X->S->x0, X->S->y0, X->S->width, arcs);
+  else
+    na = orc_arcs_rect(cu, cv, r, X->U0, X->U1, X->V0, X->V1, arcs);
+  out[0] = out[1] = out[2] = 0.0;
+  const int32_t N = X->P->n_theta;
+  double f[3];
+  if (na < 0) {
+    double w = 2.0 * M_PI / N;
+    for (int32_t m = 0; m < N; ++m) {
+      double th = (double)m * (2.0 * M_PI / N);
+      integrand(X, cu + r * cos(th), cv + r * sin(th), wt, f);
+      X->evals++;
+      for (int c = 0; c < 3; ++c) out[c] += w * f[c];
+    }
+    return;
+  }
+  for (int32_t q = 0; q < na; ++q) {
+    double t1 = arcs[2 * q], t2 = arcs[2 * q + 1];
+    double h = (t2 - t1) / N;
+    for (int32_t m = 0; m <= N; ++m) {
+      double th = t1 + (double)m * h;
+      double w = (m == 0 || m == N) ? h / 3.0 : ((m & 1) ? 4.0 * h / 3.0 : 2.0 * h / 3.0);
+      integrand(X, cu + r * cos(th), cv + r * sin(th), wt, f);
+      X->evals++;
+      for (int c = 0; c < 3; ++c) out[c] += w * f[c];
+    }
+  }
+}
+
+/* ------------------------------------------------------------------ */
+/* GK15 on one segment and the dyadic adaptive tree (*/
+/* R-8, R-9, R-10, R-12, R-12b)                                          */
+/* ------------------------------------------------------------------ */
+static void gk15(subctx* X, double a, double b, double* K, double* G, double* err) {
+  double m = 0.5 * (a + b), hw = 0.5 * (b - a);
+  double k[3] = {0, 0, 0}, g[3] = {0, 0, 0}, v[3];
+  for (int i = 0; i < 7; ++i) {
+    orc_inner_ctx(X, m - hw * XGK[i], v);
+    for (int c = 0; c < 3; ++c) k[c] += WGK[i] * v[c];
+    if (i & 1) for (int c = 0; c < 3; ++c) g[c] += WG[i / 2] * v[c];
+    orc_inner_ctx(X, m + hw * XGK[i], v);
+    for (int c = 0; c < 3; ++c) k[c] += WGK[i] * v[c];
+    if (i & 1) for (int c = 0; c < 3; ++c) g[c] += WG[i / 2] * v[c];
+  }
+  orc_inner_ctx(X, m, v);
+  for (int c = 0; c < 3; ++c) { k[c] += WGK[7] * v[c]; g[c] += WG[3] * v[c]; }
+  *err = 0.0;
+  for (int c = 0; c < 3; ++c) {
+    K[c] = hw * k[c];
+    G[c] = hw * g[c];
+    double e = fabs(K[c] - G[c]);
+    if (e > *err) *err = e;
+  }
+}
+
+/* depth-first, left to right: visit (level, index) on [A,B] */
+static void tree(subctx* X, double A, double B, double R, int32_t lev, int64_t idx,
+                 orc_result* res) {
+  const orc_params* P = X->P;
+  double fa = ldexp((double)idx, -lev), fb = ldexp((double)(idx + 1), -lev);
+  double a = A + (B - A) * fa, b = A + (B - A) * fb;
+  double K[3], G[3], err;
+  gk15(X, a, b, K, G, &err);
+  res->nseg++;
+  res->nodes += 15;
+  double tol = P->tau * ldexp(B - A, -lev) / R;
+  double margin = fabs(err - tol) / tol;
+  if (margin < res->min_margin) res->min_margin = margin;
+  if (margin < 1e-9) res->ties++;
+  if (lev > res->max_level) res->max_level = lev;
+  if (err <= tol || lev >= P->max_depth) {
+    if (!(err <= tol)) res->capped++;
+    res->nleaf++;
+    res->phi += K[0];
+    res->ax += K[1];
+    res->ay += K[2];
+    res->err += err;
+    return;
+  }
+  tree(X, A, B, R, lev + 1, 2 * idx, res);
+  tree(X, A, B, R, lev + 1, 2 * idx + 1, res);
+}
+
+/* ------------------------------------------------------------------ */
+/* rp-integral at one mesh point (Eq. 1-2; C.3)                 */
+/* ------------------------------------------------------------------ */
+int32_t orc_kappa(const orc_params* P, const orc_hist* Hh) {
+  int32_t kap = Hh->k + Hh->n_pre - 1;
+  if (kap > P->kappa_max) kap = P->kappa_max;
+  if (kap < 0) kap = 0;
+  return kap;
+}
+
+static void setup_sub(subctx* X, const orc_params* P, const orc_hist* Hh, const orc_source* S,
+                      double px, double py, int32_t j) {
+  memset(X, 0, sizeof(*X));
+  X->P = P; X->Hh = Hh; X->S = S; X->px = px; X->py = py; X->j = j;
+  for (int l = 0; l < 3; ++l) {
+    int32_t level = Hh->k - j - 2 + l;
+    int32_t sl = slot_of(level, Hh->H);
+    X->F[l] = Hh->frames + sl;
+    X->G[l] = Hh->ring ? Hh->ring + (int64_t)sl * P->ny * P->nx * 4 : NULL;
+    X->amp[l] = S->amp ? S->amp[sl] : 1.0;
+  }
+  if (S->kind == ORC_SRC_GAUSS) {
+    X->U0 = S->x0 - 8.0 * S->width; X->U1 = S->x0 + 8.0 * S->width;
+    X->V0 = S->y0 - 8.0 * S->width; X->V1 = S->y0 + 8.0 * S->width;
+  } else {
+    X->U0 = -1.5 * P->hx; X->U1 = (P->nx + 0.5) * P->hx;
+    X->V0 = -1.5 * P->hy; X->V1 = (P->ny + 0.5) * P->hy;
+  }
+}
+
+/* Mesh node (ix,iy) of the frame of step k, in the lab. */
+void orc_mesh_point(const orc_params* P, const orc_frame* F, int32_t ix, int32_t iy,
+                    double* px, double* py) {
+  double u = ix * P->hx, v = iy * P->hy;
+  *px = F->ox + u * F->c - v * F->s;
+  *py = F->oy + u * F->s + v * F->c;
+}
+
+void orc_point_lab(const orc_params* P, const orc_hist* Hh, const orc_source* S, double px,
+                   double py, orc_result* res) {
+  memset(res, 0, sizeof(*res));
+  res->min_margin = INFINITY;
+  int32_t kap = orc_kappa(P, Hh);
+  if (kap == 0) return;
+  double cdt = P->c * P->dt;
+  double R = kap * cdt;
+  for (int32_t j = 0; j < kap; ++j) {
+    subctx X;
+    setup_sub(&X, P, Hh, S, px, py, j);
+    double A, B;
+    if (!orc_clip(&X, j * cdt, (j + 1) * cdt, &A, &B)) continue;
+    if (P->n_root == 1) {
+      tree(&X, A, B, R, 0, 0, res);
+    } else {
+      tree(&X, A, B, R, 1, 0, res);
+      tree(&X, A, B, R, 1, 1, res);
+    }
+    res->evals += X.evals;
+  }
+}
+
+/* Potentials at a list of mesh points (flattened iy*nx+ix) of frame k. */
+void orc_potentials(const orc_params* P, const orc_hist* Hh, const orc_source* S,
+                    const int32_t* pts, int32_t npts, orc_result* out) {
+  const orc_frame* Fk = Hh->frames + slot_of(Hh->k, Hh->H);
+#pragma omp parallel for schedule(dynamic, 1)
+  for (int32_t i = 0; i < npts; ++i) {
+    int32_t p = pts[i];
+    double px, py;
+    orc_mesh_point(P, Fk, p % P->nx, p / P->nx, &px, &py);
+    orc_point_lab(P, Hh, S, px, py, out + i);
+  }
+}
+
+/* Test hooks: the clip, inner integral and a single tree for (point, j). */
+int32_t orc_clip_at(const orc_params* P, const orc_hist* Hh, const orc_source* S, double px,
+                    double py, int32_t j, double* A, double* B) {
+  subctx X;
+  setup_sub(&X, P, Hh, S, px, py, j);
+  double cdt = P->c * P->dt;
+  return orc_clip(&X, j * cdt, (j + 1) * cdt, A, B);
+}
+
+void orc_dists_at(const orc_params* P, const orc_hist* Hh, const orc_source* S, double px,
+                  double py, int32_t j, double r, double* dmin2, double* dmax2) {
+  subctx X;
+  setup_sub(&X, P, Hh, S, px, py, j);
+  dists_at(&X, r, dmin2, dmax2);
+}
+
+int64_t orc_inner_at(const orc_params* P, const orc_hist* Hh, const orc_source* S, double px,
+                     double py, int32_t j, double r, double* out) {
+  subctx X;
+  setup_sub(&X, P, Hh, S, px, py, j);
+  orc_inner_ctx(&X, r, out);
+  return X.evals;
+}
+
+void orc_integrand_at(const orc_params* P, const orc_hist* Hh, const orc_source* S,
+                      int32_t j, double u, double v, double tau_t, double* f) {
+  subctx X;
+  setup_sub(&X, P, Hh, S, 0.0, 0.0, j);
+  double wt[3];
+  orc_lagrange3_weights(tau_t, wt);
+  integrand(&X, u, v, wt, f);
+}
+
+void orc_gk15_at(const orc_params* P, const orc_hist* Hh, const orc_source* S, double px,
+                 double py, int32_t j, double a, double b, double* K, double* G, double* err) {
+  subctx X;
+  setup_sub(&X, P, Hh, S, px, py, j);
+  gk15(&X, a, b, K, G, err);
+}
+
+/* ------------------------------------------------------------------ */
+/* Self-fields (R-15)                                  */
+/* ------------------------------------------------------------------ */
+static double d_dir(const double* f, int32_t nx, int32_t ny, int32_t ix, int32_t iy, int dir,
+                    double h) {
+  int32_t n = dir == 0 ? nx : ny, i = dir == 0 ? ix : iy;
+#define AT(o) (dir == 0 ? f[(int64_t)iy * nx + (ix + (o))] : f[(int64_t)(iy + (o)) * nx + ix])
+  if (i == 0) return (-3.0 * AT(0) + 4.0 * AT(1) - AT(2)) / (2.0 * h);
+  if (i == n - 1) return (3.0 * AT(0) - 4.0 * AT(-1) + AT(-2)) / (2.0 * h);
+  return (AT(1) - AT(-1)) / (2.0 * h);
+#undef AT
+}
+
+/* E = -grad(phi) - (1/c) dA/dt ,  B_z = d_x A_y - d_y A_x  on mesh k.
+ * dA/dt|lab = (A_k - A_{k-1})/dt - (V . grad) A_k with V the node velocity
+ * (P_k - P_{k-1})/dt; omitted when ax_prev/ay_prev are NULL. */
+void orc_fields(const orc_params* P, const orc_frame* Fk, const orc_frame* Fkm1,
+                const double* phi, const double* ax, const double* ay, const double* ax_prev,
+                const double* ay_prev, double* ex, double* ey, double* bz) {
+  const int32_t nx = P->nx, ny = P->ny;
+  for (int32_t iy = 0; iy < ny; ++iy)
+    for (int32_t ix = 0; ix < nx; ++ix) {
+      int64_t id = (int64_t)iy * nx + ix;
+      double c = Fk->c, s = Fk->s;
+      double pu = d_dir(phi, nx, ny, ix, iy, 0, P->hx), pv = d_dir(phi, nx, ny, ix, iy, 1, P->hy);
+      double xu = d_dir(ax, nx, ny, ix, iy, 0, P->hx), xv = d_dir(ax, nx, ny, ix, iy, 1, P->hy);
+      double yu = d_dir(ay, nx, ny, ix, iy, 0, P->hx), yv = d_dir(ay, nx, ny, ix, iy, 1, P->hy);
+      double phx = c * pu - s * pv, phy = s * pu + c * pv;
+      double axx = c * xu - s * xv, axy = s * xu + c * xv; /* d_x A_x, d_y A_x */
+      double ayx = c * yu - s * yv, ayy = s * yu + c * yv; /* d_x A_y, d_y A_y */
+      double dax = 0.0, day = 0.0;
+      if (ax_prev && ay_prev && Fkm1) {
+        double pxk, pyk, pxm, pym;
+        orc_mesh_point(P, Fk, ix, iy, &pxk, &pyk);
+        orc_mesh_point(P, Fkm1, ix, iy, &pxm, &pym);
+        double vx = (pxk - pxm) / P->dt, vy = (pyk - pym) / P->dt;
+        dax = (ax[id] - ax_prev[id]) / P->dt - (vx * axx + vy * axy);
+        day = (ay[id] - ay_prev[id]) / P->dt - (vx * ayx + vy * ayy);
+      }
+      ex[id] = -phx - dax / P->c;
+      ey[id] = -phy - day / P->c;
+      bz[id] = ayx - axy;
+    }
+}
+
+/* ------------------------------------------------------------------ */
+/* Push (P:60 leap-frog Lorentz; R-15): relativistic Boris   */
+/* ------------------------------------------------------------------ */
+static double gather_tsc(const orc_params* P, const double* F, int32_t ix, int32_t iy,
+                         const double* wx, const double* wy) {
+  double s = 0.0;
+  for (int b = 0; b < 3; ++b) {
+    int32_t yy = iy + b - 1;
+    if (yy < 0 || yy >= P->ny) continue;
+    for (int a = 0; a < 3; ++a) {
+      int32_t xx = ix + a - 1;
+      if (xx < 0 || xx >= P->nx) continue;
+      s += wx[a] * wy[b] * F[(int64_t)yy * P->nx + xx];
+    }
+  }
+  return s;
+}
+
+void orc_push(const orc_params* P, const orc_frame* Fk, int64_t n, double* x, double* y,
+              double* ux, double* uy, double q_over_mc, double bz_ext, const double* ex,
+              const double* ey, const double* bz) {
+  for (int64_t i = 0; i < n; ++i) {
+    double u, v;
+    to_local(Fk, x[i], y[i], &u, &v);
+    double tx = u / P->hx, ty = v / P->hy;
+    double fx = floor(tx + 0.5), fy = floor(ty + 0.5);
+    double Ex = 0.0, Ey = 0.0, Bz = 0.0;
+    if (fx >= -2.0 && fx <= P->nx + 1.0 && fy >= -2.0 && fy <= P->ny + 1.0) {
+      double wx[3], wy[3];
+      orc_tsc_weights(tx - fx, wx);
+      orc_tsc_weights(ty - fy, wy);
+      int32_t ix = (int32_t)fx, iy = (int32_t)fy;
+      Ex = gather_tsc(P, ex, ix, iy, wx, wy);
+      Ey = gather_tsc(P, ey, ix, iy, wx, wy);
+      Bz = gather_tsc(P, bz, ix, iy, wx, wy);
+    }
+    Bz += bz_ext;
+    double h = 0.5 * q_over_mc * P->dt;
+    double umx = ux[i] + h * Ex, umy = uy[i] + h * Ey;
+    double gm = sqrt(1.0 + umx * umx + umy * umy);
+    double t = h * Bz / gm;
+    double sr = 2.0 * t / (1.0 + t * t);
+    double upx = umx + umy * t, upy = umy - umx * t;
+    double ppx = umx + upy * sr, ppy = umy - upx * sr;
+    double nux = ppx + h * Ex, nuy = ppy + h * Ey;
+    double g = sqrt(1.0 + nux * nux + nuy * nuy);
+    ux[i] = nux;
+    uy[i] = nuy;
+    x[i] += P->c * P->dt * nux / g;
+    y[i] += P->c * P->dt * nuy / g;
+  }
+}

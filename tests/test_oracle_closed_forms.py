@@ -1,0 +1,173 @@
+"""Pins of the whole oracle rp-integral (Eq. 1-2) against
+closed forms and brute-force quadrature.
+
+* Static Gaussian sheet: phi(s) = (Q/sigma) sqrt(pi/2) i0e(s^2 / 4 sigma^2).
+* Uniform disk: phi(s<a) = 4 sigma_s a E(s/a), phi(s>a) = 4 sigma_s s [E(a/s) - (1-a^2/s^2) K(a/s)]
+  (modulus convention; scipy takes m = k^2).
+* Gaussian with an amplitude quadratic in time: pins the subregion -> history-level
+  mapping of P:76 (reading R-2) and the retarded time t' = k dt - r'/c of P:43:
+  phi = int_0^R amp(t_k - r/c) (Q/sigma^2) exp(-(r-s)^2/2sigma^2) i0e(rs/sigma^2) dr.
+* Grid path, outer integral: a piecewise 32-point Gauss-Legendre brute force with breakpoints
+  at subregion ends and the geometric kinks agrees with the adaptive tree within tau.
+* Grid path, polar transform + arcs + inner rule: a Cartesian fine-cell sum of
+  rho/|x - p| (singular cell analytic) agrees to its discretisation error.
+"""
+import math
+
+import numpy as np
+import pytest
+import scipy.integrate as si
+import scipy.special as sp
+
+import oracle
+import workloads as W
+
+SQ = math.sqrt(math.pi / 2)
+
+
+def gauss_problem(kap=12, cdt=1.6, k=20, tau=1e-6 * SQ, amp=None, beta=(0.0, 0.0), n_root=2):
+    return oracle.Problem(nx=8, ny=8, hx=1.0, hy=1.0, c=1.0, dt=cdt, tau=tau, kappa_max=kap, k=k,
+                          n_pre=0, source=oracle.SRC_GAUSS, x0=0.0, y0=0.0, width=1.0, q=1.0,
+                          bx=beta[0], by=beta[1], amp=amp, n_root=n_root)
+
+
+@pytest.mark.parametrize("s", [0.0, 0.5, 1.0, 2.0, 4.0, 6.5])
+def test_static_gaussian_closed_form(s):
+    P = gauss_problem(beta=(0.3, -0.2))
+    r = P.point_lab(s * math.cos(0.4), s * math.sin(0.4))
+    exact = SQ * sp.i0e(s * s / 4)
+    assert abs(r.phi - exact) < 1e-6 * SQ
+    assert abs(r.phi - exact) < 1e-13  # the tree is far inside tau on a smooth source
+    # A = beta * phi for a rigid current (same integrand times a constant)
+    assert abs(r.ax - 0.3 * r.phi) < 1e-15 and abs(r.ay + 0.2 * r.phi) < 1e-15
+    assert r.capped == 0 and r.ties == 0
+
+
+@pytest.mark.parametrize("s", [0.0, 0.3, 0.99, 1.0, 1.7, 4.0])
+def test_uniform_disk_closed_form(s):
+    a, ss = 1.0, 1.0
+    P = oracle.Problem(nx=8, ny=8, hx=1.0, hy=1.0, c=1.0, dt=0.6, tau=1e-6, kappa_max=12, k=20,
+                       n_pre=0, source=oracle.SRC_DISK, x0=0.0, y0=0.0, width=a, q=ss)
+    r = P.point_lab(0.0, s)
+    if s < a:
+        exact = 4 * ss * a * sp.ellipe((s / a) ** 2)
+    elif s == a:
+        exact = 4 * ss * a
+    else:
+        k = a / s
+        exact = 4 * ss * s * (sp.ellipe(k * k) - (1 - k * k) * sp.ellipk(k * k))
+    assert abs(r.phi - exact) < 1e-6
+    assert abs(r.phi - exact) < 1e-12
+    assert r.capped <= 1  # at most the sqrt-singular leaf at r' = a - s
+
+
+@pytest.mark.parametrize("s", [0.0, 1.5, 3.0])
+def test_time_dependent_amplitude_pins_level_mapping(s):
+    kap, cdt, k = 10, 1.3, 15
+    H = kap + 2
+    al, be, ga = 1.0, 0.05, -0.002
+    amp_t = lambda t: al + be * t + ga * t * t
+    amp = np.zeros(H)
+    for l in range(k - H + 1, k + 1):
+        amp[l % H] = amp_t(l * cdt)
+    P = gauss_problem(kap=kap, cdt=cdt, k=k, amp=amp, tau=1e-9)
+    r = P.point_lab(s, 0.0)
+    R = kap * cdt
+    tk = k * cdt
+    f = lambda rr: amp_t(tk - rr) * math.exp(-(rr - s) ** 2 / 2) * sp.i0e(rr * s)
+    exact, _ = si.quad(f, 0, R, epsabs=1e-14, epsrel=1e-13, limit=400, points=[s])
+    assert abs(r.phi - exact) < 1e-9 * 20
+    # a one-level shift of the mapping (P:46's D_{k-j-1..k-j-3}) would move phi by ~be*cdt*phi
+    shifted, _ = si.quad(lambda rr: amp_t(tk - cdt - rr) * math.exp(-(rr - s) ** 2 / 2) * sp.i0e(rr * s),
+                         0, R, epsabs=1e-14, limit=400, points=[s])
+    assert abs(shifted - exact) > 1e3 * abs(r.phi - exact)
+
+
+def _small_grid_problem(n=16, kap=10, cdt=1.6, tau=1e-6, n_root=2):
+    sig = 1.0
+    cfg = W.Config(number=0, name="t", nx=n, ny=n, n_particles=1, steps=1, kappa_max=kap,
+                   geometry="static", sigma=sig, cdt=cdt)
+    ring = W.node_gaussian_ring(cfg, k=30, beta=(0.2, 0.1))
+    fr = W.ring_frames(cfg, 30)
+    P = oracle.Problem(nx=n, ny=n, hx=cfg.hx, hy=cfg.hy, c=1.0, dt=cdt, tau=tau, kappa_max=kap,
+                       k=30, n_pre=0, ring=ring, frames=fr, n_root=n_root)
+    return cfg, P
+
+
+def _brute_outer(P, cfg, ix, iy, pieces=16):
+    """Piecewise 32-point Gauss-Legendre of inner(r) over [0, R] with breakpoints at
+    subregion ends and the static kinks (distances from p to Rect's edge lines / corners)."""
+    px, py = P.mesh_point(ix, iy)
+    fr = cfg.extent * 0.5
+    # p in frame-local coordinates (static frame: lower-left node at (-fr, -fr))
+    cu, cv = px + fr, py + fr
+    U0, U1 = -1.5 * cfg.hx, (cfg.nx + 0.5) * cfg.hx
+    V0, V1 = -1.5 * cfg.hy, (cfg.ny + 0.5) * cfg.hy
+    kinks = [abs(cu - U0), abs(cu - U1), abs(cv - V0), abs(cv - V1)]
+    kinks += [math.hypot(cu - a, cv - b) for a in (U0, U1) for b in (V0, V1)]
+    cdt = P.params.c * P.params.dt
+    kap = P.kappa()
+    gl_x, gl_w = np.polynomial.legendre.leggauss(32)
+    total = np.zeros(3)
+    for j in range(kap):
+        a, b = j * cdt, (j + 1) * cdt
+        bps = sorted({a, b, *[kk for kk in kinks if a < kk < b]})
+        for lo, hi in zip(bps[:-1], bps[1:]):
+            edges = np.linspace(lo, hi, pieces + 1)
+            for e0, e1 in zip(edges[:-1], edges[1:]):
+                m, hw = 0.5 * (e0 + e1), 0.5 * (e1 - e0)
+                for xg, wg in zip(gl_x, gl_w):
+                    v, _ = P.inner(px, py, j, m + hw * xg)
+                    total += hw * wg * v
+    return total
+
+
+@pytest.mark.slow
+@pytest.mark.parametrize("ix,iy", [(15, 0), (8, 8), (3, 12)])
+def test_grid_outer_vs_bruteforce(ix, iy):
+    cfg, P = _small_grid_problem()
+    r = P.potentials([iy * cfg.nx + ix])[0]
+    brute = _brute_outer(P, cfg, ix, iy, pieces=8)
+    got = np.array([r["phi"], r["ax"], r["ay"]])
+    assert np.max(np.abs(got - brute)) < P.params.tau, (got, brute)
+
+
+def test_grid_cartesian_fine_cell_sum():
+    """phi(p) = iint rho(x)/|x-p| d^2x on the TSC-interpolated static grid, by a midpoint
+    sum over fine cells; the cell containing p uses iint_{[-a,a]^2} 1/r = 8 a ln(1+sqrt 2)."""
+    cfg, P = _small_grid_problem(n=16, kap=10)
+    ix, iy = 7, 9
+    r = P.potentials([iy * cfg.nx + ix])[0]
+    px, py = P.mesh_point(ix, iy)
+    half = cfg.extent * 0.5
+    cu, cv = px + half, py + half
+    # rho on a fine lattice aligned so that p is a cell centre
+    sub = 24
+    a = cfg.hx / sub / 2
+    U0, U1 = -1.5 * cfg.hx, (cfg.nx + 0.5) * cfg.hx
+    nlo = int(math.ceil((cu - U0) / (2 * a))) + 1
+    nhi = int(math.ceil((U1 - cu) / (2 * a))) + 1
+    offs = np.arange(-nlo, nhi + 1) * 2 * a
+    U, V = np.meshgrid(cu + offs, cv + offs)
+    # TSC interpolation of the node grid (level values equal: static rigid ring)
+    G = P.ring[30 % cfg.H, :, :, 0]
+    tx, ty = U / cfg.hx, V / cfg.hy
+    fx, fy = np.floor(tx + 0.5), np.floor(ty + 0.5)
+    def w(d):
+        return [0.5 * (0.5 - d) ** 2, 0.75 - d * d, 0.5 * (0.5 + d) ** 2]
+    wx, wy = w(tx - fx), w(ty - fy)
+    rho = np.zeros_like(U)
+    for b in range(3):
+        for aa in range(3):
+            xx, yy = fx.astype(int) + aa - 1, fy.astype(int) + b - 1
+            ok = (xx >= 0) & (xx < cfg.nx) & (yy >= 0) & (yy < cfg.ny)
+            val = np.where(ok, G[np.clip(yy, 0, cfg.ny - 1), np.clip(xx, 0, cfg.nx - 1)], 0.0)
+            rho += wx[aa] * wy[b] * val
+    R = np.hypot(U - cu, V - cv)
+    cellA = (2 * a) ** 2
+    with np.errstate(divide="ignore"):
+        contrib = np.where(R > 0, rho * cellA / R, 0.0)
+    centre = rho[R == 0].sum() * 8 * a * math.log(1 + math.sqrt(2))
+    phi = contrib.sum() + centre
+    print("cartesian", phi, r["phi"], phi / r["phi"] - 1)
+    assert abs(phi - r["phi"]) < 2e-3 * abs(r["phi"]), (phi, r["phi"])

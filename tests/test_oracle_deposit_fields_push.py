@@ -1,0 +1,141 @@
+"""Pins of the oracle's deposition, self-fields and push
+against conservation laws, closed forms and hand-computed tables.
+
+Golden fixture: tests/golden/bins_ties.json (hand-computed bin indices for
+particles placed exactly on the nearest-node tie t = n + 1/2; reading R-13).
+"""
+import json
+import math
+import os
+
+import numpy as np
+import pytest
+
+import oracle
+import workloads as W
+
+GOLD = os.path.join(os.path.dirname(__file__), "golden")
+
+
+def test_bins_ties_golden():
+    with open(os.path.join(GOLD, "bins_ties.json")) as f:
+        g = json.load(f)
+    fr = g["frame"]
+    for case in g["cases"]:
+        b, ix, iy, dx, dy = oracle.bin_of(case["x"], case["y"], fr, g["hx"], g["hy"], g["nx"], g["ny"])
+        assert b == case["bin"], case
+        if b >= 0:
+            assert (ix, iy) == (case["ix"], case["iy"])
+            assert dx == case["dx"] and dy == case["dy"]
+
+
+def test_single_particle_weights():
+    # a particle exactly on node (3, 4) of a unit static grid deposits 3/4 * 3/4 there,
+    # 1/8 * 3/4 on the 4 edge neighbours and 1/64 on the corners (TSC, R-14).
+    M, bins, ql = oracle.deposit([3.0], [4.0], [0.0], [0.0], 2.0, (0, 0, 1, 0), 8, 8, 1.0, 1.0)
+    assert bins[0] == 4 * 8 + 3 and ql == 0.0
+    w = np.array([1 / 8, 3 / 4, 1 / 8])
+    np.testing.assert_allclose(M[3:6, 2:5, 0], 2.0 * np.outer(w, w), rtol=0, atol=1e-16)
+    assert abs(M[..., 0].sum() - 2.0) < 1e-15
+
+
+@pytest.mark.parametrize("geometry", ["static", "bend"])
+def test_charge_conservation_and_current(geometry):
+    cfg = W.config(1) if geometry == "static" else W.config(2)
+    n = 20_000
+    x, y, ux, uy = W.particles(cfg, n=n, seed=7)
+    # put a few particles off the grid so that the lost charge is exercised
+    x = x.copy()
+    x[:5] += 20 * cfg.sigma
+    q = 1.0 / n
+    M, bins, ql = oracle.deposit(x, y, ux, uy, q, W.frame(cfg, 0), cfg.nx, cfg.ny, cfg.hx, cfg.hy)
+    assert ql >= 5 * q - 1e-18
+    assert (bins[:5] == -1).all()
+    total = M[..., 0].sum() * cfg.hx * cfg.hy + ql
+    assert abs(total - 1.0) < 1e-13
+    # J = rho * beta for a uniform beta
+    if geometry == "bend":
+        ux2 = np.full(n, 3.0)
+        uy2 = np.full(n, -4.0)
+        M2, _, _ = oracle.deposit(x, y, ux2, uy2, q, W.frame(cfg, 0), cfg.nx, cfg.ny, cfg.hx, cfg.hy)
+        g = math.sqrt(1 + 9 + 16)
+        np.testing.assert_allclose(M2[..., 1], M2[..., 0] * 3 / g, rtol=1e-14, atol=1e-300)
+        np.testing.assert_allclose(M2[..., 2], M2[..., 0] * -4 / g, rtol=1e-14, atol=1e-300)
+    assert (M[..., 3] == 0).all()
+
+
+def test_fields_exact_on_quadratics():
+    # phi, A quadratic in (u, v): 2nd-order central and one-sided differences are exact.
+    nx, ny, hx, hy = 9, 7, 0.3, 0.45
+    psi = 0.37
+    fk = (1.0, -2.0, math.cos(psi), math.sin(psi))
+    u = np.arange(nx) * hx
+    v = np.arange(ny) * hy
+    U, V = np.meshgrid(u, v)
+    phi = 1.5 * U * U - 0.7 * U * V + 0.2 * V * V + U - 3 * V
+    ax = 0.3 * U * V + 2 * U
+    ay = -0.5 * V * V + U
+    ex, ey, bz = oracle.fields(nx, ny, hx, hy, 1.0, 0.1, fk, None, phi, ax, ay)
+    pu, pv = 3 * U - 0.7 * V + 1, -0.7 * U + 0.4 * V - 3
+    c, s = fk[2], fk[3]
+    np.testing.assert_allclose(ex, -(c * pu - s * pv), atol=1e-12)
+    np.testing.assert_allclose(ey, -(s * pu + c * pv), atol=1e-12)
+    # B_z = d_x A_y - d_y A_x in the lab, with d_x = c d_u - s d_v, d_y = s d_u + c d_v
+    ayu, ayv = np.ones_like(U), -V
+    axu, axv = 0.3 * V + 2, 0.3 * U
+    want = (c * ayu - s * ayv) - (s * axu + c * axv)
+    np.testing.assert_allclose(bz, want, atol=1e-12)
+
+
+def test_fields_dA_dt_translating_mesh():
+    # A rigidly attached to the lab, mesh translating with velocity V: A_lab(x) = x (A_x = x_lab).
+    # Then dA/dt|lab = 0 although the node values change: (A_k - A_{k-1})/dt = V_x, and the
+    # convective term (V . grad) A_x = V_x cancels it exactly.
+    nx, ny, h, dt = 6, 5, 0.5, 0.2
+    fk, fkm1 = (0.3, 0.1, 1.0, 0.0), (0.1, 0.05, 1.0, 0.0)
+    U, V = np.meshgrid(np.arange(nx) * h, np.arange(ny) * h)
+    ax = fk[0] + U
+    ax_prev = fkm1[0] + U
+    z = np.zeros_like(U)
+    ex, ey, bz = oracle.fields(nx, ny, h, h, 2.0, dt, fk, fkm1, z, ax, z, ax_prev, z)
+    np.testing.assert_allclose(ex, 0.0, atol=1e-13)
+    np.testing.assert_allclose(ey, 0.0, atol=1e-13)
+    # a purely time-dependent A_x (no gradient): E_x = -(1/c) dA_x/dt
+    ax2 = np.full_like(U, 3.0)
+    ex, ey, bz = oracle.fields(nx, ny, h, h, 2.0, dt, fk, fk, z, ax2, z, ax2 - 0.4, z)
+    np.testing.assert_allclose(ex, -(0.4 / dt) / 2.0, atol=1e-13)
+
+
+def test_boris_gyration():
+    # E = 0, uniform B_z: |u| conserved exactly-ish; the orbit closes after one period and
+    # has radius |u| c / (q/mc |B|) (leap-frog: radius within O(dtheta^2)).
+    n = 1
+    x, y, ux, uy = np.array([0.0]), np.array([0.0]), np.array([3.0]), np.array([0.0])
+    qmc, B, c, dt = 1.0, -2.0, 1.0, 0.01
+    z = np.zeros((4, 4))
+    xs, ys = [], []
+    u0 = math.hypot(ux[0], uy[0])
+    for _ in range(4000):
+        x, y, ux, uy = oracle.push(4, 4, 1.0, 1.0, c, dt, (100, 100, 1, 0), x, y, ux, uy, qmc, B, z, z, z)
+        xs.append(x[0]); ys.append(y[0])
+        assert abs(math.hypot(ux[0], uy[0]) - u0) < 1e-12
+    g = math.sqrt(1 + u0 * u0)
+    R = u0 * c / (qmc * abs(B))
+    xs, ys = np.array(xs), np.array(ys)
+    cx, cy = 0.5 * (xs.max() + xs.min()), 0.5 * (ys.max() + ys.min())
+    rad = np.hypot(xs - cx, ys - cy)
+    assert abs(rad.mean() - R) < 1e-3 * R
+    assert cy > 0  # B_z < 0 with q > 0: counter-clockwise (centre on the +y side)
+
+
+def test_push_uniform_E_acceleration():
+    # B = 0, uniform E_x on the grid: du_x = q/mc E dt exactly per step (both half kicks)
+    nx = ny = 8
+    E = np.full((ny, nx), 0.5)
+    z = np.zeros((ny, nx))
+    x, y = np.array([3.2]), np.array([4.1])
+    ux, uy = np.array([0.1]), np.array([0.0])
+    x2, y2, ux2, uy2 = oracle.push(nx, ny, 1.0, 1.0, 1.0, 0.2, (0, 0, 1, 0), x, y, ux, uy, 2.0, 0.0, E, z, z)
+    assert abs(ux2[0] - (0.1 + 2.0 * 0.5 * 0.2)) < 1e-15
+    g = math.sqrt(1 + ux2[0] ** 2)
+    assert abs(x2[0] - (3.2 + 0.2 * ux2[0] / g)) < 1e-15

@@ -1,0 +1,86 @@
+"""Invariants of the oracle's potentials that hold exactly or to rounding.
+
+* Linearity with exact power-of-two scaling: (M, tau) -> (2M, 2tau) gives bit-identical 2x
+  results and the same subdivision (Eq. 2 is linear in f; accept test err <= tau (b-a)/R).
+* J = 0 => A = 0 exactly (P:32 moments; R-1).
+* Steady state (P:176-177 LCLS bend, rigid pre-history): a rigid bunch on a circular orbit
+  gives the same potentials at steps k and k+m (to rounding) and the same subdivision.
+* Static rigid history: the result does not depend on the step index k.
+"""
+import math
+
+import numpy as np
+import pytest
+
+import oracle
+import workloads as W
+
+
+def _grid_problem(ring, fr, cfg, k, tau, n_pre=0):
+    return oracle.Problem(nx=cfg.nx, ny=cfg.ny, hx=cfg.hx, hy=cfg.hy, c=cfg.c, dt=cfg.dt, tau=tau,
+                          kappa_max=cfg.kappa_max, k=k, n_pre=n_pre, ring=ring, frames=fr)
+
+
+def _cfg_static(n=16, kap=8):
+    return W.Config(number=0, name="t", nx=n, ny=n, n_particles=1, steps=1, kappa_max=kap,
+                    geometry="static", sigma=1.0, cdt=1.6)
+
+
+def test_scaling_by_two_is_exact():
+    cfg = _cfg_static()
+    x, y, ux, uy = W.particles(W.config(1), n=3000, seed=3)
+    M, _, _ = oracle.deposit(x, y, ux + 0.1, uy, 1e-3, W.frame(cfg, 0), cfg.nx, cfg.ny, cfg.hx, cfg.hy)
+    ring = np.repeat(M[None], cfg.H, axis=0)
+    fr = W.ring_frames(cfg, 5)
+    pts = np.arange(0, cfg.nx * cfg.ny, 17)
+    r1 = _grid_problem(ring, fr, cfg, 5, 1e-7).potentials(pts)
+    r2 = _grid_problem(2 * ring, fr, cfg, 5, 2e-7).potentials(pts)
+    for key in ("phi", "ax", "ay", "err"):
+        np.testing.assert_array_equal(r2[key], 2 * r1[key])
+    np.testing.assert_array_equal(r2["nseg"], r1["nseg"])
+
+
+def test_zero_current_gives_zero_vector_potential():
+    cfg = _cfg_static()
+    x, y, ux, uy = W.particles(W.config(1), n=3000, seed=4)
+    M, _, _ = oracle.deposit(x, y, ux, uy, 1e-3, W.frame(cfg, 0), cfg.nx, cfg.ny, cfg.hx, cfg.hy)
+    assert (M[..., 1:] == 0).all()
+    ring = np.repeat(M[None], cfg.H, axis=0)
+    r = _grid_problem(ring, W.ring_frames(cfg, 4), cfg, 4, 1e-6).potentials(np.arange(0, 256, 9))
+    assert (r["ax"] == 0).all() and (r["ay"] == 0).all()
+    assert (r["phi"] > 0).all()
+
+
+def test_static_result_independent_of_step():
+    cfg = _cfg_static()
+    ring = W.node_gaussian_ring(cfg, k=0)
+    ra = _grid_problem(ring, W.ring_frames(cfg, 0), cfg, 0, 1e-6, n_pre=cfg.n_pre).potentials([0, 77, 136])
+    # same rigid grids in every slot, viewed at step 23 without pre-history
+    rb = _grid_problem(ring, W.ring_frames(cfg, 23), cfg, 23, 1e-6).potentials([0, 77, 136])
+    np.testing.assert_array_equal(ra["phi"], rb["phi"])
+    np.testing.assert_array_equal(ra["nseg"], rb["nseg"])
+
+
+def _bend_small():
+    c = W.config(2)
+    return W.Config(number=2, name="bend-small", nx=24, ny=24, n_particles=1, steps=60,
+                    kappa_max=60, geometry="bend", sigma=c.sigma, cdt=c.cdt, gamma0=c.gamma0,
+                    r0=c.r0, sigma_xp=c.sigma_xp, q_over_mc=c.q_over_mc)
+
+
+@pytest.mark.slow
+def test_bend_steady_state_stationarity():
+    cfg = _bend_small()
+    ring = W.node_gaussian_ring(cfg, k=0, beta=(cfg.beta0, 0.0))
+    pts = [12 * 24 + 12, 12 * 24 + 20, 5 * 24 + 3]
+    out = []
+    for k in (0, 1, 7):
+        P = _grid_problem(ring, W.ring_frames(cfg, k), cfg, k, cfg.tau, n_pre=cfg.n_pre)
+        out.append(P.potentials(pts))
+    for r in out[1:]:
+        np.testing.assert_array_equal(r["nseg"], out[0]["nseg"])
+        rel = np.abs(r["phi"] - out[0]["phi"]) / np.abs(out[0]["phi"])
+        assert rel.max() < 1e-10, rel
+    # sanity: the bend potential at the bunch centre is O(Q/sigma)
+    scale = 1.0 / cfg.sigma * math.sqrt(math.pi / 2)
+    assert 0.5 < out[0]["phi"][0] / scale < 10
