@@ -1,0 +1,220 @@
+/*
+ * rp.h -- C ABI of librp, the B200-native retarded-potential step of
+ *   Arumugam et al., "A Machine Learning Approach for Efficient Parallel
+ *   Simulation of Beam Dynamics on GPUs", ICPP'17.
+ *   Citations "P:NN" are lines of the paper text;
+ *   "R-n" are the readings listed in DESIGN.md sec. 3 where the paper is silent.
+ *
+ * One time step k is the paper's four-step loop:
+ *   rp_deposit_step        1) particle deposition onto the N_X x N_Y grid D_k
+ *   rp_compute_potentials  2) retarded potentials at every grid point, Eq. 1-2,
+ *                             COMPUTE-POTENTIALS(k, V, tau, g, D) of Algorithm 1
+ *   rp_compute_fields      3) self-fields from the potentials
+ *   rp_push_particles      4) leap-frog Lorentz push by dt
+ *
+ * Conventions (all functions):
+ *   - Array arguments are DEVICE pointers unless the name ends in _host.  The caller
+ *     owns them; the library never frees caller memory and keeps no pointer to it
+ *     after the call returns.  Device arrays must be 8-byte aligned.
+ *   - All device work is ordered on the context's stream (rp_set_stream); calls
+ *     return after enqueueing, except where "syncs" is stated.
+ *   - Every call returns RP_OK (0) or a negative RP_E* code; no exception or exit()
+ *     crosses the ABI.  rp_strerror() gives a static description, rp_last_error()
+ *     the detailed message of the last failing call on that context.
+ *   - FP64 everywhere (double-precision GFLOP/s).  Units are Gaussian with
+ *     the caller's length/time units: phi = I_rho, A = I_{rho beta} (R-1).
+ *   - One context per stream / host thread.  Contexts are independent.
+ */
+#ifndef RP_H_
+#define RP_H_
+
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+#define RP_OK 0
+#define RP_EINVAL (-1)  /* bad argument or configuration                      */
+#define RP_ENOMEM (-2)  /* device or host allocation failed                    */
+#define RP_ECUDA (-3)   /* CUDA runtime / kernel error (see rp_last_error)     */
+#define RP_ESTATE (-5)  /* call out of order (e.g. potentials before deposit)  */
+#define RP_ENODEV (-6)  /* no usable CUDA device                               */
+
+#define RP_SRC_GRID 0   /* integrand from the deposited history (the product)  */
+#define RP_SRC_GAUSS 1  /* analytic Gaussian sheet (test source)   */
+#define RP_SRC_DISK 2   /* analytic uniform disk (test source)     */
+
+typedef struct rp_ctx rp_ctx;
+
+/* Grid frame of one time step: lab = O + u (c, s) + v (-s, c); grid node (ix, iy) sits
+ * at local (ix*hx, iy*hy).  Frames move with the bunch (R-7). */
+typedef struct {
+  double ox, oy, cos_psi, sin_psi;
+} rp_frame;
+
+typedef struct {
+  int32_t nx, ny;          /* grid nodes, >= 4 (P:32 N_X x N_Y); mesh points V = all nodes      */
+  double hx, hy;           /* node spacing, > 0                                                  */
+  int32_t history_depth;   /* kappa_max >= 1 subregions of reach; ring holds kappa_max+2 grids  */
+  double c, dt;            /* > 0; subregion width c*dt (P:45 S_j = [j c dt, (j+1) c dt])        */
+  double tau;              /* > 0; absolute tolerance per component (P:170 tau = 1e-6)           */
+  int32_t n_theta;         /* even >= 2; inner Newton-Cotes panels per arc (R-11)          */
+  int32_t max_depth;       /* 1..60 bisection cap of the outer tree (R-12)                       */
+  int32_t n_root;          /* 2: roots are the two halves of each clipped S_j (R-12b); or 1     */
+  int32_t device;          /* CUDA ordinal                                                       */
+} rp_config;
+
+typedef struct {
+  int64_t n_lost;          /* particles whose 3x3 stencil leaves the grid (R-14)                 */
+  double q_lost, q_total;
+} rp_deposit_info;
+
+typedef struct {
+  int64_t evals;           /* integrand evaluations f(r', theta', t') (flop census)             */
+  int64_t nodes;           /* r' nodes (15 per GK15 segment)                                     */
+  int64_t segments;        /* GK15 segments evaluated (sum of nseg)                              */
+  int64_t leaves;          /* accepted segments                                                  */
+  int64_t capped;          /* leaves accepted at max_depth with err > tol                        */
+  int64_t ties;            /* decisions with |err - tol| / tol < 1e-9                            */
+  int64_t items;           /* (point, subregion) pairs with support                              */
+  int32_t max_level;       /* deepest tree level reached                                         */
+  int32_t kappa;           /* subregions kappa(k) used at this step (R-3)                        */
+} rp_potential_info;
+
+/* Create a context on cfg->device: allocates the HBM history ring of history_depth+2
+ * FP64 moment grids [slot][ny+6][nx+6][4] (zero-padded by 3 nodes) and scratch.
+ * EINVAL on an invalid config, ENODEV / ENOMEM / ECUDA on device failures. */
+int rp_create(const rp_config* cfg, rp_ctx** out);
+
+/* Destroy a context (NULL is ignored).  Synchronises its stream first. */
+void rp_destroy(rp_ctx* ctx);
+
+/* Use `stream` (a cudaStream_t; NULL = legacy default stream) for all later work. */
+int rp_set_stream(rp_ctx* ctx, void* stream);
+
+/* Optional pre-history, allowed only before the first deposit (else ESTATE).
+ * n_pre in 1..history_depth+1 levels l = -n_pre .. -1; frames_host[n_pre] oldest first.
+ * rigid = 0: grids_dev holds [n_pre][ny][nx][4] FP64 moment grids (component 3 ignored).
+ * rigid = 1: grids_dev must be NULL; every pre-history level receives a copy of the
+ *            step-0 grid when the first deposit is appended (steady state).
+ * Without pre-history, kappa(k) = min(kappa_max, k - 1) (R-3). */
+int rp_history_init(rp_ctx* ctx, int32_t n_pre, const rp_frame* frames_host,
+                    const double* grids_dev, int32_t rigid);
+
+/* Partial deposition of n local particles (SoA x, y, u_x, u_y with u = gamma*beta) of
+ * charge q each on frame_k (TSC, R-14): writes partial_dev [ny][nx][4] =
+ * (rho, rho*beta_x, rho*beta_y, 0), overwritten.  Bins are computed without FMA so
+ * they are bit-identical to the oracle (R-13).  Atomics-free: particles are radix-sorted
+ * by bin and every node sums its 9 neighbour bins in a fixed order.
+ * info (nullable) syncs the stream. */
+int rp_deposit(rp_ctx* ctx, const double* x, const double* y, const double* ux,
+               const double* uy, double q, int64_t n, const rp_frame* frame_k,
+               double* partial_dev, rp_deposit_info* info);
+
+/* Advance to the next step k (0 at the first call) and store
+ * D_k = sum_{i < n_parts} partials_dev[i] (summed in index order = rank order) into ring
+ * slot k mod H with frame_k ("stored linearly on the device memory").
+ * partials_dev is [n_parts][ny][nx][4]. */
+int rp_history_append(rp_ctx* ctx, const double* partials_dev, int32_t n_parts,
+                      const rp_frame* frame_k);
+
+/* rp_deposit into context scratch + rp_history_append(n_parts = 1). */
+int rp_deposit_step(rp_ctx* ctx, const double* x, const double* y, const double* ux,
+                    const double* uy, double q, int64_t n, const rp_frame* frame_k,
+                    rp_deposit_info* info);
+
+/* Retarded potentials at all nx*ny nodes of the current frame (Eq. 1-2, Alg. 1).
+ * For every (point p, subregion j < kappa(k)): support clip [A, B] of S_j (R-5), then a
+ * deterministic top-down dyadic GK15 tree from the n_root halves of [A, B]: accept a
+ * segment iff max_c |K15_c - G7_c| <= tau (b - a) / R(p), R(p) = kappa(k) c dt, or at
+ * max_depth (R-8..R-12).  Work items are scheduled longest-predicted-first from the
+ * previous step's per-(p, j) segment counts (the paper's forecast g, used for
+ * scheduling only).  Outputs [ny*nx] (flattened iy*nx + ix): phi = sum K_0,
+ * ax = sum K_1, ay = sum K_2, err = sum of leaf errors, nseg = segments evaluated.
+ * err / nseg may be NULL.  info (nullable) syncs. */
+int rp_compute_potentials(rp_ctx* ctx, double* phi, double* ax, double* ay, double* err,
+                          int32_t* nseg, rp_potential_info* info);
+
+/* As rp_compute_potentials but only for the points owned by `rank` of `world` under the
+ * context's shard map (mesh-point data parallelism): points are dealt
+ * longest-predicted-first in a snake order over ranks from the previous step's counts,
+ * identical on every rank.  Writes shard_out [cap][6] FP64 records
+ * (point id, phi, ax, ay, err, nseg) for the owned points, rows >= *n_out zero-filled;
+ * cap >= rp_shard_capacity().  Combine the all-gathered shards with rp_shard_scatter. */
+int rp_compute_potentials_shard(rp_ctx* ctx, int32_t rank, int32_t world, double* shard_out,
+                                int64_t cap, int64_t* n_out, rp_potential_info* info);
+
+/* Rows per shard buffer: ceil(nx*ny / world). */
+int64_t rp_shard_capacity(const rp_ctx* ctx, int32_t world);
+
+/* Scatter `world` gathered shard buffers [world][cap][6] into full-mesh outputs and
+ * record the counts for the next step's schedule (identical on every rank). */
+int rp_shard_scatter(rp_ctx* ctx, const double* shards, int32_t world, int64_t cap,
+                     double* phi, double* ax, double* ay, double* err, int32_t* nseg);
+
+/* Self-fields on mesh k (R-15): second-order central differences (one-sided at the
+ * edges) in frame coordinates rotated to the lab;
+ *   E = -grad phi - (1/c) dA/dt,  dA/dt = (A_k - A_{k-1})/dt - (V.grad) A_k,
+ *   V = node velocity (P_k - P_{k-1})/dt;  B_z = d_x A_y - d_y A_x.
+ * ax_prev / ay_prev (step k-1 on its own mesh) may both be NULL: dA/dt is then 0.
+ * All arrays [ny*nx]. */
+int rp_compute_fields(rp_ctx* ctx, const double* phi, const double* ax, const double* ay,
+                      const double* ax_prev, const double* ay_prev, double* ex, double* ey,
+                      double* bz);
+
+/* Relativistic Boris leap-frog push by dt (R-15) of n particles in place:
+ * TSC gather of (E_x, E_y, B_z) on frame k (same weights as deposition), plus a uniform
+ * external B_z = bz_ext; du/dt = q_over_mc (E + beta x B); x += c dt u / gamma. */
+int rp_push_particles(rp_ctx* ctx, double* x, double* y, double* ux, double* uy, int64_t n,
+                      double q_over_mc, double bz_ext, const double* ex, const double* ey,
+                      const double* bz);
+
+/* One whole step through HOST buffers (end-to-end path): copies the particles
+ * host->device, runs deposit_step, compute_potentials, compute_fields (with the previous
+ * step's A kept by the context), push, and copies the pushed particles and the six mesh
+ * outputs back.  x_host .. uy_host are updated in place; mesh_host is [6][ny*nx]
+ * (phi, ax, ay, ex, ey, bz).  Pinned host memory gives full-bandwidth copies.  Syncs. */
+int rp_step_host(rp_ctx* ctx, double* x_host, double* y_host, double* ux_host,
+                 double* uy_host, int64_t n, double q, const rp_frame* frame_k,
+                 double q_over_mc, double bz_ext, double* mesh_host, rp_potential_info* info);
+
+/* ---- state access (checkpoint / parity from a common seeded state) ---- */
+
+/* Overwrite the whole history: step index k, pre-history depth n_pre (for kappa(k)),
+ * frames_host[H] and ring_dev [H][ny][nx][4] in ring-slot order (slot = level mod H).
+ * Clears the schedule forecast.  Allowed at any time. */
+int rp_load_state(rp_ctx* ctx, int32_t k, int32_t n_pre, const rp_frame* frames_host,
+                  const double* ring_dev);
+
+/* Copy the ring out ([H][ny][nx][4], unpadded) and/or the frames; NULLs skip.  Syncs. */
+int rp_save_state(rp_ctx* ctx, int32_t* k_out, double* ring_dev, rp_frame* frames_host);
+
+/* Bin index of every particle of the last rp_deposit (-1 = lost), [n]. */
+int rp_debug_bins(rp_ctx* ctx, int32_t* bins_dev, int64_t n);
+
+/* Test hook: potentials with an analytic source in place of the grid:
+ * kind = RP_SRC_GAUSS (centre (x0,y0) frame-local, width = sigma, q = Q) or RP_SRC_DISK
+ * (width = radius, q = surface density); (bx, by) = beta; amp_host[H] per-slot amplitudes
+ * (NULL = 1).  Same clip / tree / inner rule / kernels as the grid path. */
+int rp_debug_potentials_analytic(rp_ctx* ctx, int32_t kind, double x0, double y0,
+                                 double width, double q, double bx, double by,
+                                 const double* amp_host, double* phi, double* ax, double* ay,
+                                 double* err, int32_t* nseg, rp_potential_info* info);
+
+/* Number of kernel launches this context has issued (for bench.py's gpu_launches). */
+int64_t rp_launch_count(const rp_ctx* ctx);
+
+/* Static text for an RP_E* code. */
+const char* rp_strerror(int code);
+
+/* Detailed message of the last failing call on ctx (never NULL). */
+const char* rp_last_error(const rp_ctx* ctx);
+
+/* ABI version (major*100 + minor). */
+int rp_version(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* RP_H_ */

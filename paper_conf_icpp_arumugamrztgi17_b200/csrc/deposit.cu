@@ -1,0 +1,232 @@
+// deposit.cu -- step 1 of the paper's loop: particle deposition onto the grid of
+// moments D_k, and the history append.  Atomics-free sorted-bin scatter:
+//   k_bin        particle -> nearest node (bit-exact, no FMA; R-13), TSC offsets, beta
+//   CUB sort     stable radix sort of (bin, particle id)
+//   k_bin_start  per-bin start offsets (binary search in the sorted keys)
+//   k_gather     particle records into sorted order (coalesced reads below)
+//   k_node_sum   one warp per node: fixed-order sum over its 9 neighbour bins -> M_k
+//   k_append     D_k = sum of per-rank partials in rank order -> ring slot k mod H
+#include <cub/device/device_radix_sort.cuh>
+
+#include "rp_internal.cuh"
+
+namespace {
+
+__global__ void k_bin(int64_t n, const double* __restrict__ x, const double* __restrict__ y,
+                      const double* __restrict__ ux, const double* __restrict__ uy,
+                      rp_frame F, double hx, double hy, int nx, int ny,
+                      int32_t* __restrict__ key, int32_t* __restrict__ perm,
+                      double4* __restrict__ rec) {
+  int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+  if (i >= n) return;
+  // local coordinates and nearest node: IEEE round-to-nearest, no contraction (R-13)
+  double dx = __dsub_rn(x[i], F.ox), dy = __dsub_rn(y[i], F.oy);
+  double u = __dadd_rn(__dmul_rn(F.cos_psi, dx), __dmul_rn(F.sin_psi, dy));
+  double v = __dsub_rn(__dmul_rn(F.cos_psi, dy), __dmul_rn(F.sin_psi, dx));
+  double tx = __ddiv_rn(u, hx), ty = __ddiv_rn(v, hy);
+  double fx = floor(__dadd_rn(tx, 0.5)), fy = floor(__dadd_rn(ty, 0.5));
+  bool ok = fx >= 1.0 && fx <= (double)(nx - 2) && fy >= 1.0 && fy <= (double)(ny - 2);
+  double a = ux[i], b = uy[i];
+  double g = sqrt(1.0 + a * a + b * b);
+  key[i] = ok ? (int32_t)fy * nx + (int32_t)fx : nx * ny;
+  perm[i] = (int32_t)i;
+  rec[i] = make_double4(__dsub_rn(tx, fx), __dsub_rn(ty, fy), a / g, b / g);
+}
+
+__global__ void k_bin_start(const int32_t* __restrict__ keys, int64_t n, int nbins,
+                            int32_t* __restrict__ start) {
+  int b = blockIdx.x * blockDim.x + threadIdx.x;
+  if (b > nbins) return;
+  int64_t lo = 0, hi = n;  // first index with keys[idx] >= b
+  while (lo < hi) {
+    int64_t m = (lo + hi) >> 1;
+    if (keys[m] < b) lo = m + 1; else hi = m;
+  }
+  start[b] = (int32_t)lo;
+}
+
+__global__ void k_gather(int64_t n, const int32_t* __restrict__ perm,
+                         const double4* __restrict__ rec, double4* __restrict__ out) {
+  int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+  if (i < n) out[i] = rec[perm[i]];
+}
+
+__device__ __forceinline__ void tsc(double d, double& wm, double& w0, double& wp) {
+  double a = 0.5 - d, b = 0.5 + d;
+  wm = 0.5 * (a * a);
+  w0 = 0.75 - d * d;
+  wp = 0.5 * (b * b);
+}
+
+// One warp per grid node.  Node (ix, iy) receives from the particles of bin
+// (ix - oa, iy - ob), oa, ob in {-1, 0, 1}, the weight w_oa(dx) w_ob(dy) (TSC).
+__global__ void k_node_sum(int nx, int ny, const int32_t* __restrict__ start,
+                           const double4* __restrict__ rec, double scale,
+                           double* __restrict__ M) {
+  int warp = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+  int lane = threadIdx.x & 31;
+  if (warp >= nx * ny) return;
+  int ix = warp % nx, iy = warp / nx;
+  double s0 = 0.0, s1 = 0.0, s2 = 0.0;
+  for (int ob = -1; ob <= 1; ++ob) {
+    int by = iy - ob;
+    if (by < 1 || by > ny - 2) continue;
+    for (int oa = -1; oa <= 1; ++oa) {
+      int bx = ix - oa;
+      if (bx < 1 || bx > nx - 2) continue;
+      int b = by * nx + bx;
+      int p0 = start[b], p1 = start[b + 1];
+      for (int p = p0 + lane; p < p1; p += 32) {
+        double4 r = rec[p];
+        double wm, w0, wp, vm, v0, vp;
+        tsc(r.x, wm, w0, wp);
+        tsc(r.y, vm, v0, vp);
+        double wx = oa < 0 ? wm : (oa == 0 ? w0 : wp);
+        double wy = ob < 0 ? vm : (ob == 0 ? v0 : vp);
+        double w = wx * wy;
+        s0 += w;
+        s1 += w * r.z;
+        s2 += w * r.w;
+      }
+    }
+  }
+  for (int o = 16; o > 0; o >>= 1) {
+    s0 += __shfl_xor_sync(0xffffffffu, s0, o);
+    s1 += __shfl_xor_sync(0xffffffffu, s1, o);
+    s2 += __shfl_xor_sync(0xffffffffu, s2, o);
+  }
+  if (lane == 0) {
+    double* m = M + 4 * (size_t)warp;
+    m[0] = scale * s0;
+    m[1] = scale * s1;
+    m[2] = scale * s2;
+    m[3] = 0.0;
+  }
+}
+
+// ring slot (padded) <- sum of n_parts unpadded partial grids, in part order
+__global__ void k_append(int nx, int ny, int PX, const double* __restrict__ parts,
+                         int n_parts, double* __restrict__ slot) {
+  int id = blockIdx.x * blockDim.x + threadIdx.x;
+  if (id >= nx * ny) return;
+  int ix = id % nx, iy = id / nx;
+  size_t np = (size_t)nx * ny * 4;
+  double a = 0.0, b = 0.0, c = 0.0;
+  for (int i = 0; i < n_parts; ++i) {
+    const double* m = parts + i * np + 4 * (size_t)id;
+    a += m[0];
+    b += m[1];
+    c += m[2];
+  }
+  double* d = slot + 4 * ((size_t)(iy + RP_PAD) * PX + (ix + RP_PAD));
+  d[0] = a;
+  d[1] = b;
+  d[2] = c;
+  d[3] = 0.0;
+}
+
+int grow_deposit(rp_ctx* ctx, int64_t n) {
+  if (n <= ctx->dep_cap) return RP_OK;
+  int64_t cap = n + n / 8 + 1024;
+  cudaFree(ctx->keys); cudaFree(ctx->keys_sorted); cudaFree(ctx->perm);
+  cudaFree(ctx->perm_sorted); cudaFree(ctx->rec); cudaFree(ctx->rec_sorted);
+  ctx->keys = ctx->keys_sorted = ctx->perm = ctx->perm_sorted = nullptr;
+  ctx->rec = ctx->rec_sorted = nullptr;
+  ctx->dep_cap = 0;
+  RP_CUDA(cudaMalloc(&ctx->keys, cap * sizeof(int32_t)));
+  RP_CUDA(cudaMalloc(&ctx->keys_sorted, cap * sizeof(int32_t)));
+  RP_CUDA(cudaMalloc(&ctx->perm, cap * sizeof(int32_t)));
+  RP_CUDA(cudaMalloc(&ctx->perm_sorted, cap * sizeof(int32_t)));
+  RP_CUDA(cudaMalloc(&ctx->rec, cap * sizeof(double4)));
+  RP_CUDA(cudaMalloc(&ctx->rec_sorted, cap * sizeof(double4)));
+  ctx->dep_cap = cap;
+  return RP_OK;
+}
+
+}  // namespace
+
+int rp_ensure_cub_tmp(rp_ctx* ctx, size_t bytes) {
+  if (bytes <= ctx->cub_tmp_bytes) return RP_OK;
+  cudaFree(ctx->cub_tmp);
+  ctx->cub_tmp = nullptr;
+  ctx->cub_tmp_bytes = 0;
+  size_t b = bytes + bytes / 4 + 4096;
+  RP_CUDA(cudaMalloc(&ctx->cub_tmp, b));
+  ctx->cub_tmp_bytes = b;
+  return RP_OK;
+}
+
+int rp_deposit_impl(rp_ctx* ctx, const double* x, const double* y, const double* ux,
+                    const double* uy, double q, int64_t n, const rp_frame* fk,
+                    double* partial, rp_deposit_info* info) {
+  const rp_config& c = ctx->cfg;
+  if (n < 0 || n > 0x7fffffffLL || !fk || !partial) return rp_fail(ctx, RP_EINVAL, "deposit: bad args");
+  if (n > 0 && (!x || !y || !ux || !uy)) return rp_fail(ctx, RP_EINVAL, "deposit: null particle array");
+  int rc = grow_deposit(ctx, n > 0 ? n : 1);
+  if (rc) return rc;
+  const int nbins = c.nx * c.ny;  // + 1 "lost" bin with key nbins
+  cudaStream_t st = ctx->stream;
+  ctx->last_n = n;
+  if (n > 0) {
+    int T = 256;
+    k_bin<<<(unsigned)((n + T - 1) / T), T, 0, st>>>(n, x, y, ux, uy, *fk, c.hx, c.hy, c.nx,
+                                                      c.ny, ctx->keys, ctx->perm, ctx->rec);
+    RP_CHECK_LAUNCH();
+    int end_bit = 1;
+    while ((1LL << end_bit) <= nbins) ++end_bit;
+    size_t tmp = 0;
+    RP_CUDA(cub::DeviceRadixSort::SortPairs(nullptr, tmp, ctx->keys, ctx->keys_sorted, ctx->perm,
+                                            ctx->perm_sorted, (int)n, 0, end_bit, st));
+    rc = rp_ensure_cub_tmp(ctx, tmp);
+    if (rc) return rc;
+    tmp = ctx->cub_tmp_bytes;
+    RP_CUDA(cub::DeviceRadixSort::SortPairs(ctx->cub_tmp, tmp, ctx->keys, ctx->keys_sorted,
+                                            ctx->perm, ctx->perm_sorted, (int)n, 0, end_bit, st));
+    k_bin_start<<<(nbins + 1 + 255) / 256, 256, 0, st>>>(ctx->keys_sorted, n, nbins, ctx->bin_start);
+    RP_CHECK_LAUNCH();
+    k_gather<<<(unsigned)((n + T - 1) / T), T, 0, st>>>(n, ctx->perm_sorted, ctx->rec, ctx->rec_sorted);
+    RP_CHECK_LAUNCH();
+  } else {
+    RP_CUDA(cudaMemsetAsync(ctx->bin_start, 0, (nbins + 1) * sizeof(int32_t), st));
+  }
+  double scale = q / (c.hx * c.hy);
+  int warps_per_block = 8;
+  k_node_sum<<<(nbins + warps_per_block - 1) / warps_per_block, 32 * warps_per_block, 0, st>>>(
+      c.nx, c.ny, ctx->bin_start, ctx->rec_sorted, scale, partial);
+  RP_CHECK_LAUNCH();
+  if (info) {
+    int32_t kept = 0;
+    RP_CUDA(cudaMemcpyAsync(&kept, ctx->bin_start + nbins, sizeof(int32_t), cudaMemcpyDeviceToHost, st));
+    RP_CUDA(cudaStreamSynchronize(st));
+    if (n == 0) kept = 0;
+    info->n_lost = n - kept;
+    info->q_lost = q * (double)(n - kept);
+    info->q_total = q * (double)n;
+  }
+  return RP_OK;
+}
+
+int rp_append_impl(rp_ctx* ctx, const double* parts, int32_t n_parts, const rp_frame* fk) {
+  const rp_config& c = ctx->cfg;
+  if (!parts || n_parts < 1 || !fk) return rp_fail(ctx, RP_EINVAL, "append: bad args");
+  cudaStream_t st = ctx->stream;
+  int knew = ctx->k + 1;
+  int s = slot_of(knew, ctx->H);
+  double* slot = ctx->ring + (size_t)s * ctx->slot_doubles;
+  int npts = c.nx * c.ny;
+  k_append<<<(npts + 255) / 256, 256, 0, st>>>(c.nx, c.ny, ctx->PX, parts, n_parts, slot);
+  RP_CHECK_LAUNCH();
+  ctx->fh[s] = *fk;
+  RP_CUDA(cudaMemcpyAsync(ctx->frames_dev + s, fk, sizeof(rp_frame), cudaMemcpyHostToDevice, st));
+  if (knew == 0 && ctx->rigid_pending) {
+    for (int l = -ctx->n_pre; l < 0; ++l) {
+      double* d = ctx->ring + (size_t)slot_of(l, ctx->H) * ctx->slot_doubles;
+      RP_CUDA(cudaMemcpyAsync(d, slot, ctx->slot_doubles * sizeof(double), cudaMemcpyDeviceToDevice, st));
+    }
+    ctx->rigid_pending = 0;
+  }
+  ctx->k = knew;
+  // frames are read by later kernels from frames_dev; the host copy is pageable, so the
+  // H2D copy above is synchronous w.r.t. the host buffer (safe to reuse fk).
+  return RP_OK;
+}

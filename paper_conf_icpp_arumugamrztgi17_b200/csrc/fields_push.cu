@@ -1,0 +1,140 @@
+// fields_push.cu -- steps 3 and 4 of the paper's loop (P:58 self-forces from the potentials,
+// P:60 leap-frog Lorentz push).  Both are O(N_x N_y) / O(N) streaming kernels bound by HBM;
+// one thread per mesh node / particle, coalesced SoA access.
+#include "rp_internal.cuh"
+
+namespace {
+
+// second-order derivative along u (dir 0) or v (dir 1); one-sided at the edges (R-15)
+__device__ __forceinline__ double dd(const double* __restrict__ f, int nx, int ny, int ix, int iy,
+                                     int dir, double h) {
+  int n = dir == 0 ? nx : ny, i = dir == 0 ? ix : iy;
+  size_t s = dir == 0 ? 1 : (size_t)nx;
+  const double* p = f + (size_t)iy * nx + ix;
+  if (i == 0) return (-3.0 * p[0] + 4.0 * p[s] - p[2 * s]) / (2.0 * h);
+  if (i == n - 1) return (3.0 * p[0] - 4.0 * p[-(ptrdiff_t)s] + p[-2 * (ptrdiff_t)s]) / (2.0 * h);
+  return (p[s] - p[-(ptrdiff_t)s]) / (2.0 * h);
+}
+
+__global__ void k_fields(int nx, int ny, double hx, double hy, double c, double dt, rp_frame Fk,
+                         rp_frame Fm, int have_prev, const double* __restrict__ phi,
+                         const double* __restrict__ ax, const double* __restrict__ ay,
+                         const double* __restrict__ axp, const double* __restrict__ ayp,
+                         double* __restrict__ ex, double* __restrict__ ey,
+                         double* __restrict__ bz) {
+  int id = blockIdx.x * blockDim.x + threadIdx.x;
+  if (id >= nx * ny) return;
+  int ix = id % nx, iy = id / nx;
+  double cs = Fk.cos_psi, sn = Fk.sin_psi;
+  double pu = dd(phi, nx, ny, ix, iy, 0, hx), pv = dd(phi, nx, ny, ix, iy, 1, hy);
+  double xu = dd(ax, nx, ny, ix, iy, 0, hx), xv = dd(ax, nx, ny, ix, iy, 1, hy);
+  double yu = dd(ay, nx, ny, ix, iy, 0, hx), yv = dd(ay, nx, ny, ix, iy, 1, hy);
+  double phx = cs * pu - sn * pv, phy = sn * pu + cs * pv;
+  double axx = cs * xu - sn * xv, axy = sn * xu + cs * xv;  // d_x A_x, d_y A_x
+  double ayx = cs * yu - sn * yv, ayy = sn * yu + cs * yv;  // d_x A_y, d_y A_y
+  double dax = 0.0, day = 0.0;
+  if (have_prev) {
+    double u = ix * hx, v = iy * hy;
+    double pxk = Fk.ox + u * Fk.cos_psi - v * Fk.sin_psi;
+    double pyk = Fk.oy + u * Fk.sin_psi + v * Fk.cos_psi;
+    double pxm = Fm.ox + u * Fm.cos_psi - v * Fm.sin_psi;
+    double pym = Fm.oy + u * Fm.sin_psi + v * Fm.cos_psi;
+    double vx = (pxk - pxm) / dt, vy = (pyk - pym) / dt;
+    dax = (ax[id] - axp[id]) / dt - (vx * axx + vy * axy);
+    day = (ay[id] - ayp[id]) / dt - (vx * ayx + vy * ayy);
+  }
+  ex[id] = -phx - dax / c;
+  ey[id] = -phy - day / c;
+  bz[id] = ayx - axy;
+}
+
+__device__ __forceinline__ void tsc(double d, double& wm, double& w0, double& wp) {
+  double a = 0.5 - d, b = 0.5 + d;
+  wm = 0.5 * (a * a);
+  w0 = 0.75 - d * d;
+  wp = 0.5 * (b * b);
+}
+
+__global__ void k_push(int64_t n, double* __restrict__ x, double* __restrict__ y,
+                       double* __restrict__ ux, double* __restrict__ uy, rp_frame F, int nx,
+                       int ny, double inv_hx, double inv_hy, double c, double dt, double qmc,
+                       double bz_ext, const double* __restrict__ ex,
+                       const double* __restrict__ ey, const double* __restrict__ bz) {
+  int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+  if (i >= n) return;
+  double X = x[i], Y = y[i];
+  double dx = X - F.ox, dy = Y - F.oy;
+  double u = F.cos_psi * dx + F.sin_psi * dy;
+  double v = F.cos_psi * dy - F.sin_psi * dx;
+  double tx = u * inv_hx, ty = v * inv_hy;
+  double fx = floor(tx + 0.5), fy = floor(ty + 0.5);
+  double Ex = 0.0, Ey = 0.0, Bz = 0.0;
+  if (fx >= -2.0 && fx <= nx + 1.0 && fy >= -2.0 && fy <= ny + 1.0) {
+    double wx[3], wy[3];
+    tsc(tx - fx, wx[0], wx[1], wx[2]);
+    tsc(ty - fy, wy[0], wy[1], wy[2]);
+    int ix = (int)fx, iy = (int)fy;
+#pragma unroll
+    for (int b = 0; b < 3; ++b) {
+      int yy = iy + b - 1;
+      if (yy < 0 || yy >= ny) continue;
+#pragma unroll
+      for (int a = 0; a < 3; ++a) {
+        int xx = ix + a - 1;
+        if (xx < 0 || xx >= nx) continue;
+        size_t id = (size_t)yy * nx + xx;
+        double w = wx[a] * wy[b];
+        Ex += w * __ldg(ex + id);
+        Ey += w * __ldg(ey + id);
+        Bz += w * __ldg(bz + id);
+      }
+    }
+  }
+  Bz += bz_ext;
+  double h = 0.5 * qmc * dt;
+  double umx = ux[i] + h * Ex, umy = uy[i] + h * Ey;
+  double gm = sqrt(1.0 + umx * umx + umy * umy);
+  double t = h * Bz / gm;
+  double s = 2.0 * t / (1.0 + t * t);
+  double upx = umx + umy * t, upy = umy - umx * t;
+  double ppx = umx + upy * s, ppy = umy - upx * s;
+  double nux = ppx + h * Ex, nuy = ppy + h * Ey;
+  double g = sqrt(1.0 + nux * nux + nuy * nuy);
+  ux[i] = nux;
+  uy[i] = nuy;
+  x[i] = X + c * dt * nux / g;
+  y[i] = Y + c * dt * nuy / g;
+}
+
+}  // namespace
+
+int rp_fields_impl(rp_ctx* ctx, const double* phi, const double* ax, const double* ay,
+                   const double* axp, const double* ayp, double* ex, double* ey, double* bz) {
+  const rp_config& c = ctx->cfg;
+  if (ctx->k < 0) return rp_fail(ctx, RP_ESTATE, "fields before the first deposit");
+  if (!phi || !ax || !ay || !ex || !ey || !bz) return rp_fail(ctx, RP_EINVAL, "fields: null array");
+  if ((axp == nullptr) != (ayp == nullptr)) return rp_fail(ctx, RP_EINVAL, "fields: give both or neither prev");
+  int have_prev = axp != nullptr;
+  rp_frame Fk = ctx->fh[slot_of(ctx->k, ctx->H)];
+  rp_frame Fm = ctx->fh[slot_of(ctx->k - 1, ctx->H)];
+  int npts = c.nx * c.ny;
+  k_fields<<<(npts + 255) / 256, 256, 0, ctx->stream>>>(c.nx, c.ny, c.hx, c.hy, c.c, c.dt, Fk, Fm,
+                                                         have_prev, phi, ax, ay, axp, ayp, ex, ey, bz);
+  RP_CHECK_LAUNCH();
+  return RP_OK;
+}
+
+int rp_push_impl(rp_ctx* ctx, double* x, double* y, double* ux, double* uy, int64_t n, double qmc,
+                 double bz_ext, const double* ex, const double* ey, const double* bz) {
+  const rp_config& c = ctx->cfg;
+  if (ctx->k < 0) return rp_fail(ctx, RP_ESTATE, "push before the first deposit");
+  if (n < 0) return rp_fail(ctx, RP_EINVAL, "push: n < 0");
+  if (n == 0) return RP_OK;
+  if (!x || !y || !ux || !uy || !ex || !ey || !bz) return rp_fail(ctx, RP_EINVAL, "push: null array");
+  rp_frame Fk = ctx->fh[slot_of(ctx->k, ctx->H)];
+  k_push<<<(unsigned)((n + 255) / 256), 256, 0, ctx->stream>>>(n, x, y, ux, uy, Fk, c.nx, c.ny,
+                                                                1.0 / c.hx, 1.0 / c.hy, c.c, c.dt,
+                                                                qmc, bz_ext, ex, ey, bz);
+  RP_CHECK_LAUNCH();
+  return RP_OK;
+}

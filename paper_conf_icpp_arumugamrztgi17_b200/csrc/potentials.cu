@@ -1,0 +1,783 @@
+// potentials.cu -- step 2 of the paper's loop: retarded potentials at every grid point
+// (Eq. 1-2; Algorithm 1 COMPUTE-POTENTIALS), B200-native.
+//
+// Kernels (one launch each per call):
+//   k_clip       one thread per (point p, subregion j): support clip [A, B] of S_j (R-5),
+//                bit-identical to the oracle (IEEE _rn intrinsics, no contraction); emits the
+//                scheduling key from the previous step's segment count (the forecast g of
+//                P:85-95 used for scheduling only; LPT order).
+//   CUB sort     (key, item) -> longest-predicted-first order.
+//   k_integrate  persistent warps pull (p, j) items; each warp walks the canonical dyadic
+//                GK15 tree of its item depth-first without a stack (R-8..R-12).  Per
+//                segment lanes 0..14 build the 15 r' nodes (retarded frame, circle/support
+//                arcs, R-5/R-7), then all 32 lanes sweep the flattened (node, arc, theta)
+//                evaluations of f (27-point TSC x Lagrange-3 gather, R-6) and reduce with
+//                xor shuffles, so every accept/split decision is warp-uniform.
+//   k_reduce     per point, sum the items in j order -> phi, A, err, nseg; counts.
+// FP64 throughout.  No tensor cores: the work is an irregular gather stencil,
+// not a dense contraction.
+#include <cub/device/device_radix_sort.cuh>
+#include <math.h>
+
+#include "rp_internal.cuh"
+
+int rp_ensure_cub_tmp(rp_ctx* ctx, size_t bytes);
+
+namespace {
+
+// QUADPACK qk15 nodes / Kronrod weights / Gauss-7 weights (R-8)
+__constant__ double c_xgk[8] = {
+    0.991455371120812639206854697526329, 0.949107912342758524526189684047851,
+    0.864864423359769072789712788640926, 0.741531185599394439863864773280788,
+    0.586087235467691130294144845693013, 0.405845151377397166906606412076961,
+    0.207784955007898467600689403773245, 0.000000000000000000000000000000000};
+__constant__ double c_wgk[8] = {
+    0.022935322010529224963732008058970, 0.063092092629978553290700663189204,
+    0.104790010322250183839876322541518, 0.140653259715525918745189590510238,
+    0.169004726639267902826583426598550, 0.190350578064785409913256402421014,
+    0.204432940075298892414161999234649, 0.209482141084727828012999174891714};
+__constant__ double c_wg[4] = {
+    0.129484966168869693270611432679082, 0.279705391489276667901467771423780,
+    0.381830050505118944950369775488975, 0.417959183673469387755102040816327};
+
+enum : int { C_ITEMS = 0, C_NEXT = 1, C_EVALS = 2, C_SEGS = 3, C_LEAVES = 4, C_CAPPED = 5,
+             C_TIES = 6, C_MAXLEV = 7, C_NODES = 8, C_NOUT = 9, C_COUNT = 16 };
+
+constexpr double kTwoPi = 6.283185307179586476925286766559;
+constexpr int kMaxArcs = 8;
+constexpr int kWarps = 4;  // warps per CTA of k_integrate
+
+struct Params {
+  int nx, ny, PX, npts, kmax, kap, k, H, n_theta, max_depth, n_root;
+  double hx, hy, inv_hx, inv_hy, cdt, tau, R;
+  size_t slot_doubles;
+  const double* ring;        // padded ring, slot 0 node (-PAD, -PAD)
+  const rp_frame* frames;    // [H]
+  const double* amp;         // [H] analytic amplitudes
+  // analytic source
+  double sx0, sy0, swidth, sq, sbx, sby;
+};
+
+struct Item {
+  double px, py;              // mesh point, lab
+  int j;
+  rp_frame F0, F1, F2;        // frames of levels k-j-2, k-j-1, k-j
+  const double* g0;           // level grids at padded node (0, 0)
+  const double* g1;
+  const double* g2;
+  double a0, a1, a2;          // analytic amplitudes
+  double U0, U1, V0, V1;      // rectangle support (grid / gauss), frame-local
+};
+
+// ------------------------------------------------------------- bit-exact geometry
+// These mirror the arithmetic order of the definition with IEEE
+// round-to-nearest intrinsics so clip limits and segment endpoints are reproducible.
+__device__ __forceinline__ void lag3(double t, double& w0, double& w1, double& w2) {
+  w0 = __dmul_rn(__dmul_rn(0.5, t), __dsub_rn(t, 1.0));
+  w1 = __dsub_rn(1.0, __dmul_rn(t, t));
+  w2 = __dmul_rn(__dmul_rn(0.5, t), __dadd_rn(t, 1.0));
+}
+
+__device__ __forceinline__ double lerp3(double x0, double x1, double x2, double w0, double w2) {
+  return __dadd_rn(__dadd_rn(x1, __dmul_rn(w0, __dsub_rn(x0, x1))), __dmul_rn(w2, __dsub_rn(x2, x1)));
+}
+
+// frame-local centre of the circle about p at the retarded time of radius r (R-7)
+__device__ __forceinline__ void centre_at(const Item& it, const Params& P, double r, double& cu,
+                                          double& cv, double& w0, double& w1, double& w2) {
+  double t = __dsub_rn((double)(it.j + 1), __ddiv_rn(r, P.cdt));
+  lag3(t, w0, w1, w2);
+  double ox = lerp3(it.F0.ox, it.F1.ox, it.F2.ox, w0, w2);
+  double oy = lerp3(it.F0.oy, it.F1.oy, it.F2.oy, w0, w2);
+  double c = lerp3(it.F0.cos_psi, it.F1.cos_psi, it.F2.cos_psi, w0, w2);
+  double s = lerp3(it.F0.sin_psi, it.F1.sin_psi, it.F2.sin_psi, w0, w2);
+  double dx = __dsub_rn(it.px, ox), dy = __dsub_rn(it.py, oy);
+  cu = __dadd_rn(__dmul_rn(c, dx), __dmul_rn(s, dy));
+  cv = __dadd_rn(__dmul_rn(-s, dx), __dmul_rn(c, dy));
+}
+
+template <int KIND>
+__device__ __forceinline__ void support_d2(const Item& it, const Params& P, double cu, double cv,
+                                           double& dmin2, double& dmax2) {
+  if (KIND == RP_SRC_DISK) {
+    double ex = __dsub_rn(cu, P.sx0), ey = __dsub_rn(cv, P.sy0);
+    double s = __dsqrt_rn(__dadd_rn(__dmul_rn(ex, ex), __dmul_rn(ey, ey)));
+    double lo = __dsub_rn(s, P.swidth);
+    lo = lo > 0.0 ? lo : 0.0;
+    double hi = __dadd_rn(s, P.swidth);
+    dmin2 = __dmul_rn(lo, lo);
+    dmax2 = __dmul_rn(hi, hi);
+    return;
+  }
+  double ex = 0.0, ey = 0.0;
+  if (cu < it.U0) ex = __dsub_rn(it.U0, cu); else if (cu > it.U1) ex = __dsub_rn(cu, it.U1);
+  if (cv < it.V0) ey = __dsub_rn(it.V0, cv); else if (cv > it.V1) ey = __dsub_rn(cv, it.V1);
+  dmin2 = __dadd_rn(__dmul_rn(ex, ex), __dmul_rn(ey, ey));
+  double a = fabs(__dsub_rn(cu, it.U0)), b = fabs(__dsub_rn(cu, it.U1));
+  double fx = a > b ? a : b;
+  a = fabs(__dsub_rn(cv, it.V0));
+  b = fabs(__dsub_rn(cv, it.V1));
+  double fy = a > b ? a : b;
+  dmax2 = __dadd_rn(__dmul_rn(fx, fx), __dmul_rn(fy, fy));
+}
+
+template <int KIND>
+__device__ __forceinline__ void dists_at(const Item& it, const Params& P, double r, double& dmin2,
+                                         double& dmax2) {
+  double cu, cv, w0, w1, w2;
+  centre_at(it, P, r, cu, cv, w0, w1, w2);
+  support_d2<KIND>(it, P, cu, cv, dmin2, dmax2);
+}
+
+template <int KIND>
+__device__ void setup_item(Item& it, const Params& P, int p, int j) {
+  int ix = p % P.nx, iy = p / P.nx;
+  const rp_frame Fk = P.frames[slot_of_dev(P.k, P.H)];
+  double u = __dmul_rn((double)ix, P.hx), v = __dmul_rn((double)iy, P.hy);
+  it.px = __dsub_rn(__dadd_rn(Fk.ox, __dmul_rn(u, Fk.cos_psi)), __dmul_rn(v, Fk.sin_psi));
+  it.py = __dadd_rn(__dadd_rn(Fk.oy, __dmul_rn(u, Fk.sin_psi)), __dmul_rn(v, Fk.cos_psi));
+  it.j = j;
+  int s0 = slot_of_dev(P.k - j - 2, P.H), s1 = slot_of_dev(P.k - j - 1, P.H),
+      s2 = slot_of_dev(P.k - j, P.H);
+  it.F0 = P.frames[s0];
+  it.F1 = P.frames[s1];
+  it.F2 = P.frames[s2];
+  size_t off = (size_t)4 * (RP_PAD * P.PX + RP_PAD);
+  it.g0 = P.ring + (size_t)s0 * P.slot_doubles + off;
+  it.g1 = P.ring + (size_t)s1 * P.slot_doubles + off;
+  it.g2 = P.ring + (size_t)s2 * P.slot_doubles + off;
+  if (KIND != RP_SRC_GRID) {
+    it.a0 = P.amp[s0];
+    it.a1 = P.amp[s1];
+    it.a2 = P.amp[s2];
+  } else {
+    it.a0 = it.a1 = it.a2 = 1.0;
+  }
+  if (KIND == RP_SRC_GAUSS) {
+    double w8 = __dmul_rn(8.0, P.swidth);
+    it.U0 = __dsub_rn(P.sx0, w8); it.U1 = __dadd_rn(P.sx0, w8);
+    it.V0 = __dsub_rn(P.sy0, w8); it.V1 = __dadd_rn(P.sy0, w8);
+  } else {
+    it.U0 = __dmul_rn(-1.5, P.hx);
+    it.U1 = __dmul_rn(__dadd_rn((double)P.nx, 0.5), P.hx);
+    it.V0 = __dmul_rn(-1.5, P.hy);
+    it.V1 = __dmul_rn(__dadd_rn((double)P.ny, 0.5), P.hy);
+  }
+}
+
+// ------------------------------------------------------------- k_clip
+template <int KIND>
+__global__ void k_clip(Params P, const int32_t* __restrict__ owner, int rank,
+                       const uint16_t* __restrict__ cost_prev, double2* __restrict__ AB,
+                       uint16_t* __restrict__ key, int32_t* __restrict__ iota,
+                       unsigned long long* __restrict__ counters) {
+  int64_t id = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+  int64_t total = (int64_t)P.npts * P.kmax;
+  if (id >= total) return;
+  iota[id] = (int32_t)id;
+  int p = (int)(id / P.kmax), j = (int)(id % P.kmax);
+  uint16_t kk = 0xFFFF;
+  double A = 0.0, B = 0.0;
+  if (j < P.kap && (owner == nullptr || owner[p] == rank)) {
+    Item it;
+    setup_item<KIND>(it, P, p, j);
+    double a = __dmul_rn((double)j, P.cdt), b = __dmul_rn((double)(j + 1), P.cdt);
+    double dmn, dmx;
+    bool empty = false;
+    dists_at<KIND>(it, P, b, dmn, dmx);
+    if (dmn > __dmul_rn(b, b)) empty = true;
+    if (!empty) {
+      dists_at<KIND>(it, P, a, dmn, dmx);
+      if (dmx < __dmul_rn(a, a)) empty = true;
+    }
+    if (!empty) {
+      if (dmn <= __dmul_rn(a, a)) {
+        A = a;
+      } else {
+        double lo = a, hi = b;
+        for (int t = 0; t < 64; ++t) {
+          double m = __dmul_rn(0.5, __dadd_rn(lo, hi));
+          dists_at<KIND>(it, P, m, dmn, dmx);
+          if (dmn <= __dmul_rn(m, m)) hi = m; else lo = m;
+        }
+        A = hi;
+      }
+      dists_at<KIND>(it, P, b, dmn, dmx);
+      if (dmx >= __dmul_rn(b, b)) {
+        B = b;
+      } else {
+        double lo = a, hi = b;
+        for (int t = 0; t < 64; ++t) {
+          double m = __dmul_rn(0.5, __dadd_rn(lo, hi));
+          dists_at<KIND>(it, P, m, dmn, dmx);
+          if (dmx >= __dmul_rn(m, m)) lo = m; else hi = m;
+        }
+        B = lo;
+      }
+      if (A < B) {
+        unsigned c = cost_prev ? cost_prev[id] : 0u;
+        kk = (uint16_t)(0xFFFEu - (c < 0xFFFEu ? c : 0xFFFEu));
+      }
+    }
+  }
+  AB[id] = make_double2(A, B);
+  key[id] = kk;
+  // count items: warp aggregate then one atomic per warp (integer -> deterministic)
+  unsigned m = __ballot_sync(__activemask(), kk != 0xFFFF);
+  if ((threadIdx.x & 31) == (__ffs(__activemask()) - 1) && m)
+    atomicAdd(&counters[C_ITEMS], (unsigned long long)__popc(m));
+}
+
+// ------------------------------------------------------------- integrand
+template <int KIND>
+__device__ __forceinline__ void integrand(const Item& it, const Params& P, double u, double v,
+                                          double w0, double w1, double w2, double& f0,
+                                          double& f1, double& f2) {
+  if (KIND == RP_SRC_GRID) {
+    double tx = u * P.inv_hx, ty = v * P.inv_hy;
+    double fx = floor(tx + 0.5), fy = floor(ty + 0.5);
+    double dx = tx - fx, dy = ty - fy;
+    double ax = 0.5 - dx, bx = 0.5 + dx, ay = 0.5 - dy, by = 0.5 + dy;
+    double wx0 = 0.5 * ax * ax, wx1 = 0.75 - dx * dx, wx2 = 0.5 * bx * bx;
+    double wy0 = 0.5 * ay * ay, wy1 = 0.75 - dy * dy, wy2 = 0.5 * by * by;
+    // clamp keeps every stencil inside the zero border (points outside the support
+    // rectangle never reach here; the clamp only guards memory)
+    int ix = (int)fmin(fmax(fx, -2.0), (double)(P.nx + 1));
+    int iy = (int)fmin(fmax(fy, -2.0), (double)(P.ny + 1));
+    size_t base = (size_t)4 * ((iy - 1) * P.PX + (ix - 1));
+    double s[3][3];
+#pragma unroll
+    for (int l = 0; l < 3; ++l) { s[l][0] = 0.0; s[l][1] = 0.0; s[l][2] = 0.0; }
+    const double wxa[3] = {wx0, wx1, wx2};
+    const double wyb[3] = {wy0, wy1, wy2};
+#pragma unroll
+    for (int b = 0; b < 3; ++b) {
+#pragma unroll
+      for (int a = 0; a < 3; ++a) {
+        double w = wxa[a] * wyb[b];
+        size_t o = base + (size_t)4 * (b * P.PX + a);
+        double2 m0 = __ldg(reinterpret_cast<const double2*>(it.g0 + o));
+        double z0 = __ldg(it.g0 + o + 2);
+        double2 m1 = __ldg(reinterpret_cast<const double2*>(it.g1 + o));
+        double z1 = __ldg(it.g1 + o + 2);
+        double2 m2 = __ldg(reinterpret_cast<const double2*>(it.g2 + o));
+        double z2 = __ldg(it.g2 + o + 2);
+        s[0][0] += w * m0.x; s[0][1] += w * m0.y; s[0][2] += w * z0;
+        s[1][0] += w * m1.x; s[1][1] += w * m1.y; s[1][2] += w * z1;
+        s[2][0] += w * m2.x; s[2][1] += w * m2.y; s[2][2] += w * z2;
+      }
+    }
+    f0 = w0 * s[0][0] + w1 * s[1][0] + w2 * s[2][0];
+    f1 = w0 * s[0][1] + w1 * s[1][1] + w2 * s[2][1];
+    f2 = w0 * s[0][2] + w1 * s[1][2] + w2 * s[2][2];
+    return;
+  }
+  double amp = w0 * it.a0 + w1 * it.a1 + w2 * it.a2;
+  double rho;
+  if (KIND == RP_SRC_GAUSS) {
+    double ex = u - P.sx0, ey = v - P.sy0, sg = P.swidth;
+    rho = P.sq / (kTwoPi * sg * sg) * exp(-(ex * ex + ey * ey) / (2.0 * sg * sg));
+  } else {
+    rho = P.sq;
+  }
+  rho *= amp;
+  f0 = rho;
+  f1 = rho * P.sbx;
+  f2 = rho * P.sby;
+}
+
+// ------------------------------------------------------------- arcs (R-5)
+__device__ __forceinline__ bool in_rect(double u, double v, const Item& it) {
+  return u >= it.U0 && u <= it.U1 && v >= it.V0 && v <= it.V1;
+}
+
+__device__ __forceinline__ void cswap(double& a, double& b) {
+  double lo = fmin(a, b), hi = fmax(a, b);
+  a = lo;
+  b = hi;
+}
+
+// arcs of circle (cu, cv; r) inside the support; returns -1 (full circle) or the count,
+// writing (theta1, dtheta = (theta2 - theta1) / N) pairs.
+template <int KIND>
+__device__ int arcs(const Item& it, const Params& P, double cu, double cv, double r,
+                    double* th1, double* dth) {
+  const double N = (double)P.n_theta;
+  if (KIND == RP_SRC_DISK) {
+    double ex = P.sx0 - cu, ey = P.sy0 - cv;
+    double s = sqrt(ex * ex + ey * ey), a = P.swidth;
+    if (s + r <= a) return -1;
+    if (r >= s + a || s >= r + a) return 0;
+    double ph = atan2(ey, ex);
+    double al = acos((r * r + s * s - a * a) / (2.0 * r * s));
+    th1[0] = ph - al;
+    dth[0] = ((ph + al) - (ph - al)) / N;
+    return 1;
+  }
+  const double inf = __longlong_as_double(0x7ff0000000000000LL);
+  double t[8];
+#pragma unroll
+  for (int i = 0; i < 8; ++i) t[i] = inf;
+  {
+    double d = (it.U0 - cu) / r;
+    if (fabs(d) < 1.0) {
+      double al = acos(d), c2 = kTwoPi - al;
+      double v1 = cv + r * sin(al), v2 = cv + r * sin(c2);
+      if (v1 >= it.V0 && v1 <= it.V1) t[0] = al;
+      if (v2 >= it.V0 && v2 <= it.V1) t[1] = c2;
+    }
+    d = (it.U1 - cu) / r;
+    if (fabs(d) < 1.0) {
+      double al = acos(d), c2 = kTwoPi - al;
+      double v1 = cv + r * sin(al), v2 = cv + r * sin(c2);
+      if (v1 >= it.V0 && v1 <= it.V1) t[2] = al;
+      if (v2 >= it.V0 && v2 <= it.V1) t[3] = c2;
+    }
+    d = (it.V0 - cv) / r;
+    if (fabs(d) < 1.0) {
+      double be = asin(d);
+      double c1 = be < 0.0 ? be + kTwoPi : be, c2 = M_PI - be;
+      double u1 = cu + r * cos(c1), u2 = cu + r * cos(c2);
+      if (u1 >= it.U0 && u1 <= it.U1) t[4] = c1;
+      if (u2 >= it.U0 && u2 <= it.U1) t[5] = c2;
+    }
+    d = (it.V1 - cv) / r;
+    if (fabs(d) < 1.0) {
+      double be = asin(d);
+      double c1 = be < 0.0 ? be + kTwoPi : be, c2 = M_PI - be;
+      double u1 = cu + r * cos(c1), u2 = cu + r * cos(c2);
+      if (u1 >= it.U0 && u1 <= it.U1) t[6] = c1;
+      if (u2 >= it.U0 && u2 <= it.U1) t[7] = c2;
+    }
+  }
+  // sorting network (19 comparators) on 8 keys, +inf = absent
+  cswap(t[0], t[1]); cswap(t[2], t[3]); cswap(t[4], t[5]); cswap(t[6], t[7]);
+  cswap(t[0], t[2]); cswap(t[1], t[3]); cswap(t[4], t[6]); cswap(t[5], t[7]);
+  cswap(t[1], t[2]); cswap(t[5], t[6]); cswap(t[0], t[4]); cswap(t[3], t[7]);
+  cswap(t[1], t[5]); cswap(t[2], t[6]);
+  cswap(t[1], t[4]); cswap(t[3], t[6]);
+  cswap(t[2], t[4]); cswap(t[3], t[5]);
+  cswap(t[3], t[4]);
+  if (t[0] == inf) return in_rect(cu + r, cv, it) ? -1 : 0;
+  // unique crossings u_0 < u_1 < ... ; intervals (u_i, u_{i+1}) and (u_last, u_0 + 2 pi)
+  int na = 0;
+  double first = t[0], prev = t[0];
+#pragma unroll
+  for (int i = 1; i < 8; ++i) {
+    double cur = t[i];
+    if (cur != inf && cur != prev) {
+      double mid = 0.5 * (prev + cur);
+      double sm, cm;
+      sincos(mid, &sm, &cm);
+      if (in_rect(cu + r * cm, cv + r * sm, it)) {
+        th1[na] = prev;
+        dth[na] = (cur - prev) / N;
+        ++na;
+      }
+      prev = cur;
+    }
+  }
+  {
+    double cur = first + kTwoPi;
+    double mid = 0.5 * (prev + cur);
+    double sm, cm;
+    sincos(mid, &sm, &cm);
+    if (in_rect(cu + r * cm, cv + r * sm, it)) {
+      th1[na] = prev;
+      dth[na] = (cur - prev) / N;
+      ++na;
+    }
+  }
+  return na;
+}
+
+// ------------------------------------------------------------- k_integrate
+struct WarpSmem {
+  double r[16], cu[16], cv[16], w0[16], w1[16], w2[16], wk[16], wg[16];
+  double th1[16][kMaxArcs], dth[16][kMaxArcs];
+  int na[16], off[17];
+};
+
+__device__ __forceinline__ double warp_sum(double v) {
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);
+  return v;
+}
+
+template <int KIND>
+__global__ void __launch_bounds__(32 * kWarps) k_integrate(
+    Params P, const int32_t* __restrict__ order, const double2* __restrict__ AB,
+    const double2* __restrict__ trig_full, double4* __restrict__ item_val,
+    int4* __restrict__ item_cnt, uint2* __restrict__ item_aux,
+    unsigned long long* __restrict__ counters) {
+  __shared__ WarpSmem smem[kWarps];
+  const int lane = threadIdx.x & 31;
+  WarpSmem& S = smem[threadIdx.x >> 5];
+  const unsigned long long n_items = counters[C_ITEMS];
+  const int N = P.n_theta;
+  const double Nd = (double)N;
+  const double wfull = kTwoPi / Nd;
+  const double third = 1.0 / 3.0;
+  for (;;) {
+    unsigned long long idx = 0;
+    if (lane == 0) idx = atomicAdd(&counters[C_NEXT], 1ULL);
+    idx = __shfl_sync(0xffffffffu, idx, 0);
+    if (idx >= n_items) break;
+    const int item = order[idx];
+    const int p = item / P.kmax, j = item % P.kmax;
+    const double2 ab = AB[item];
+    const double A = ab.x, BA = __dsub_rn(ab.y, ab.x);
+    Item it;
+    setup_item<KIND>(it, P, p, j);
+
+    double s_phi = 0.0, s_ax = 0.0, s_ay = 0.0, s_err = 0.0;
+    int nseg = 0, nleaf = 0, capped = 0, ties = 0, maxlev = 0;
+    unsigned evals = 0;
+    int lev = P.n_root == 2 ? 1 : 0;
+    long long ix = 0;
+    for (;;) {
+      const double fa = ldexp((double)ix, -lev), fb = ldexp((double)(ix + 1), -lev);
+      const double a = __dadd_rn(A, __dmul_rn(BA, fa)), b = __dadd_rn(A, __dmul_rn(BA, fb));
+      const double m = __dmul_rn(0.5, __dadd_rn(a, b)), hw = __dmul_rn(0.5, __dsub_rn(b, a));
+      // ---- node phase: lanes 0..14 build the r' nodes of the GK15 rule
+      int cnt = 0;
+      if (lane < 15) {
+        const int i = lane < 7 ? lane : (lane == 7 ? 7 : 14 - lane);
+        double r;
+        if (lane < 7) r = __dsub_rn(m, __dmul_rn(hw, c_xgk[i]));
+        else if (lane == 7) r = m;
+        else r = __dadd_rn(m, __dmul_rn(hw, c_xgk[i]));
+        double cu, cv, w0, w1, w2;
+        centre_at(it, P, r, cu, cv, w0, w1, w2);
+        double th1[kMaxArcs], dth[kMaxArcs];
+        int na = arcs<KIND>(it, P, cu, cv, r, th1, dth);
+        S.r[lane] = r; S.cu[lane] = cu; S.cv[lane] = cv;
+        S.w0[lane] = w0; S.w1[lane] = w1; S.w2[lane] = w2;
+        S.wk[lane] = hw * c_wgk[i];
+        S.wg[lane] = (i & 1) ? hw * c_wg[i >> 1] : (i == 7 ? hw * c_wg[3] : 0.0);
+        S.na[lane] = na;
+        for (int q = 0; q < (na > 0 ? na : 0); ++q) {
+          S.th1[lane][q] = th1[q];
+          S.dth[lane][q] = dth[q];
+        }
+        cnt = na < 0 ? N : na * (N + 1);
+      }
+      // inclusive scan of counts over lanes -> exclusive node offsets
+      int incl = cnt;
+#pragma unroll
+      for (int o = 1; o < 32; o <<= 1) {
+        int y = __shfl_up_sync(0xffffffffu, incl, o);
+        if (lane >= o) incl += y;
+      }
+      if (lane < 15) S.off[lane] = incl - cnt;
+      const int E = __shfl_sync(0xffffffffu, incl, 31);
+      if (lane == 15) S.off[15] = E;
+      __syncwarp();
+      // ---- evaluation phase: all lanes sweep the flattened (node, arc, theta) list
+      double k0 = 0.0, k1 = 0.0, k2 = 0.0, g0 = 0.0, g1 = 0.0, g2 = 0.0;
+      int n = 0;
+      for (int e = lane; e < E; e += 32) {
+        while (e >= S.off[n + 1]) ++n;
+        const int local = e - S.off[n];
+        const int na = S.na[n];
+        double cs, sn, w;
+        if (na < 0) {
+          const double2 t = trig_full[local];
+          cs = t.x;
+          sn = t.y;
+          w = wfull;
+        } else {
+          const int q = local / (N + 1);
+          const int mm = local - q * (N + 1);
+          const double d = S.dth[n][q];
+          sincos(S.th1[n][q] + (double)mm * d, &sn, &cs);
+          const double coef = (mm == 0 || mm == N) ? 1.0 : ((mm & 1) ? 4.0 : 2.0);
+          w = coef * d * third;
+        }
+        const double r = S.r[n];
+        double f0, f1, f2;
+        integrand<KIND>(it, P, S.cu[n] + r * cs, S.cv[n] + r * sn, S.w0[n], S.w1[n], S.w2[n],
+                        f0, f1, f2);
+        const double wk = w * S.wk[n], wg = w * S.wg[n];
+        k0 += wk * f0; k1 += wk * f1; k2 += wk * f2;
+        g0 += wg * f0; g1 += wg * f1; g2 += wg * f2;
+      }
+      k0 = warp_sum(k0); k1 = warp_sum(k1); k2 = warp_sum(k2);
+      g0 = warp_sum(g0); g1 = warp_sum(g1); g2 = warp_sum(g2);
+      __syncwarp();
+      evals += (unsigned)E;
+      ++nseg;
+      if (lev > maxlev) maxlev = lev;
+      double err = fabs(k0 - g0);
+      err = fmax(err, fabs(k1 - g1));
+      err = fmax(err, fabs(k2 - g2));
+      const double tol = __ddiv_rn(__dmul_rn(P.tau, ldexp(BA, -lev)), P.R);
+      if (fabs(err - tol) / tol < 1e-9) ++ties;
+      if (err <= tol || lev >= P.max_depth) {
+        if (!(err <= tol)) ++capped;
+        ++nleaf;
+        s_phi += k0; s_ax += k1; s_ay += k2; s_err += err;
+        while ((ix & 1) && lev > 0) { ix >>= 1; --lev; }
+        if (lev == 0) break;
+        ++ix;
+      } else {
+        ++lev;
+        ix <<= 1;
+      }
+    }
+    if (lane == 0) {
+      item_val[item] = make_double4(s_phi, s_ax, s_ay, s_err);
+      item_cnt[item] = make_int4(nseg, nleaf, capped, ties);
+      item_aux[item] = make_uint2((unsigned)maxlev, evals);
+    }
+  }
+}
+
+// ------------------------------------------------------------- k_reduce
+__global__ void k_reduce(int npts, int kmax, int kap, const uint16_t* __restrict__ key,
+                         const double4* __restrict__ val, const int4* __restrict__ cnt,
+                         const uint2* __restrict__ aux, const int32_t* __restrict__ owner,
+                         int rank, const int32_t* __restrict__ row_of, int world,
+                         double* __restrict__ phi, double* __restrict__ ax,
+                         double* __restrict__ ay, double* __restrict__ err,
+                         int32_t* __restrict__ nseg, double* __restrict__ shard,
+                         uint16_t* __restrict__ cost, int32_t* __restrict__ nseg_pt,
+                         unsigned long long* __restrict__ counters) {
+  int p = blockIdx.x * blockDim.x + threadIdx.x;
+  if (p >= npts) return;
+  if (owner && owner[p] != rank) return;
+  double a = 0.0, b = 0.0, c = 0.0, e = 0.0;
+  long long ns = 0, nl = 0, cp = 0, ti = 0, ev = 0;
+  int ml = 0;
+  for (int j = 0; j < kmax; ++j) {
+    size_t id = (size_t)p * kmax + j;
+    if (j >= kap || key[id] == 0xFFFF) {
+      cost[id] = 0;
+      continue;
+    }
+    double4 v = val[id];
+    int4 q = cnt[id];
+    uint2 x = aux[id];
+    a += v.x; b += v.y; c += v.z; e += v.w;
+    ns += q.x; nl += q.y; cp += q.z; ti += q.w;
+    ev += x.y;
+    if ((int)x.x > ml) ml = (int)x.x;
+    cost[id] = (uint16_t)(q.x < 0xFFFE ? q.x : 0xFFFE);
+  }
+  if (shard) {
+    double* r = shard + 6 * (size_t)row_of[p];
+    r[0] = (double)p; r[1] = a; r[2] = b; r[3] = c; r[4] = e; r[5] = (double)ns;
+  } else {
+    phi[p] = a;
+    ax[p] = b;
+    ay[p] = c;
+    if (err) err[p] = e;
+    if (nseg) nseg[p] = (int32_t)ns;
+    nseg_pt[p] = (int32_t)ns;
+  }
+  atomicAdd(&counters[C_SEGS], (unsigned long long)ns);
+  atomicAdd(&counters[C_LEAVES], (unsigned long long)nl);
+  atomicAdd(&counters[C_CAPPED], (unsigned long long)cp);
+  atomicAdd(&counters[C_TIES], (unsigned long long)ti);
+  atomicAdd(&counters[C_EVALS], (unsigned long long)ev);
+  atomicMax(&counters[C_MAXLEV], (unsigned long long)ml);
+  atomicAdd(&counters[C_NOUT], 1ULL);
+}
+
+// ------------------------------------------------------------- shard map
+__global__ void k_point_keys(int npts, const int32_t* __restrict__ nseg_pt, int have,
+                             int32_t* __restrict__ key, int32_t* __restrict__ idx) {
+  int p = blockIdx.x * blockDim.x + threadIdx.x;
+  if (p >= npts) return;
+  int w = have ? nseg_pt[p] : 0;
+  key[p] = 0x7fffffff - (w < 0 ? 0 : w);  // ascending key = descending predicted work
+  idx[p] = p;
+}
+
+__global__ void k_owner(int npts, int world, const int32_t* __restrict__ order,
+                        int32_t* __restrict__ owner, int32_t* __restrict__ row) {
+  int i = blockIdx.x * blockDim.x + threadIdx.x;
+  if (i >= npts) return;
+  int b = i / world, r = i % world;
+  int rank = (b & 1) ? world - 1 - r : r;  // snake deal: longest-first, balanced
+  int p = order[i];
+  owner[p] = rank;
+  row[p] = b;
+}
+
+__global__ void k_scatter(int npts, int world, int64_t cap, const double* __restrict__ sh,
+                          double* __restrict__ phi, double* __restrict__ ax,
+                          double* __restrict__ ay, double* __restrict__ err,
+                          int32_t* __restrict__ nseg, int32_t* __restrict__ nseg_pt) {
+  int64_t t = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+  if (t >= (int64_t)world * cap) return;
+  int r = (int)(t / cap);
+  int64_t b = t % cap;
+  int64_t i = b * world + ((b & 1) ? world - 1 - r : r);
+  if (i >= npts) return;
+  const double* rec = sh + 6 * t;
+  int p = (int)rec[0];
+  phi[p] = rec[1];
+  ax[p] = rec[2];
+  ay[p] = rec[3];
+  if (err) err[p] = rec[4];
+  int ns = (int)rec[5];
+  if (nseg) nseg[p] = ns;
+  nseg_pt[p] = ns;
+}
+
+}  // namespace
+
+int rp_alloc_potential_scratch(rp_ctx* ctx) {
+  const rp_config& c = ctx->cfg;
+  size_t npts = (size_t)c.nx * c.ny, nd = npts * c.history_depth;
+  RP_CUDA(cudaMalloc(&ctx->clipAB, nd * sizeof(double2)));
+  RP_CUDA(cudaMalloc(&ctx->sched_key, nd * sizeof(uint16_t)));
+  RP_CUDA(cudaMalloc(&ctx->sched_key_sorted, nd * sizeof(uint16_t)));
+  RP_CUDA(cudaMalloc(&ctx->sched_idx, nd * sizeof(int32_t)));
+  RP_CUDA(cudaMalloc(&ctx->sched_order, nd * sizeof(int32_t)));
+  RP_CUDA(cudaMalloc(&ctx->cost_prev, nd * sizeof(uint16_t)));
+  RP_CUDA(cudaMemset(ctx->cost_prev, 0, nd * sizeof(uint16_t)));
+  RP_CUDA(cudaMalloc(&ctx->item_val, nd * sizeof(double4)));
+  RP_CUDA(cudaMalloc(&ctx->item_cnt, nd * sizeof(int4)));
+  RP_CUDA(cudaMalloc(&ctx->item_aux, nd * sizeof(uint2)));
+  RP_CUDA(cudaMalloc(&ctx->counters, 16 * sizeof(unsigned long long)));
+  RP_CUDA(cudaMalloc(&ctx->amp_dev, ctx->H * sizeof(double)));
+  RP_CUDA(cudaMalloc(&ctx->point_key, npts * sizeof(int32_t)));
+  RP_CUDA(cudaMalloc(&ctx->point_key_sorted, npts * sizeof(int32_t)));
+  RP_CUDA(cudaMalloc(&ctx->point_idx, npts * sizeof(int32_t)));
+  RP_CUDA(cudaMalloc(&ctx->point_order, npts * sizeof(int32_t)));
+  RP_CUDA(cudaMalloc(&ctx->point_owner, npts * sizeof(int32_t)));
+  RP_CUDA(cudaMalloc(&ctx->nseg_prev_pt, npts * sizeof(int32_t)));
+  RP_CUDA(cudaMemset(ctx->nseg_prev_pt, 0, npts * sizeof(int32_t)));
+  // full-circle trapezoid nodes (cos, sin)(m * 2 pi / N), R-11
+  double2* h = new double2[c.n_theta];
+  for (int m = 0; m < c.n_theta; ++m) {
+    double th = (double)m * (2.0 * M_PI / c.n_theta);
+    h[m] = make_double2(cos(th), sin(th));
+  }
+  cudaError_t e = cudaMalloc(&ctx->trig_full, c.n_theta * sizeof(double2));
+  if (e == cudaSuccess) e = cudaMemcpy(ctx->trig_full, h, c.n_theta * sizeof(double2), cudaMemcpyHostToDevice);
+  delete[] h;
+  RP_CUDA(e);
+  return RP_OK;
+}
+
+template <int KIND>
+static int run_potentials(rp_ctx* ctx, const Params& P, int32_t rank, int32_t world,
+                          double* phi, double* ax, double* ay, double* err, int32_t* nseg,
+                          double* shard_out, int64_t cap) {
+  cudaStream_t st = ctx->stream;
+  const int64_t nd = (int64_t)P.npts * P.kmax;
+  const int32_t* owner = nullptr;
+  int32_t* row = nullptr;
+  if (shard_out) {
+    // shard map from the previous step's per-point counts (identical on every rank)
+    k_point_keys<<<(P.npts + 255) / 256, 256, 0, st>>>(P.npts, ctx->nseg_prev_pt,
+                                                        ctx->has_forecast, ctx->point_key,
+                                                        ctx->point_idx);
+    RP_CHECK_LAUNCH();
+    size_t tmp = 0;
+    RP_CUDA(cub::DeviceRadixSort::SortPairs(nullptr, tmp, ctx->point_key, ctx->point_key_sorted,
+                                            ctx->point_idx, ctx->point_order, P.npts, 0, 32, st));
+    int rc = rp_ensure_cub_tmp(ctx, tmp);
+    if (rc) return rc;
+    tmp = ctx->cub_tmp_bytes;
+    RP_CUDA(cub::DeviceRadixSort::SortPairs(ctx->cub_tmp, tmp, ctx->point_key,
+                                            ctx->point_key_sorted, ctx->point_idx,
+                                            ctx->point_order, P.npts, 0, 32, st));
+    k_owner<<<(P.npts + 255) / 256, 256, 0, st>>>(P.npts, world, ctx->point_order,
+                                                   ctx->point_owner, ctx->point_key);
+    RP_CHECK_LAUNCH();
+    owner = ctx->point_owner;
+    row = ctx->point_key;  // reused as row index
+    RP_CUDA(cudaMemsetAsync(shard_out, 0, (size_t)cap * 6 * sizeof(double), st));
+  }
+  RP_CUDA(cudaMemsetAsync(ctx->counters, 0, 16 * sizeof(unsigned long long), st));
+  if (nd > 0) {
+    k_clip<KIND><<<(unsigned)((nd + 255) / 256), 256, 0, st>>>(
+        P, owner, rank, ctx->has_forecast ? ctx->cost_prev : nullptr, ctx->clipAB,
+        ctx->sched_key, ctx->sched_idx, ctx->counters);
+    RP_CHECK_LAUNCH();
+    size_t tmp = 0;
+    RP_CUDA(cub::DeviceRadixSort::SortPairs(nullptr, tmp, ctx->sched_key, ctx->sched_key_sorted,
+                                            ctx->sched_idx, ctx->sched_order, (int)nd, 0, 16, st));
+    int rc = rp_ensure_cub_tmp(ctx, tmp);
+    if (rc) return rc;
+    tmp = ctx->cub_tmp_bytes;
+    RP_CUDA(cub::DeviceRadixSort::SortPairs(ctx->cub_tmp, tmp, ctx->sched_key,
+                                            ctx->sched_key_sorted, ctx->sched_idx,
+                                            ctx->sched_order, (int)nd, 0, 16, st));
+    int occ = 0;
+    RP_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_integrate<KIND>, 32 * kWarps, 0));
+    if (occ < 1) occ = 1;
+    k_integrate<KIND><<<ctx->sm_count * occ, 32 * kWarps, 0, st>>>(
+        P, ctx->sched_order, ctx->clipAB, ctx->trig_full, ctx->item_val, ctx->item_cnt,
+        ctx->item_aux, ctx->counters);
+    RP_CHECK_LAUNCH();
+  }
+  k_reduce<<<(P.npts + 255) / 256, 256, 0, st>>>(
+      P.npts, P.kmax, P.kap, ctx->sched_key, ctx->item_val, ctx->item_cnt, ctx->item_aux, owner,
+      rank, row, world, phi, ax, ay, err, nseg, shard_out, ctx->cost_prev, ctx->nseg_prev_pt,
+      ctx->counters);
+  RP_CHECK_LAUNCH();
+  ctx->has_forecast = 1;
+  return RP_OK;
+}
+
+int rp_potentials_impl(rp_ctx* ctx, int kind, const double src[6], int32_t rank, int32_t world,
+                       double* phi, double* ax, double* ay, double* err, int32_t* nseg,
+                       double* shard_out, int64_t cap, int64_t* n_out, rp_potential_info* info) {
+  const rp_config& c = ctx->cfg;
+  if (ctx->k < 0) return rp_fail(ctx, RP_ESTATE, "potentials before the first deposit");
+  if (!shard_out && (!phi || !ax || !ay)) return rp_fail(ctx, RP_EINVAL, "potentials: null output");
+  Params P;
+  P.nx = c.nx; P.ny = c.ny; P.PX = ctx->PX; P.npts = c.nx * c.ny; P.kmax = c.history_depth;
+  P.kap = kappa_of(ctx); P.k = ctx->k; P.H = ctx->H; P.n_theta = c.n_theta;
+  P.max_depth = c.max_depth; P.n_root = c.n_root;
+  P.hx = c.hx; P.hy = c.hy; P.inv_hx = 1.0 / c.hx; P.inv_hy = 1.0 / c.hy;
+  P.cdt = c.c * c.dt; P.tau = c.tau; P.R = (double)P.kap * P.cdt;
+  P.slot_doubles = ctx->slot_doubles; P.ring = ctx->ring; P.frames = ctx->frames_dev;
+  P.amp = ctx->amp_dev;
+  P.sx0 = src ? src[0] : 0; P.sy0 = src ? src[1] : 0; P.swidth = src ? src[2] : 0;
+  P.sq = src ? src[3] : 0; P.sbx = src ? src[4] : 0; P.sby = src ? src[5] : 0;
+  int rc;
+  if (kind == RP_SRC_GRID)
+    rc = run_potentials<RP_SRC_GRID>(ctx, P, rank, world, phi, ax, ay, err, nseg, shard_out, cap);
+  else if (kind == RP_SRC_GAUSS)
+    rc = run_potentials<RP_SRC_GAUSS>(ctx, P, rank, world, phi, ax, ay, err, nseg, shard_out, cap);
+  else
+    rc = run_potentials<RP_SRC_DISK>(ctx, P, rank, world, phi, ax, ay, err, nseg, shard_out, cap);
+  if (rc) return rc;
+  if (info || n_out) {
+    unsigned long long h[16];
+    RP_CUDA(cudaMemcpyAsync(h, ctx->counters, sizeof(h), cudaMemcpyDeviceToHost, ctx->stream));
+    RP_CUDA(cudaStreamSynchronize(ctx->stream));
+    if (info) {
+      info->items = (int64_t)h[C_ITEMS];
+      info->evals = (int64_t)h[C_EVALS];
+      info->segments = (int64_t)h[C_SEGS];
+      info->nodes = 15 * (int64_t)h[C_SEGS];
+      info->leaves = (int64_t)h[C_LEAVES];
+      info->capped = (int64_t)h[C_CAPPED];
+      info->ties = (int64_t)h[C_TIES];
+      info->max_level = (int32_t)h[C_MAXLEV];
+      info->kappa = P.kap;
+    }
+    if (n_out) *n_out = (int64_t)h[C_NOUT];
+  }
+  return RP_OK;
+}
+
+int rp_scatter_impl(rp_ctx* ctx, const double* shards, int32_t world, int64_t cap, double* phi,
+                    double* ax, double* ay, double* err, int32_t* nseg) {
+  const rp_config& c = ctx->cfg;
+  int npts = c.nx * c.ny;
+  int64_t tot = (int64_t)world * cap;
+  k_scatter<<<(unsigned)((tot + 255) / 256), 256, 0, ctx->stream>>>(npts, world, cap, shards, phi,
+                                                                     ax, ay, err, nseg,
+                                                                     ctx->nseg_prev_pt);
+  RP_CHECK_LAUNCH();
+  ctx->has_forecast = 1;
+  return RP_OK;
+}

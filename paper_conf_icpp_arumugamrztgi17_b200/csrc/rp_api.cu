@@ -1,0 +1,363 @@
+// rp_api.cu -- the C ABI of librp (include/rp.h): context, history ring, state access and
+// the argument checking around the kernels of deposit.cu, potentials.cu, fields_push.cu.
+#include <new>
+
+#include "rp_internal.cuh"
+
+namespace {
+
+int validate(const rp_config* c) {
+  if (!c) return RP_EINVAL;
+  if (c->nx < 4 || c->ny < 4 || (int64_t)c->nx * c->ny > (1LL << 30)) return RP_EINVAL;
+  if (!(c->hx > 0) || !(c->hy > 0) || !(c->c > 0) || !(c->dt > 0) || !(c->tau > 0)) return RP_EINVAL;
+  if (c->history_depth < 1 || c->history_depth > 1000000) return RP_EINVAL;
+  if ((int64_t)c->nx * c->ny * c->history_depth > 0x7fffffffLL) return RP_EINVAL;
+  if (c->n_theta < 2 || (c->n_theta & 1) || c->n_theta > 4096) return RP_EINVAL;
+  if (c->max_depth < 1 || c->max_depth > 60) return RP_EINVAL;
+  if (c->n_root != 1 && c->n_root != 2) return RP_EINVAL;
+  return RP_OK;
+}
+
+__global__ void k_unpad(int nx, int ny, int PX, const double* __restrict__ slot,
+                        double* __restrict__ out) {
+  int id = blockIdx.x * blockDim.x + threadIdx.x;
+  if (id >= nx * ny) return;
+  int ix = id % nx, iy = id / nx;
+  const double* s = slot + 4 * ((size_t)(iy + RP_PAD) * PX + (ix + RP_PAD));
+  double* d = out + 4 * (size_t)id;
+  d[0] = s[0]; d[1] = s[1]; d[2] = s[2]; d[3] = s[3];
+}
+
+__global__ void k_pad(int nx, int ny, int PX, const double* __restrict__ in,
+                      double* __restrict__ slot) {
+  int id = blockIdx.x * blockDim.x + threadIdx.x;
+  if (id >= nx * ny) return;
+  int ix = id % nx, iy = id / nx;
+  const double* s = in + 4 * (size_t)id;
+  double* d = slot + 4 * ((size_t)(iy + RP_PAD) * PX + (ix + RP_PAD));
+  d[0] = s[0]; d[1] = s[1]; d[2] = s[2]; d[3] = 0.0;
+}
+
+__global__ void k_bins_out(int64_t n, int nbins, const int32_t* __restrict__ keys,
+                           int32_t* __restrict__ out) {
+  int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+  if (i < n) out[i] = keys[i] == nbins ? -1 : keys[i];
+}
+
+void free_all(rp_ctx* c) {
+  void* ptrs[] = {c->ring, c->frames_dev, c->keys, c->keys_sorted, c->perm, c->perm_sorted,
+                  c->rec, c->rec_sorted, c->bin_start, c->partial, c->cub_tmp, c->clipAB,
+                  c->sched_key, c->sched_key_sorted, c->sched_idx, c->sched_order, c->cost_prev,
+                  c->item_val, c->item_cnt, c->item_aux, c->counters, c->amp_dev, c->trig_full,
+                  c->point_key, c->point_key_sorted, c->point_idx, c->point_order,
+                  c->point_owner, c->nseg_prev_pt, c->hx_d, c->hy_d, c->hux_d, c->huy_d,
+                  c->mesh_d};
+  for (void* p : ptrs)
+    if (p) cudaFree(p);
+  delete[] c->fh;
+}
+
+}  // namespace
+
+extern "C" {
+
+int rp_version(void) { return 100; }
+
+const char* rp_strerror(int code) {
+  switch (code) {
+    case RP_OK: return "ok";
+    case RP_EINVAL: return "invalid argument or configuration";
+    case RP_ENOMEM: return "out of memory";
+    case RP_ECUDA: return "CUDA error";
+    case RP_ESTATE: return "call out of order";
+    case RP_ENODEV: return "no usable CUDA device";
+    default: return "unknown error";
+  }
+}
+
+const char* rp_last_error(const rp_ctx* ctx) { return ctx ? ctx->err.c_str() : "null context"; }
+
+int64_t rp_launch_count(const rp_ctx* ctx) { return ctx ? ctx->launches : 0; }
+
+int rp_create(const rp_config* cfg, rp_ctx** out) {
+  if (!out) return RP_EINVAL;
+  *out = nullptr;
+  if (validate(cfg) != RP_OK) return RP_EINVAL;
+  int ndev = 0;
+  if (cudaGetDeviceCount(&ndev) != cudaSuccess || ndev <= cfg->device || cfg->device < 0) {
+    cudaGetLastError();
+    return RP_ENODEV;
+  }
+  rp_ctx* ctx = new (std::nothrow) rp_ctx();
+  if (!ctx) return RP_ENOMEM;
+  ctx->cfg = *cfg;
+  auto fail = [&](int rc) {
+    free_all(ctx);
+    delete ctx;
+    return rc;
+  };
+  if (cudaSetDevice(cfg->device) != cudaSuccess) return fail(RP_ENODEV);
+  cudaDeviceGetAttribute(&ctx->sm_count, cudaDevAttrMultiProcessorCount, cfg->device);
+  ctx->H = cfg->history_depth + 2;
+  ctx->PX = cfg->nx + 2 * RP_PAD;
+  ctx->PY = cfg->ny + 2 * RP_PAD;
+  ctx->slot_doubles = (size_t)ctx->PX * ctx->PY * 4;
+  ctx->fh = new (std::nothrow) rp_frame[ctx->H];
+  if (!ctx->fh) return fail(RP_ENOMEM);
+  for (int i = 0; i < ctx->H; ++i) ctx->fh[i] = rp_frame{0.0, 0.0, 1.0, 0.0};
+  size_t ring_bytes = (size_t)ctx->H * ctx->slot_doubles * sizeof(double);
+  if (cudaMalloc(&ctx->ring, ring_bytes) != cudaSuccess) return fail(RP_ENOMEM);
+  if (cudaMemset(ctx->ring, 0, ring_bytes) != cudaSuccess) return fail(RP_ECUDA);
+  if (cudaMalloc(&ctx->frames_dev, ctx->H * sizeof(rp_frame)) != cudaSuccess) return fail(RP_ENOMEM);
+  if (cudaMemcpy(ctx->frames_dev, ctx->fh, ctx->H * sizeof(rp_frame), cudaMemcpyHostToDevice) != cudaSuccess)
+    return fail(RP_ECUDA);
+  size_t npts = (size_t)cfg->nx * cfg->ny;
+  if (cudaMalloc(&ctx->bin_start, (npts + 2) * sizeof(int32_t)) != cudaSuccess) return fail(RP_ENOMEM);
+  if (cudaMalloc(&ctx->partial, npts * 4 * sizeof(double)) != cudaSuccess) return fail(RP_ENOMEM);
+  int rc = rp_alloc_potential_scratch(ctx);
+  if (rc) return fail(rc);
+  // analytic amplitudes default to 1
+  double* ones = new double[ctx->H];
+  for (int i = 0; i < ctx->H; ++i) ones[i] = 1.0;
+  cudaError_t e = cudaMemcpy(ctx->amp_dev, ones, ctx->H * sizeof(double), cudaMemcpyHostToDevice);
+  delete[] ones;
+  if (e != cudaSuccess) return fail(RP_ECUDA);
+  *out = ctx;
+  return RP_OK;
+}
+
+void rp_destroy(rp_ctx* ctx) {
+  if (!ctx) return;
+  cudaStreamSynchronize(ctx->stream);
+  free_all(ctx);
+  delete ctx;
+}
+
+int rp_set_stream(rp_ctx* ctx, void* stream) {
+  if (!ctx) return RP_EINVAL;
+  ctx->stream = (cudaStream_t)stream;
+  return RP_OK;
+}
+
+int rp_history_init(rp_ctx* ctx, int32_t n_pre, const rp_frame* frames_host,
+                    const double* grids_dev, int32_t rigid) {
+  if (!ctx) return RP_EINVAL;
+  if (ctx->k >= 0) return rp_fail(ctx, RP_ESTATE, "history_init after the first deposit");
+  if (n_pre < 1 || n_pre > ctx->cfg.history_depth + 1 || !frames_host)
+    return rp_fail(ctx, RP_EINVAL, "history_init: n_pre out of range or no frames");
+  if (rigid && grids_dev) return rp_fail(ctx, RP_EINVAL, "history_init: rigid needs grids_dev == NULL");
+  if (!rigid && !grids_dev) return rp_fail(ctx, RP_EINVAL, "history_init: grids_dev required");
+  const rp_config& c = ctx->cfg;
+  for (int i = 0; i < n_pre; ++i) {
+    int level = -n_pre + i;
+    int s = slot_of(level, ctx->H);
+    ctx->fh[s] = frames_host[i];
+    if (!rigid) {
+      k_pad<<<(c.nx * c.ny + 255) / 256, 256, 0, ctx->stream>>>(
+          c.nx, c.ny, ctx->PX, grids_dev + (size_t)i * c.nx * c.ny * 4,
+          ctx->ring + (size_t)s * ctx->slot_doubles);
+      RP_CHECK_LAUNCH();
+    }
+  }
+  RP_CUDA(cudaMemcpyAsync(ctx->frames_dev, ctx->fh, ctx->H * sizeof(rp_frame), cudaMemcpyHostToDevice,
+                          ctx->stream));
+  RP_CUDA(cudaStreamSynchronize(ctx->stream));
+  ctx->n_pre = n_pre;
+  ctx->rigid_pending = rigid ? 1 : 0;
+  ctx->prehist_set = 1;
+  return RP_OK;
+}
+
+int rp_deposit(rp_ctx* ctx, const double* x, const double* y, const double* ux, const double* uy,
+               double q, int64_t n, const rp_frame* frame_k, double* partial_dev,
+               rp_deposit_info* info) {
+  if (!ctx) return RP_EINVAL;
+  return rp_deposit_impl(ctx, x, y, ux, uy, q, n, frame_k, partial_dev, info);
+}
+
+int rp_history_append(rp_ctx* ctx, const double* partials_dev, int32_t n_parts,
+                      const rp_frame* frame_k) {
+  if (!ctx) return RP_EINVAL;
+  return rp_append_impl(ctx, partials_dev, n_parts, frame_k);
+}
+
+int rp_deposit_step(rp_ctx* ctx, const double* x, const double* y, const double* ux,
+                    const double* uy, double q, int64_t n, const rp_frame* frame_k,
+                    rp_deposit_info* info) {
+  if (!ctx) return RP_EINVAL;
+  int rc = rp_deposit_impl(ctx, x, y, ux, uy, q, n, frame_k, ctx->partial, info);
+  if (rc) return rc;
+  return rp_append_impl(ctx, ctx->partial, 1, frame_k);
+}
+
+int rp_compute_potentials(rp_ctx* ctx, double* phi, double* ax, double* ay, double* err,
+                          int32_t* nseg, rp_potential_info* info) {
+  if (!ctx) return RP_EINVAL;
+  return rp_potentials_impl(ctx, RP_SRC_GRID, nullptr, 0, 1, phi, ax, ay, err, nseg, nullptr, 0,
+                            nullptr, info);
+}
+
+int64_t rp_shard_capacity(const rp_ctx* ctx, int32_t world) {
+  if (!ctx || world < 1) return 0;
+  int64_t n = (int64_t)ctx->cfg.nx * ctx->cfg.ny;
+  return (n + world - 1) / world;
+}
+
+int rp_compute_potentials_shard(rp_ctx* ctx, int32_t rank, int32_t world, double* shard_out,
+                                int64_t cap, int64_t* n_out, rp_potential_info* info) {
+  if (!ctx) return RP_EINVAL;
+  if (world < 1 || rank < 0 || rank >= world || !shard_out || cap < rp_shard_capacity(ctx, world))
+    return rp_fail(ctx, RP_EINVAL, "potentials_shard: bad rank/world/cap");
+  return rp_potentials_impl(ctx, RP_SRC_GRID, nullptr, rank, world, nullptr, nullptr, nullptr,
+                            nullptr, nullptr, shard_out, cap, n_out, info);
+}
+
+int rp_shard_scatter(rp_ctx* ctx, const double* shards, int32_t world, int64_t cap, double* phi,
+                     double* ax, double* ay, double* err, int32_t* nseg) {
+  if (!ctx) return RP_EINVAL;
+  if (!shards || world < 1 || cap < rp_shard_capacity(ctx, world) || !phi || !ax || !ay)
+    return rp_fail(ctx, RP_EINVAL, "shard_scatter: bad args");
+  return rp_scatter_impl(ctx, shards, world, cap, phi, ax, ay, err, nseg);
+}
+
+int rp_compute_fields(rp_ctx* ctx, const double* phi, const double* ax, const double* ay,
+                      const double* ax_prev, const double* ay_prev, double* ex, double* ey,
+                      double* bz) {
+  if (!ctx) return RP_EINVAL;
+  return rp_fields_impl(ctx, phi, ax, ay, ax_prev, ay_prev, ex, ey, bz);
+}
+
+int rp_push_particles(rp_ctx* ctx, double* x, double* y, double* ux, double* uy, int64_t n,
+                      double q_over_mc, double bz_ext, const double* ex, const double* ey,
+                      const double* bz) {
+  if (!ctx) return RP_EINVAL;
+  return rp_push_impl(ctx, x, y, ux, uy, n, q_over_mc, bz_ext, ex, ey, bz);
+}
+
+int rp_step_host(rp_ctx* ctx, double* xh, double* yh, double* uxh, double* uyh, int64_t n,
+                 double q, const rp_frame* frame_k, double q_over_mc, double bz_ext,
+                 double* mesh_host, rp_potential_info* info) {
+  if (!ctx) return RP_EINVAL;
+  if (n < 0 || (n > 0 && (!xh || !yh || !uxh || !uyh)) || !mesh_host || !frame_k)
+    return rp_fail(ctx, RP_EINVAL, "step_host: bad args");
+  const size_t npts = (size_t)ctx->cfg.nx * ctx->cfg.ny;
+  if (n > ctx->host_cap) {
+    cudaFree(ctx->hx_d); cudaFree(ctx->hy_d); cudaFree(ctx->hux_d); cudaFree(ctx->huy_d);
+    ctx->hx_d = ctx->hy_d = ctx->hux_d = ctx->huy_d = nullptr;
+    ctx->host_cap = 0;
+    RP_CUDA(cudaMalloc(&ctx->hx_d, n * sizeof(double)));
+    RP_CUDA(cudaMalloc(&ctx->hy_d, n * sizeof(double)));
+    RP_CUDA(cudaMalloc(&ctx->hux_d, n * sizeof(double)));
+    RP_CUDA(cudaMalloc(&ctx->huy_d, n * sizeof(double)));
+    ctx->host_cap = n;
+  }
+  if (!ctx->mesh_d) RP_CUDA(cudaMalloc(&ctx->mesh_d, 8 * npts * sizeof(double)));
+  cudaStream_t st = ctx->stream;
+  size_t nb = (size_t)n * sizeof(double);
+  if (n > 0) {
+    RP_CUDA(cudaMemcpyAsync(ctx->hx_d, xh, nb, cudaMemcpyHostToDevice, st));
+    RP_CUDA(cudaMemcpyAsync(ctx->hy_d, yh, nb, cudaMemcpyHostToDevice, st));
+    RP_CUDA(cudaMemcpyAsync(ctx->hux_d, uxh, nb, cudaMemcpyHostToDevice, st));
+    RP_CUDA(cudaMemcpyAsync(ctx->huy_d, uyh, nb, cudaMemcpyHostToDevice, st));
+  }
+  double* m = ctx->mesh_d;
+  double *phi = m, *ax = m + npts, *ay = m + 2 * npts, *ex = m + 3 * npts, *ey = m + 4 * npts,
+         *bz = m + 5 * npts, *axp = m + 6 * npts, *ayp = m + 7 * npts;
+  int rc = rp_deposit_step(ctx, ctx->hx_d, ctx->hy_d, ctx->hux_d, ctx->huy_d, q, n, frame_k, nullptr);
+  if (rc) return rc;
+  rc = rp_potentials_impl(ctx, RP_SRC_GRID, nullptr, 0, 1, phi, ax, ay, nullptr, nullptr, nullptr,
+                          0, nullptr, nullptr);
+  if (rc) return rc;
+  rc = rp_fields_impl(ctx, phi, ax, ay, ctx->have_prev_A ? axp : nullptr,
+                      ctx->have_prev_A ? ayp : nullptr, ex, ey, bz);
+  if (rc) return rc;
+  RP_CUDA(cudaMemcpyAsync(axp, ax, 2 * npts * sizeof(double), cudaMemcpyDeviceToDevice, st));
+  ctx->have_prev_A = 1;
+  rc = rp_push_impl(ctx, ctx->hx_d, ctx->hy_d, ctx->hux_d, ctx->huy_d, n, q_over_mc, bz_ext, ex, ey, bz);
+  if (rc) return rc;
+  RP_CUDA(cudaMemcpyAsync(mesh_host, m, 6 * npts * sizeof(double), cudaMemcpyDeviceToHost, st));
+  if (n > 0) {
+    RP_CUDA(cudaMemcpyAsync(xh, ctx->hx_d, nb, cudaMemcpyDeviceToHost, st));
+    RP_CUDA(cudaMemcpyAsync(yh, ctx->hy_d, nb, cudaMemcpyDeviceToHost, st));
+    RP_CUDA(cudaMemcpyAsync(uxh, ctx->hux_d, nb, cudaMemcpyDeviceToHost, st));
+    RP_CUDA(cudaMemcpyAsync(uyh, ctx->huy_d, nb, cudaMemcpyDeviceToHost, st));
+  }
+  RP_CUDA(cudaStreamSynchronize(st));
+  (void)info;
+  return RP_OK;
+}
+
+int rp_load_state(rp_ctx* ctx, int32_t k, int32_t n_pre, const rp_frame* frames_host,
+                  const double* ring_dev) {
+  if (!ctx) return RP_EINVAL;
+  if (k < 0 || n_pre < 0 || n_pre > ctx->cfg.history_depth + 1 || !frames_host || !ring_dev)
+    return rp_fail(ctx, RP_EINVAL, "load_state: bad args");
+  const rp_config& c = ctx->cfg;
+  for (int s = 0; s < ctx->H; ++s) {
+    ctx->fh[s] = frames_host[s];
+    k_pad<<<(c.nx * c.ny + 255) / 256, 256, 0, ctx->stream>>>(
+        c.nx, c.ny, ctx->PX, ring_dev + (size_t)s * c.nx * c.ny * 4,
+        ctx->ring + (size_t)s * ctx->slot_doubles);
+    RP_CHECK_LAUNCH();
+  }
+  RP_CUDA(cudaMemcpyAsync(ctx->frames_dev, ctx->fh, ctx->H * sizeof(rp_frame), cudaMemcpyHostToDevice,
+                          ctx->stream));
+  RP_CUDA(cudaStreamSynchronize(ctx->stream));
+  ctx->k = k;
+  ctx->n_pre = n_pre;
+  ctx->rigid_pending = 0;
+  ctx->prehist_set = 1;
+  ctx->has_forecast = 0;
+  ctx->have_prev_A = 0;
+  return RP_OK;
+}
+
+int rp_save_state(rp_ctx* ctx, int32_t* k_out, double* ring_dev, rp_frame* frames_host) {
+  if (!ctx) return RP_EINVAL;
+  const rp_config& c = ctx->cfg;
+  if (k_out) *k_out = ctx->k;
+  if (frames_host)
+    for (int s = 0; s < ctx->H; ++s) frames_host[s] = ctx->fh[s];
+  if (ring_dev) {
+    for (int s = 0; s < ctx->H; ++s) {
+      k_unpad<<<(c.nx * c.ny + 255) / 256, 256, 0, ctx->stream>>>(
+          c.nx, c.ny, ctx->PX, ctx->ring + (size_t)s * ctx->slot_doubles,
+          ring_dev + (size_t)s * c.nx * c.ny * 4);
+      RP_CHECK_LAUNCH();
+    }
+  }
+  RP_CUDA(cudaStreamSynchronize(ctx->stream));
+  return RP_OK;
+}
+
+int rp_debug_bins(rp_ctx* ctx, int32_t* bins_dev, int64_t n) {
+  if (!ctx) return RP_EINVAL;
+  if (!bins_dev || n != ctx->last_n) return rp_fail(ctx, RP_EINVAL, "debug_bins: n must equal the last deposit's n");
+  if (n == 0) return RP_OK;
+  k_bins_out<<<(unsigned)((n + 255) / 256), 256, 0, ctx->stream>>>(n, ctx->cfg.nx * ctx->cfg.ny,
+                                                                    ctx->keys, bins_dev);
+  RP_CHECK_LAUNCH();
+  return RP_OK;
+}
+
+int rp_debug_potentials_analytic(rp_ctx* ctx, int32_t kind, double x0, double y0, double width,
+                                 double q, double bx, double by, const double* amp_host,
+                                 double* phi, double* ax, double* ay, double* err, int32_t* nseg,
+                                 rp_potential_info* info) {
+  if (!ctx) return RP_EINVAL;
+  if ((kind != RP_SRC_GAUSS && kind != RP_SRC_DISK) || !(width > 0))
+    return rp_fail(ctx, RP_EINVAL, "debug_potentials_analytic: bad source");
+  double* h = new double[ctx->H];
+  for (int i = 0; i < ctx->H; ++i) h[i] = amp_host ? amp_host[i] : 1.0;
+  cudaError_t e = cudaMemcpy(ctx->amp_dev, h, ctx->H * sizeof(double), cudaMemcpyHostToDevice);
+  delete[] h;
+  RP_CUDA(e);
+  double src[6] = {x0, y0, width, q, bx, by};
+  int saved = ctx->has_forecast;
+  ctx->has_forecast = 0;
+  int rc = rp_potentials_impl(ctx, kind, src, 0, 1, phi, ax, ay, err, nseg, nullptr, 0, nullptr, info);
+  ctx->has_forecast = saved;
+  return rc;
+}
+
+}  // extern "C"

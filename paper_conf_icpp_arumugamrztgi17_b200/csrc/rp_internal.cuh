@@ -1,0 +1,131 @@
+// rp_internal.cuh -- context and shared device helpers of librp (product path).
+// Nothing here is shared with oracle/ (test infrastructure): the two are written
+// independently from PAPER.md and DESIGN.md's readings.
+#pragma once
+
+#include <cuda_runtime.h>
+#include <stdint.h>
+#include <string.h>
+
+#include <string>
+
+#include "../../include/rp.h"
+
+#define RP_PAD 3  // zero border (nodes) around every ring grid: stencils never bounds-check
+
+struct rp_ctx {
+  rp_config cfg;
+  int H = 0;                 // ring slots = history_depth + 2
+  int PX = 0, PY = 0;        // padded grid dims (nx + 6, ny + 6)
+  size_t slot_doubles = 0;   // PX * PY * 4
+  cudaStream_t stream = 0;
+  int sm_count = 0;
+
+  // history: ring [H][PY][PX][4] FP64 and frames [H]
+  double* ring = nullptr;
+  rp_frame* frames_dev = nullptr;
+  rp_frame* fh = nullptr;    // host copy of frames [H]
+  int k = -1;                // current step (-1 before the first append)
+  int n_pre = 0;             // pre-history levels available below step 0
+  int rigid_pending = 0;     // rigid pre-history: fill on first append
+  int prehist_set = 0;
+
+  // deposition scratch (grown on demand)
+  int64_t dep_cap = 0;
+  int32_t* keys = nullptr;      // bin per particle (nx*ny for lost)
+  int32_t* keys_sorted = nullptr;
+  int32_t* perm = nullptr;      // particle index
+  int32_t* perm_sorted = nullptr;
+  double4* rec = nullptr;       // (dx, dy, bx, by) per particle
+  double4* rec_sorted = nullptr;
+  int32_t* bin_start = nullptr; // [nx*ny + 1]
+  int64_t last_n = 0;
+  double* partial = nullptr;    // [ny][nx][4] scratch for rp_deposit_step
+  void* cub_tmp = nullptr;
+  size_t cub_tmp_bytes = 0;
+
+  // potentials scratch: dense (point, subregion) arrays of npts * kappa_max
+  double2* clipAB = nullptr;        // [A, B] per (p, j)
+  uint16_t* sched_key = nullptr;    // sort keys (0xFFFF = empty)
+  uint16_t* sched_key_sorted = nullptr;
+  int32_t* sched_idx = nullptr;     // iota
+  int32_t* sched_order = nullptr;   // sorted item ids (p * kappa_max + j)
+  uint16_t* cost_prev = nullptr;    // forecast: previous step's segments per (p, j)
+  double4* item_val = nullptr;      // (phi, ax, ay, err) per (p, j)
+  int4* item_cnt = nullptr;         // (nseg, nleaf, capped, ties) per (p, j)
+  uint2* item_aux = nullptr;        // (max_level, evals) per (p, j)
+  unsigned long long* counters = nullptr;  // [16] device counters
+  double* amp_dev = nullptr;        // [H] analytic amplitudes
+  double2* trig_full = nullptr;     // [n_theta] (cos, sin)(2 pi m / n_theta)
+  int has_forecast = 0;
+
+  // sharding scratch
+  int32_t* point_key = nullptr;     // per point predicted work key
+  int32_t* point_key_sorted = nullptr;
+  int32_t* point_idx = nullptr;
+  int32_t* point_order = nullptr;
+  int32_t* point_owner = nullptr;   // rank owning each point
+  int32_t* nseg_prev_pt = nullptr;  // per point segments of the last step (shard map)
+
+  // end-to-end (host buffer) path scratch
+  int64_t host_cap = 0;
+  double* hx_d = nullptr; double* hy_d = nullptr; double* hux_d = nullptr; double* huy_d = nullptr;
+  double* mesh_d = nullptr;         // [8][npts]: phi ax ay ex ey bz ax_prev ay_prev
+  int have_prev_A = 0;
+
+  int64_t launches = 0;
+  std::string err;
+};
+
+// ---------------------------------------------------------------- error helpers
+#define RP_CUDA(call)                                                            \
+  do {                                                                           \
+    cudaError_t e_ = (call);                                                     \
+    if (e_ != cudaSuccess) {                                                     \
+      ctx->err = std::string(#call) + ": " + cudaGetErrorString(e_);             \
+      return e_ == cudaErrorMemoryAllocation ? RP_ENOMEM : RP_ECUDA;             \
+    }                                                                            \
+  } while (0)
+
+#define RP_CHECK_LAUNCH()                                                        \
+  do {                                                                           \
+    ctx->launches++;                                                             \
+    cudaError_t e_ = cudaGetLastError();                                         \
+    if (e_ != cudaSuccess) {                                                     \
+      ctx->err = std::string("kernel launch: ") + cudaGetErrorString(e_);        \
+      return RP_ECUDA;                                                           \
+    }                                                                            \
+  } while (0)
+
+static inline int rp_fail(rp_ctx* ctx, int code, const char* msg) {
+  if (ctx) ctx->err = msg;
+  return code;
+}
+
+static inline int slot_of(int level, int H) { return ((level % H) + H) % H; }
+__device__ __forceinline__ int slot_of_dev(int level, int H) { return ((level % H) + H) % H; }
+
+static inline int kappa_of(const rp_ctx* ctx) {
+  int kap = ctx->k + ctx->n_pre - 1;
+  if (kap > ctx->cfg.history_depth) kap = ctx->cfg.history_depth;
+  if (kap < 0) kap = 0;
+  return kap;
+}
+
+// internal entry points implemented in the .cu files
+int rp_deposit_impl(rp_ctx* ctx, const double* x, const double* y, const double* ux,
+                    const double* uy, double q, int64_t n, const rp_frame* frame_k,
+                    double* partial_dev, rp_deposit_info* info);
+int rp_append_impl(rp_ctx* ctx, const double* partials, int32_t n_parts, const rp_frame* fk);
+int rp_potentials_impl(rp_ctx* ctx, int src_kind, const double src[6], int32_t rank,
+                       int32_t world, double* phi, double* ax, double* ay, double* err,
+                       int32_t* nseg, double* shard_out, int64_t cap, int64_t* n_out,
+                       rp_potential_info* info);
+int rp_fields_impl(rp_ctx* ctx, const double* phi, const double* ax, const double* ay,
+                   const double* axp, const double* ayp, double* ex, double* ey, double* bz);
+int rp_push_impl(rp_ctx* ctx, double* x, double* y, double* ux, double* uy, int64_t n,
+                 double qmc, double bz_ext, const double* ex, const double* ey,
+                 const double* bz);
+int rp_scatter_impl(rp_ctx* ctx, const double* shards, int32_t world, int64_t cap,
+                    double* phi, double* ax, double* ay, double* err, int32_t* nseg);
+int rp_alloc_potential_scratch(rp_ctx* ctx);

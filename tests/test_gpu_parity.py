@@ -1,0 +1,400 @@
+"""GPU parity: the CUDA path (through the C ABI) against the oracle, element by element,
+on the same seeded inputs.
+
+Bars: deposition bins bit-exact; moment grids within 1e-12 of max|M|; potentials within
+1e-11 * max(|phi|,|A|) per point with equal segment counts (oracle tie-flagged points are
+reported, not failed); fields within 1e-11 relative; push within 1e-13.
+"""
+import math
+
+import numpy as np
+import pytest
+
+import oracle
+import workloads as W
+from tests import gpu_util as G
+
+pytestmark = pytest.mark.gpu
+
+
+@pytest.fixture(scope="module")
+def torch():
+    import torch as t
+    assert t.cuda.is_available()
+    return t
+
+
+def _dev_arrays(torch, *arrs):
+    return [torch.tensor(np.ascontiguousarray(a), dtype=torch.float64, device="cuda") for a in arrs]
+
+
+# ------------------------------------------------------------------ deposition
+@pytest.mark.parametrize("cfgno", [1, 2])
+def test_deposit_bins_bit_exact_and_moments(torch, cfgno):
+    from paper_conf_icpp_arumugamrztgi17_b200 import rp
+    cfg = W.config(cfgno)
+    x, y, ux, uy = W.particles(cfg)
+    x = x.copy()
+    x[:3] += 30 * cfg.sigma  # some lost particles
+    M, bins, ql = oracle.deposit(x, y, ux, uy, cfg.q_particle, W.frame(cfg, 0), cfg.nx, cfg.ny,
+                                 cfg.hx, cfg.hy)
+    ctx = G.make_ctx(cfg)
+    try:
+        xd, yd, uxd, uyd = _dev_arrays(torch, x, y, ux, uy)
+        part = torch.zeros((cfg.ny, cfg.nx, 4), dtype=torch.float64, device="cuda")
+        info = rp.rp_deposit(ctx, xd, yd, uxd, uyd, cfg.q_particle, W.frame(cfg, 0), part, info=True)
+        b = torch.zeros(len(x), dtype=torch.int32, device="cuda")
+        rp.rp_debug_bins(ctx, b)
+        torch.cuda.synchronize()
+        np.testing.assert_array_equal(b.cpu().numpy(), bins)
+        Mg = part.cpu().numpy()
+        scale = np.abs(M).max()
+        assert np.abs(Mg - M).max() <= 1e-12 * scale
+        assert info.n_lost == int((bins < 0).sum())
+        assert abs(info.q_lost - ql) < 1e-15
+        tot = Mg[..., 0].sum() * cfg.hx * cfg.hy + info.q_lost
+        assert abs(tot - 1.0) < 1e-12
+    finally:
+        rp.rp_destroy(ctx)
+
+
+def test_deposit_golden_ties(torch):
+    import json, os
+    from paper_conf_icpp_arumugamrztgi17_b200 import rp
+    g = json.load(open(os.path.join(os.path.dirname(__file__), "golden", "bins_ties.json")))
+    x = np.array([c["x"] for c in g["cases"]])
+    y = np.array([c["y"] for c in g["cases"]])
+    z = np.zeros_like(x)
+    ctx = rp.rp_create(g["nx"], g["ny"], g["hx"], g["hy"], 2, 1.0, 1.0, 1e-6)
+    try:
+        xd, yd, zd, zd2 = _dev_arrays(torch, x, y, z, z)
+        part = torch.zeros((g["ny"], g["nx"], 4), dtype=torch.float64, device="cuda")
+        rp.rp_deposit(ctx, xd, yd, zd, zd2, 1.0, g["frame"], part)
+        b = torch.zeros(len(x), dtype=torch.int32, device="cuda")
+        rp.rp_debug_bins(ctx, b)
+        np.testing.assert_array_equal(b.cpu().numpy(), [c["bin"] for c in g["cases"]])
+    finally:
+        rp.rp_destroy(ctx)
+
+
+# ------------------------------------------------------------------ potentials
+def _deposit_rigid_ring(cfg, n=None, seed=None):
+    x, y, ux, uy = W.particles(cfg, n=n, seed=seed)
+    q = 1.0 / len(x)
+    M, _, _ = oracle.deposit(x, y, ux, uy, q, W.frame(cfg, 0), cfg.nx, cfg.ny, cfg.hx, cfg.hy)
+    return np.repeat(M[None], cfg.H, axis=0), (x, y, ux, uy, q)
+
+
+def test_potentials_static_cfg1_full_mesh(torch):
+    """Config 1 (BASELINE.json configs[0]), step 0 with rigid pre-history, every mesh point."""
+    from paper_conf_icpp_arumugamrztgi17_b200 import rp
+    cfg = W.config(1)
+    ring, _ = _deposit_rigid_ring(cfg)
+    frames = W.ring_frames(cfg, 0)
+    pts = np.arange(cfg.nx * cfg.ny)
+    orc = G.oracle_problem(cfg, ring, frames, 0, cfg.n_pre).potentials(pts)
+    ctx = G.make_ctx(cfg)
+    try:
+        G.load_state(ctx, cfg, 0, cfg.n_pre, ring, frames)
+        gpu, info = G.gpu_potentials(ctx, len(pts))
+        fail, worst, nties = G.compare_potentials(gpu, orc, pts)
+        assert not fail.any(), (np.nonzero(fail)[0][:10], worst)
+        assert worst < G.REL
+        assert info.segments == int(orc["nseg"].sum())
+        assert info.capped == int(orc["capped"].sum())
+        assert info.evals == int(orc["evals"].sum())
+        assert info.kappa == cfg.kappa_max
+    finally:
+        rp.rp_destroy(ctx)
+
+
+def test_potentials_bend_cfg2_full_size_sampled(torch):
+    """Config 2 (the bench workload) at full size through the product path: GPU deposit of
+    1e6 particles + rigid pre-history + potentials on the whole 64x64 mesh in the bench's
+    launch configuration; the oracle computes a stratified sample of points."""
+    from paper_conf_icpp_arumugamrztgi17_b200 import rp
+    cfg = W.config(2)
+    ring, (x, y, ux, uy, q) = _deposit_rigid_ring(cfg)
+    pts = W.sample_points(cfg.nx, cfg.ny, 40, seed=5)
+    orc = G.oracle_problem(cfg, ring, W.ring_frames(cfg, 0), 0, cfg.n_pre).potentials(pts)
+    ctx = G.make_ctx(cfg)
+    try:
+        pre = W.frames(cfg, range(-cfg.n_pre, 0))
+        rp.rp_history_init(ctx, cfg.n_pre, pre, None, True)
+        xd, yd, uxd, uyd = _dev_arrays(torch, x, y, ux, uy)
+        rp.rp_deposit_step(ctx, xd, yd, uxd, uyd, q, W.frame(cfg, 0))
+        gpu, info = G.gpu_potentials(ctx, cfg.nx * cfg.ny)
+        fail, worst, nties = G.compare_potentials(gpu, orc, pts)
+        assert not fail.any(), (pts[fail][:10], worst)
+        assert np.isfinite(gpu["phi"]).all()
+    finally:
+        rp.rp_destroy(ctx)
+
+
+def _bend_small(n=24, kap=60):
+    c = W.config(2)
+    return W.Config(number=2, name="bend-small", nx=n, ny=n, n_particles=1, steps=kap,
+                    kappa_max=kap, geometry="bend", sigma=c.sigma, cdt=c.cdt, gamma0=c.gamma0,
+                    r0=c.r0, sigma_xp=c.sigma_xp, q_over_mc=c.q_over_mc)
+
+
+def test_potentials_bend_small_full_mesh_two_steps(torch):
+    """Moving frames, node-sampled history with a time-varying amplitude, two consecutive
+    steps (the second uses the first step's counts as the schedule forecast)."""
+    from paper_conf_icpp_arumugamrztgi17_b200 import rp
+    cfg = _bend_small()
+    ctx = G.make_ctx(cfg)
+    try:
+        for k in (5, 6):
+            ring = W.node_gaussian_ring(cfg, k=k, beta=(cfg.beta0, 0.01),
+                                        amp_of_level=lambda l: 1.0 + 0.01 * l)
+            frames = W.ring_frames(cfg, k)
+            pts = np.arange(cfg.nx * cfg.ny)
+            orc = G.oracle_problem(cfg, ring, frames, k, cfg.n_pre).potentials(pts)
+            G.load_state(ctx, cfg, k, cfg.n_pre, ring, frames)
+            gpu, info = G.gpu_potentials(ctx, len(pts))
+            fail, worst, nties = G.compare_potentials(gpu, orc, pts)
+            assert not fail.any(), (np.nonzero(fail)[0][:10], worst)
+    finally:
+        rp.rp_destroy(ctx)
+
+
+@pytest.mark.parametrize("variant", [dict(n_root=1), dict(max_depth=5), dict(n_theta=16)])
+def test_potentials_variants(torch, variant):
+    from paper_conf_icpp_arumugamrztgi17_b200 import rp
+    cfg = W.Config(number=0, name="v", nx=20, ny=13, n_particles=4000, steps=4, kappa_max=7,
+                   geometry="static", sigma=1.0, cdt=1.9, **variant)
+    ring, _ = _deposit_rigid_ring(cfg, n=4000, seed=9)
+    frames = W.ring_frames(cfg, 3)
+    pts = np.arange(cfg.nx * cfg.ny)
+    orc = G.oracle_problem(cfg, ring, frames, 3, 0).potentials(pts)
+    ctx = G.make_ctx(cfg)
+    try:
+        G.load_state(ctx, cfg, 3, 0, ring, frames)
+        gpu, info = G.gpu_potentials(ctx, len(pts))
+        fail, worst, _ = G.compare_potentials(gpu, orc, pts)
+        assert not fail.any(), (np.nonzero(fail)[0][:10], worst)
+        if "max_depth" in variant:
+            assert info.capped > 0 and info.capped == int(orc["capped"].sum())
+    finally:
+        rp.rp_destroy(ctx)
+
+
+def test_potentials_degenerate_kappa_zero_and_min_grid(torch):
+    from paper_conf_icpp_arumugamrztgi17_b200 import rp
+    cfg = W.Config(number=0, name="min", nx=4, ny=4, n_particles=50, steps=3, kappa_max=2,
+                   geometry="static", sigma=0.3, cdt=0.5)
+    x, y, ux, uy = W.particles(cfg, n=50, seed=1)
+    ctx = G.make_ctx(cfg)
+    try:
+        xd, yd, uxd, uyd = _dev_arrays(torch, x, y, ux, uy)
+        for k in range(3):
+            rp.rp_deposit_step(ctx, xd, yd, uxd, uyd, 1.0 / 50, W.frame(cfg, k))
+            gpu, info = G.gpu_potentials(ctx, 16)
+            if k < 2:  # no pre-history: kappa(k) = k - 1 <= 0 -> nothing to integrate (R-3)
+                assert info.kappa == 0 and (gpu["phi"] == 0).all() and (gpu["nseg"] == 0).all()
+        # k = 2: kappa = 1, compare with the oracle on the ring the GPU was given
+        ring = np.zeros((cfg.H, 4, 4, 4))
+        M, _, _ = oracle.deposit(x, y, ux, uy, 1.0 / 50, W.frame(cfg, 0), 4, 4, cfg.hx, cfg.hy)
+        for l in range(3):
+            ring[l % cfg.H] = M
+        orc = G.oracle_problem(cfg, ring, W.ring_frames(cfg, 2), 2, 0).potentials(np.arange(16))
+        fail, worst, _ = G.compare_potentials(gpu, orc, np.arange(16))
+        assert not fail.any(), worst
+    finally:
+        rp.rp_destroy(ctx)
+
+
+# ------------------------------------------------------------------ analytic sources
+@pytest.mark.parametrize("kind", ["gauss", "disk"])
+def test_analytic_sources_closed_form_on_gpu(torch, kind):
+    import scipy.special as sp
+    from paper_conf_icpp_arumugamrztgi17_b200 import rp
+    sq = math.sqrt(math.pi / 2)
+    if kind == "gauss":
+        cfg = W.Config(number=0, name="g", nx=9, ny=9, n_particles=1, steps=1, kappa_max=12,
+                       geometry="static", sigma=1.0, cdt=1.6)
+        src = dict(kind=rp.RP_SRC_GAUSS, x0=0.0, y0=0.0, width=1.0, q=1.0, bx=0.3, by=-0.2)
+        okind = oracle.SRC_GAUSS
+    else:
+        cfg = W.Config(number=0, name="d", nx=9, ny=9, n_particles=1, steps=1, kappa_max=12,
+                       geometry="static", sigma=1.0, cdt=0.8)
+        src = dict(kind=rp.RP_SRC_DISK, x0=0.0, y0=0.0, width=1.0, q=1.0, bx=0.0, by=0.0)
+        okind = oracle.SRC_DISK
+    # mesh nodes at (ix*h - 5, iy*h - 5) with h = 10/8: the source at the origin
+    ring = np.zeros((cfg.H, cfg.ny, cfg.nx, 4))
+    frames = W.ring_frames(cfg, 20)
+    ctx = G.make_ctx(cfg, tau=1e-6 * sq if kind == "gauss" else 1e-6)
+    try:
+        G.load_state(ctx, cfg, 20, 0, ring, frames)
+        d = {k: torch.zeros(81, dtype=torch.float64, device="cuda") for k in ("phi", "ax", "ay", "err")}
+        nseg = torch.zeros(81, dtype=torch.int32, device="cuda")
+        # analytic source centre in frame-local coordinates: the lab origin = local (5, 5)
+        rp.rp_debug_potentials_analytic(ctx, src["kind"], 5.0, 5.0, src["width"], src["q"],
+                                        src["bx"], src["by"], None, d["phi"], d["ax"], d["ay"],
+                                        d["err"], nseg)
+        gpu = {k: v.cpu().numpy() for k, v in d.items()}
+        gpu["nseg"] = nseg.cpu().numpy()
+        P = G.oracle_problem(cfg, None, frames, 20, 0, source=okind, x0=5.0, y0=5.0,
+                             width=src["width"], q=src["q"], bx=src["bx"], by=src["by"],
+                             tau=1e-6 * sq if kind == "gauss" else 1e-6)
+        pts = np.arange(81)
+        orc = P.potentials(pts)
+        fail, worst, _ = G.compare_potentials(gpu, orc, pts)
+        assert not fail.any(), worst
+        for p in pts:
+            px, py = P.mesh_point(p % 9, p // 9)
+            s = math.hypot(px, py)
+            if kind == "gauss":
+                exact = sq * sp.i0e(s * s / 4)
+            elif s < 1:
+                exact = 4 * sp.ellipe(s * s)
+            elif s == 1:
+                exact = 4.0
+            else:
+                exact = 4 * s * (sp.ellipe(1 / s ** 2) - (1 - 1 / s ** 2) * sp.ellipk(1 / s ** 2))
+            assert abs(gpu["phi"][p] - exact) < 1e-6
+    finally:
+        rp.rp_destroy(ctx)
+
+
+# ------------------------------------------------------------------ fields and push
+def test_fields_parity(torch):
+    from paper_conf_icpp_arumugamrztgi17_b200 import rp
+    cfg = _bend_small(n=17, kap=4)
+    rng = np.random.default_rng(21)
+    npts = cfg.nx * cfg.ny
+    phi, ax, ay, axp, ayp = (rng.standard_normal(npts) for _ in range(5))
+    fk, fm = W.frame(cfg, 1), W.frame(cfg, 0)
+    ex, ey, bz = oracle.fields(cfg.nx, cfg.ny, cfg.hx, cfg.hy, cfg.c, cfg.dt, fk, fm,
+                               phi.reshape(cfg.ny, cfg.nx), ax.reshape(cfg.ny, cfg.nx),
+                               ay.reshape(cfg.ny, cfg.nx), axp.reshape(cfg.ny, cfg.nx),
+                               ayp.reshape(cfg.ny, cfg.nx))
+    ctx = G.make_ctx(cfg)
+    try:
+        ring = np.zeros((cfg.H, cfg.ny, cfg.nx, 4))
+        G.load_state(ctx, cfg, 1, 0, ring, W.ring_frames(cfg, 1))
+        d = _dev_arrays(torch, phi, ax, ay, axp, ayp)
+        out = [torch.zeros(npts, dtype=torch.float64, device="cuda") for _ in range(3)]
+        rp.rp_compute_fields(ctx, *d, *out)
+        for got, want in zip(out, (ex, ey, bz)):
+            g = got.cpu().numpy().reshape(cfg.ny, cfg.nx)
+            assert np.abs(g - want).max() <= 1e-11 * np.abs(want).max()
+        # without the previous step: dA/dt = 0
+        rp.rp_compute_fields(ctx, d[0], d[1], d[2], None, None, *out)
+        ex0, ey0, bz0 = oracle.fields(cfg.nx, cfg.ny, cfg.hx, cfg.hy, cfg.c, cfg.dt, fk, None,
+                                      phi.reshape(cfg.ny, cfg.nx), ax.reshape(cfg.ny, cfg.nx),
+                                      ay.reshape(cfg.ny, cfg.nx))
+        assert np.abs(out[0].cpu().numpy().reshape(cfg.ny, cfg.nx) - ex0).max() <= 1e-11 * np.abs(ex0).max()
+    finally:
+        rp.rp_destroy(ctx)
+
+
+def test_push_parity(torch):
+    from paper_conf_icpp_arumugamrztgi17_b200 import rp
+    cfg = W.config(2)
+    x, y, ux, uy = W.particles(cfg, n=200_000, seed=3)
+    rng = np.random.default_rng(4)
+    npts = cfg.nx * cfg.ny
+    scale = 1e8
+    ex, ey, bz = (scale * rng.standard_normal(npts) for _ in range(3))
+    fk = W.frame(cfg, 0)
+    want = oracle.push(cfg.nx, cfg.ny, cfg.hx, cfg.hy, cfg.c, cfg.dt, fk, x, y, ux, uy,
+                       cfg.q_over_mc, cfg.bz_ext, ex, ey, bz)
+    ctx = G.make_ctx(cfg)
+    try:
+        ring = np.zeros((cfg.H, cfg.ny, cfg.nx, 4))
+        G.load_state(ctx, cfg, 0, 0, ring, W.ring_frames(cfg, 0))
+        xd, yd, uxd, uyd, exd, eyd, bzd = _dev_arrays(torch, x, y, ux, uy, ex, ey, bz)
+        rp.rp_push_particles(ctx, xd, yd, uxd, uyd, cfg.q_over_mc, cfg.bz_ext, exd, eyd, bzd)
+        got = [t.cpu().numpy() for t in (xd, yd, uxd, uyd)]
+        # positions: absolute 1e-13 of the orbit scale; momenta: 1e-13 relative
+        assert np.abs(got[0] - want[0]).max() < 1e-13 * cfg.r0 * 1e-2 + 1e-15
+        assert np.abs(got[1] - want[1]).max() < 1e-13 * cfg.r0 * 1e-2 + 1e-15
+        assert np.abs(got[2] - want[2]).max() < 1e-13 * np.abs(want[2]).max()
+        assert np.abs(got[3] - want[3]).max() < 1e-13 * np.abs(want[2]).max()
+    finally:
+        rp.rp_destroy(ctx)
+
+
+# ------------------------------------------------------------------ sharding, e2e, loop
+def test_shard_path_equals_full_mesh(torch):
+    """Mesh-point sharding simulated on one GPU: ranks 0..W-1 each compute
+    their shard; the scattered result is bit-identical to the single-call result."""
+    from paper_conf_icpp_arumugamrztgi17_b200 import rp
+    cfg = W.config(1)
+    ring, _ = _deposit_rigid_ring(cfg)
+    frames = W.ring_frames(cfg, 0)
+    ctx = G.make_ctx(cfg)
+    try:
+        G.load_state(ctx, cfg, 0, cfg.n_pre, ring, frames)
+        full, _ = G.gpu_potentials(ctx, 1024)
+        for world in (2, 3, 8):
+            for step in range(2):  # second pass uses the counts as the shard forecast
+                cap = rp.rp_shard_capacity(ctx, world)
+                shards = torch.zeros((world, cap, 6), dtype=torch.float64, device="cuda")
+                tot = 0
+                for r in range(world):
+                    n, _ = rp.rp_compute_potentials_shard(ctx, r, world, shards[r])
+                    tot += n
+                assert tot == 1024
+                out = {k: torch.zeros(1024, dtype=torch.float64, device="cuda") for k in ("phi", "ax", "ay", "err")}
+                nseg = torch.zeros(1024, dtype=torch.int32, device="cuda")
+                rp.rp_shard_scatter(ctx, shards, world, out["phi"], out["ax"], out["ay"], out["err"], nseg)
+                for k in ("phi", "ax", "ay", "err"):
+                    np.testing.assert_array_equal(out[k].cpu().numpy(), full[k])
+                np.testing.assert_array_equal(nseg.cpu().numpy(), full["nseg"])
+    finally:
+        rp.rp_destroy(ctx)
+
+
+def test_step_host_matches_device_path(torch):
+    from paper_conf_icpp_arumugamrztgi17_b200 import rp
+    cfg = W.config(1)
+    x, y, ux, uy = W.particles(cfg)
+    q = cfg.q_particle
+    pre = W.frames(cfg, range(-cfg.n_pre, 0))
+    # device path
+    ctx = G.make_ctx(cfg)
+    ctx2 = G.make_ctx(cfg)
+    try:
+        rp.rp_history_init(ctx, cfg.n_pre, pre, None, True)
+        rp.rp_history_init(ctx2, cfg.n_pre, pre, None, True)
+        xd, yd, uxd, uyd = _dev_arrays(torch, x, y, ux, uy)
+        n = cfg.nx * cfg.ny
+        phi, ax, ay, ex, ey, bz, axp, ayp = (torch.zeros(n, dtype=torch.float64, device="cuda") for _ in range(8))
+        hx, hy, hux, huy = (torch.tensor(a).pin_memory() for a in (x, y, ux, uy))
+        mesh = torch.zeros((6, n), dtype=torch.float64).pin_memory()
+        for k in range(3):
+            rp.rp_deposit_step(ctx, xd, yd, uxd, uyd, q, W.frame(cfg, k))
+            rp.rp_compute_potentials(ctx, phi, ax, ay)
+            rp.rp_compute_fields(ctx, phi, ax, ay, axp if k else None, ayp if k else None, ex, ey, bz)
+            axp.copy_(ax); ayp.copy_(ay)
+            rp.rp_push_particles(ctx, xd, yd, uxd, uyd, cfg.q_over_mc, 0.0, ex, ey, bz)
+            rp.rp_step_host(ctx2, hx, hy, hux, huy, q, W.frame(cfg, k), cfg.q_over_mc, 0.0, mesh)
+            torch.cuda.synchronize()
+            for i, t in enumerate((phi, ax, ay, ex, ey, bz)):
+                np.testing.assert_array_equal(mesh[i].numpy(), t.cpu().numpy())
+            np.testing.assert_array_equal(hx.numpy(), xd.cpu().numpy())
+        assert rp.rp_launch_count(ctx) > 0
+    finally:
+        rp.rp_destroy(ctx)
+        rp.rp_destroy(ctx2)
+
+
+def test_call_order_errors(torch):
+    from paper_conf_icpp_arumugamrztgi17_b200 import rp
+    cfg = W.config(1)
+    ctx = G.make_ctx(cfg)
+    try:
+        z = torch.zeros(1024, dtype=torch.float64, device="cuda")
+        with pytest.raises(rp.RpError) as e:
+            rp.rp_compute_potentials(ctx, z, z, z)
+        assert e.value.code == -5
+        x = torch.zeros(10, dtype=torch.float64, device="cuda")
+        rp.rp_deposit_step(ctx, x, x, x, x, 0.1, W.frame(cfg, 0))
+        with pytest.raises(rp.RpError) as e:
+            rp.rp_history_init(ctx, 2, W.frames(cfg, [-2, -1]), None, True)
+        assert e.value.code == -5
+    finally:
+        rp.rp_destroy(ctx)
