@@ -202,6 +202,27 @@ int rp_debug_potentials_analytic(rp_ctx* ctx, int32_t kind, double x0, double y0
                                  const double* amp_host, double* phi, double* ax, double* ay,
                                  double* err, int32_t* nseg, rp_potential_info* info);
 
+/* Per-kernel device time, measured with CUDA events recorded on the context's stream around
+ * each launch while profiling is enabled (bench.py's live roofline numbers). */
+typedef struct {
+  double deposit_ms;       /* bin + sort + gather + node sums                                   */
+  double append_ms;        /* rank-order sum into the ring                                      */
+  double clip_ms;          /* support clip + schedule keys                                      */
+  double sort_ms;          /* schedule sort (CUB)                                               */
+  double integrate_ms;     /* the GK15 integrator (dominant kernel)                             */
+  double reduce_ms;        /* per-point reduction                                               */
+  double fields_ms;
+  double push_ms;
+  int64_t integrate_launches;
+} rp_profile;
+
+/* enable != 0 starts (and resets) event timing; 0 stops it.  Adds two event records per
+ * instrumented launch; off by default. */
+int rp_profile_enable(rp_ctx* ctx, int32_t enable);
+
+/* Sum of the recorded device times since the last enable.  Syncs the stream. */
+int rp_profile_read(rp_ctx* ctx, rp_profile* out);
+
 /* Number of kernel launches this context has issued (for bench.py's gpu_launches). */
 int64_t rp_launch_count(const rp_ctx* ctx);
 

@@ -167,6 +167,7 @@ int rp_deposit_impl(rp_ctx* ctx, const double* x, const double* y, const double*
   const int nbins = c.nx * c.ny;  // + 1 "lost" bin with key nbins
   cudaStream_t st = ctx->stream;
   ctx->last_n = n;
+  ProfScope ps(ctx, PK_DEPOSIT);
   if (n > 0) {
     int T = 256;
     k_bin<<<(unsigned)((n + T - 1) / T), T, 0, st>>>(n, x, y, ux, uy, *fk, c.hx, c.hy, c.nx,
@@ -214,6 +215,7 @@ int rp_append_impl(rp_ctx* ctx, const double* parts, int32_t n_parts, const rp_f
   int s = slot_of(knew, ctx->H);
   double* slot = ctx->ring + (size_t)s * ctx->slot_doubles;
   int npts = c.nx * c.ny;
+  ProfScope ps(ctx, PK_APPEND);
   k_append<<<(npts + 255) / 256, 256, 0, st>>>(c.nx, c.ny, ctx->PX, parts, n_parts, slot);
   RP_CHECK_LAUNCH();
   ctx->fh[s] = *fk;

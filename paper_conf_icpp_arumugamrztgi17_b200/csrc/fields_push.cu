@@ -118,6 +118,7 @@ int rp_fields_impl(rp_ctx* ctx, const double* phi, const double* ax, const doubl
   rp_frame Fk = ctx->fh[slot_of(ctx->k, ctx->H)];
   rp_frame Fm = ctx->fh[slot_of(ctx->k - 1, ctx->H)];
   int npts = c.nx * c.ny;
+  ProfScope ps(ctx, PK_FIELDS);
   k_fields<<<(npts + 255) / 256, 256, 0, ctx->stream>>>(c.nx, c.ny, c.hx, c.hy, c.c, c.dt, Fk, Fm,
                                                          have_prev, phi, ax, ay, axp, ayp, ex, ey, bz);
   RP_CHECK_LAUNCH();
@@ -132,6 +133,7 @@ int rp_push_impl(rp_ctx* ctx, double* x, double* y, double* ux, double* uy, int6
   if (n == 0) return RP_OK;
   if (!x || !y || !ux || !uy || !ex || !ey || !bz) return rp_fail(ctx, RP_EINVAL, "push: null array");
   rp_frame Fk = ctx->fh[slot_of(ctx->k, ctx->H)];
+  ProfScope ps(ctx, PK_PUSH);
   k_push<<<(unsigned)((n + 255) / 256), 256, 0, ctx->stream>>>(n, x, y, ux, uy, Fk, c.nx, c.ny,
                                                                 1.0 / c.hx, 1.0 / c.hy, c.c, c.dt,
                                                                 qmc, bz_ext, ex, ey, bz);

@@ -395,8 +395,100 @@ __device__ int arcs(const Item& it, const Params& P, double cu, double cv, doubl
 struct WarpSmem {
   double r[16], cu[16], cv[16], w0[16], w1[16], w2[16], wk[16], wg[16];
   double th1[16][kMaxArcs], dth[16][kMaxArcs];
-  int na[16], off[17];
+  int na[16], cnt[16];
 };
+
+constexpr int kChunk = 5, kNChunks = 3;  // 15 r' nodes = 3 chunks of 5
+
+// One theta slot e of the r' nodes 5*ch .. 5*ch+4 of the current segment.
+template <int KIND>
+__device__ __forceinline__ void eval_chunk(const Item& it, const Params& P, const WarpSmem& S,
+                                           const double2* __restrict__ trig_full, int e, int ch,
+                                           int N, double wfull, double third, double& k0,
+                                           double& k1, double& k2, double& g0, double& g1,
+                                           double& g2) {
+  int cix = -1000000, ciy = -1000000;
+  double st[3][9][3];  // [level][3*b + a][component] of the cached stencil
+#pragma unroll
+  for (int l = 0; l < 3; ++l)
+#pragma unroll
+    for (int i = 0; i < 9; ++i) st[l][i][0] = st[l][i][1] = st[l][i][2] = 0.0;
+#pragma unroll
+  for (int t = 0; t < kChunk; ++t) {
+    const int n = kChunk * ch + t;
+    if (e >= S.cnt[n]) continue;
+    const int na = S.na[n];
+    double cs, sn, w;
+    if (na < 0) {
+      const double2 tr = trig_full[e];
+      cs = tr.x;
+      sn = tr.y;
+      w = wfull;
+    } else {
+      const int q = e / (N + 1);
+      const int mm = e - q * (N + 1);
+      const double d = S.dth[n][q];
+      sincos(S.th1[n][q] + (double)mm * d, &sn, &cs);
+      const double coef = (mm == 0 || mm == N) ? 1.0 : ((mm & 1) ? 4.0 : 2.0);
+      w = coef * d * third;
+    }
+    const double r = S.r[n];
+    const double u = S.cu[n] + r * cs, v = S.cv[n] + r * sn;
+    double f0, f1, f2;
+    if (KIND == RP_SRC_GRID) {
+      const double tx = u * P.inv_hx, ty = v * P.inv_hy;
+      const double fx = floor(tx + 0.5), fy = floor(ty + 0.5);
+      const double dx = tx - fx, dy = ty - fy;
+      const double ax = 0.5 - dx, bx = 0.5 + dx, ay = 0.5 - dy, by = 0.5 + dy;
+      const double wx[3] = {0.5 * ax * ax, 0.75 - dx * dx, 0.5 * bx * bx};
+      const double wy[3] = {0.5 * ay * ay, 0.75 - dy * dy, 0.5 * by * by};
+      // clamp keeps every stencil inside the zero border (memory guard only)
+      const int ix = (int)fmin(fmax(fx, -2.0), (double)(P.nx + 1));
+      const int iy = (int)fmin(fmax(fy, -2.0), (double)(P.ny + 1));
+      if (ix != cix || iy != ciy) {
+        cix = ix;
+        ciy = iy;
+        const size_t base = (size_t)4 * ((iy - 1) * P.PX + (ix - 1));
+        const double* g[3] = {it.g0, it.g1, it.g2};
+#pragma unroll
+        for (int l = 0; l < 3; ++l)
+#pragma unroll
+          for (int b = 0; b < 3; ++b)
+#pragma unroll
+            for (int a = 0; a < 3; ++a) {
+              const size_t o = base + (size_t)4 * (b * P.PX + a);
+              const double2 m01 = __ldg(reinterpret_cast<const double2*>(g[l] + o));
+              st[l][3 * b + a][0] = m01.x;
+              st[l][3 * b + a][1] = m01.y;
+              st[l][3 * b + a][2] = __ldg(g[l] + o + 2);
+            }
+      }
+      double s[3][3];
+#pragma unroll
+      for (int l = 0; l < 3; ++l) {
+        s[l][0] = s[l][1] = s[l][2] = 0.0;
+#pragma unroll
+        for (int b = 0; b < 3; ++b)
+#pragma unroll
+          for (int a = 0; a < 3; ++a) {
+            const double ww = wx[a] * wy[b];
+            s[l][0] += ww * st[l][3 * b + a][0];
+            s[l][1] += ww * st[l][3 * b + a][1];
+            s[l][2] += ww * st[l][3 * b + a][2];
+          }
+      }
+      const double w0 = S.w0[n], w1 = S.w1[n], w2 = S.w2[n];
+      f0 = w0 * s[0][0] + w1 * s[1][0] + w2 * s[2][0];
+      f1 = w0 * s[0][1] + w1 * s[1][1] + w2 * s[2][1];
+      f2 = w0 * s[0][2] + w1 * s[1][2] + w2 * s[2][2];
+    } else {
+      integrand<KIND>(it, P, u, v, S.w0[n], S.w1[n], S.w2[n], f0, f1, f2);
+    }
+    const double wk = w * S.wk[n], wg = w * S.wg[n];
+    k0 += wk * f0; k1 += wk * f1; k2 += wk * f2;
+    g0 += wg * f0; g1 += wg * f1; g2 += wg * f2;
+  }
+}
 
 __device__ __forceinline__ double warp_sum(double v) {
 #pragma unroll
@@ -469,38 +561,20 @@ __global__ void __launch_bounds__(32 * kWarps) k_integrate(
         int y = __shfl_up_sync(0xffffffffu, incl, o);
         if (lane >= o) incl += y;
       }
-      if (lane < 15) S.off[lane] = incl - cnt;
+      if (lane < 16) S.cnt[lane] = lane < 15 ? cnt : 0;
       const int E = __shfl_sync(0xffffffffu, incl, 31);
-      if (lane == 15) S.off[15] = E;
       __syncwarp();
-      // ---- evaluation phase: all lanes sweep the flattened (node, arc, theta) list
+      // ---- evaluation phase: lane <-> (theta slot e, chunk c of kChunk r' nodes).  In a
+      // deep segment the points X_{n,e} of one chunk fall in the same cell, so the 27-node x
+      // 3-component stencil is loaded once into registers and reused across the chunk.
+      int emax = cnt;
+#pragma unroll
+      for (int o = 16; o > 0; o >>= 1) emax = max(emax, __shfl_xor_sync(0xffffffffu, emax, o));
       double k0 = 0.0, k1 = 0.0, k2 = 0.0, g0 = 0.0, g1 = 0.0, g2 = 0.0;
-      int n = 0;
-      for (int e = lane; e < E; e += 32) {
-        while (e >= S.off[n + 1]) ++n;
-        const int local = e - S.off[n];
-        const int na = S.na[n];
-        double cs, sn, w;
-        if (na < 0) {
-          const double2 t = trig_full[local];
-          cs = t.x;
-          sn = t.y;
-          w = wfull;
-        } else {
-          const int q = local / (N + 1);
-          const int mm = local - q * (N + 1);
-          const double d = S.dth[n][q];
-          sincos(S.th1[n][q] + (double)mm * d, &sn, &cs);
-          const double coef = (mm == 0 || mm == N) ? 1.0 : ((mm & 1) ? 4.0 : 2.0);
-          w = coef * d * third;
-        }
-        const double r = S.r[n];
-        double f0, f1, f2;
-        integrand<KIND>(it, P, S.cu[n] + r * cs, S.cv[n] + r * sn, S.w0[n], S.w1[n], S.w2[n],
-                        f0, f1, f2);
-        const double wk = w * S.wk[n], wg = w * S.wg[n];
-        k0 += wk * f0; k1 += wk * f1; k2 += wk * f2;
-        g0 += wg * f0; g1 += wg * f1; g2 += wg * f2;
+      const int units = emax * kNChunks;
+      for (int u = lane; u < units; u += 32) {
+        const int e = u / kNChunks, ch = u - e * kNChunks;
+        eval_chunk<KIND>(it, P, S, trig_full, e, ch, N, wfull, third, k0, k1, k2, g0, g1, g2);
       }
       k0 = warp_sum(k0); k1 = warp_sum(k1); k2 = warp_sum(k2);
       g0 = warp_sum(g0); g1 = warp_sum(g1); g2 = warp_sum(g2);
@@ -695,27 +769,37 @@ static int run_potentials(rp_ctx* ctx, const Params& P, int32_t rank, int32_t wo
   }
   RP_CUDA(cudaMemsetAsync(ctx->counters, 0, 16 * sizeof(unsigned long long), st));
   if (nd > 0) {
-    k_clip<KIND><<<(unsigned)((nd + 255) / 256), 256, 0, st>>>(
-        P, owner, rank, ctx->has_forecast ? ctx->cost_prev : nullptr, ctx->clipAB,
-        ctx->sched_key, ctx->sched_idx, ctx->counters);
-    RP_CHECK_LAUNCH();
-    size_t tmp = 0;
-    RP_CUDA(cub::DeviceRadixSort::SortPairs(nullptr, tmp, ctx->sched_key, ctx->sched_key_sorted,
-                                            ctx->sched_idx, ctx->sched_order, (int)nd, 0, 16, st));
-    int rc = rp_ensure_cub_tmp(ctx, tmp);
-    if (rc) return rc;
-    tmp = ctx->cub_tmp_bytes;
-    RP_CUDA(cub::DeviceRadixSort::SortPairs(ctx->cub_tmp, tmp, ctx->sched_key,
-                                            ctx->sched_key_sorted, ctx->sched_idx,
-                                            ctx->sched_order, (int)nd, 0, 16, st));
+    {
+      ProfScope ps(ctx, PK_CLIP);
+      k_clip<KIND><<<(unsigned)((nd + 255) / 256), 256, 0, st>>>(
+          P, owner, rank, ctx->has_forecast ? ctx->cost_prev : nullptr, ctx->clipAB,
+          ctx->sched_key, ctx->sched_idx, ctx->counters);
+      RP_CHECK_LAUNCH();
+    }
+    {
+      ProfScope ps(ctx, PK_SORT);
+      size_t tmp = 0;
+      RP_CUDA(cub::DeviceRadixSort::SortPairs(nullptr, tmp, ctx->sched_key, ctx->sched_key_sorted,
+                                              ctx->sched_idx, ctx->sched_order, (int)nd, 0, 16, st));
+      int rc = rp_ensure_cub_tmp(ctx, tmp);
+      if (rc) return rc;
+      tmp = ctx->cub_tmp_bytes;
+      RP_CUDA(cub::DeviceRadixSort::SortPairs(ctx->cub_tmp, tmp, ctx->sched_key,
+                                              ctx->sched_key_sorted, ctx->sched_idx,
+                                              ctx->sched_order, (int)nd, 0, 16, st));
+    }
     int occ = 0;
     RP_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_integrate<KIND>, 32 * kWarps, 0));
     if (occ < 1) occ = 1;
-    k_integrate<KIND><<<ctx->sm_count * occ, 32 * kWarps, 0, st>>>(
-        P, ctx->sched_order, ctx->clipAB, ctx->trig_full, ctx->item_val, ctx->item_cnt,
-        ctx->item_aux, ctx->counters);
-    RP_CHECK_LAUNCH();
+    {
+      ProfScope ps(ctx, PK_INTEGRATE);
+      k_integrate<KIND><<<ctx->sm_count * occ, 32 * kWarps, 0, st>>>(
+          P, ctx->sched_order, ctx->clipAB, ctx->trig_full, ctx->item_val, ctx->item_cnt,
+          ctx->item_aux, ctx->counters);
+      RP_CHECK_LAUNCH();
+    }
   }
+  ProfScope ps_red(ctx, PK_REDUCE);
   k_reduce<<<(P.npts + 255) / 256, 256, 0, st>>>(
       P.npts, P.kmax, P.kap, ctx->sched_key, ctx->item_val, ctx->item_cnt, ctx->item_aux, owner,
       rank, row, world, phi, ax, ay, err, nseg, shard_out, ctx->cost_prev, ctx->nseg_prev_pt,

@@ -54,6 +54,11 @@ void free_all(rp_ctx* c) {
                   c->mesh_d};
   for (void* p : ptrs)
     if (p) cudaFree(p);
+  for (auto& r : c->prof) {
+    cudaEventDestroy(r.a);
+    cudaEventDestroy(r.b);
+  }
+  for (auto e : c->ev_pool) cudaEventDestroy(e);
   delete[] c->fh;
 }
 
@@ -78,6 +83,43 @@ const char* rp_strerror(int code) {
 const char* rp_last_error(const rp_ctx* ctx) { return ctx ? ctx->err.c_str() : "null context"; }
 
 int64_t rp_launch_count(const rp_ctx* ctx) { return ctx ? ctx->launches : 0; }
+
+int rp_profile_enable(rp_ctx* ctx, int32_t enable) {
+  if (!ctx) return RP_EINVAL;
+  RP_CUDA(cudaStreamSynchronize(ctx->stream));
+  for (auto& r : ctx->prof) {
+    ctx->ev_pool.push_back(r.a);
+    ctx->ev_pool.push_back(r.b);
+  }
+  ctx->prof.clear();
+  for (double& v : ctx->prof_acc) v = 0.0;
+  ctx->prof_integrate_launches = 0;
+  ctx->prof_on = enable ? 1 : 0;
+  return RP_OK;
+}
+
+int rp_profile_read(rp_ctx* ctx, rp_profile* out) {
+  if (!ctx || !out) return RP_EINVAL;
+  RP_CUDA(cudaStreamSynchronize(ctx->stream));
+  for (auto& r : ctx->prof) {
+    float ms = 0.f;
+    RP_CUDA(cudaEventElapsedTime(&ms, r.a, r.b));
+    ctx->prof_acc[r.kind] += ms;
+    ctx->ev_pool.push_back(r.a);
+    ctx->ev_pool.push_back(r.b);
+  }
+  ctx->prof.clear();
+  out->deposit_ms = ctx->prof_acc[PK_DEPOSIT];
+  out->append_ms = ctx->prof_acc[PK_APPEND];
+  out->clip_ms = ctx->prof_acc[PK_CLIP];
+  out->sort_ms = ctx->prof_acc[PK_SORT];
+  out->integrate_ms = ctx->prof_acc[PK_INTEGRATE];
+  out->reduce_ms = ctx->prof_acc[PK_REDUCE];
+  out->fields_ms = ctx->prof_acc[PK_FIELDS];
+  out->push_ms = ctx->prof_acc[PK_PUSH];
+  out->integrate_launches = ctx->prof_integrate_launches;
+  return RP_OK;
+}
 
 int rp_create(const rp_config* cfg, rp_ctx** out) {
   if (!out) return RP_EINVAL;

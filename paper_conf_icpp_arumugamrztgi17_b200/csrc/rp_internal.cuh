@@ -8,6 +8,7 @@
 #include <string.h>
 
 #include <string>
+#include <vector>
 
 #include "../../include/rp.h"
 
@@ -75,6 +76,48 @@ struct rp_ctx {
 
   int64_t launches = 0;
   std::string err;
+
+  // event timing (rp_profile_enable / rp_profile_read)
+  struct ProfRec { int kind; cudaEvent_t a, b; };
+  int prof_on = 0;
+  std::vector<ProfRec> prof;
+  std::vector<cudaEvent_t> ev_pool;
+  double prof_acc[8] = {0, 0, 0, 0, 0, 0, 0, 0};
+  int64_t prof_integrate_launches = 0;
+};
+
+enum { PK_DEPOSIT = 0, PK_APPEND, PK_CLIP, PK_SORT, PK_INTEGRATE, PK_REDUCE, PK_FIELDS, PK_PUSH };
+
+static inline cudaEvent_t prof_event(rp_ctx* ctx) {
+  if (!ctx->ev_pool.empty()) {
+    cudaEvent_t e = ctx->ev_pool.back();
+    ctx->ev_pool.pop_back();
+    return e;
+  }
+  cudaEvent_t e = nullptr;
+  cudaEventCreate(&e);
+  return e;
+}
+
+// RAII: records an event pair around the enclosed launches when profiling is on
+struct ProfScope {
+  rp_ctx* ctx;
+  int kind;
+  cudaEvent_t a = nullptr;
+  ProfScope(rp_ctx* c, int k) : ctx(c), kind(k) {
+    if (ctx->prof_on) {
+      a = prof_event(ctx);
+      cudaEventRecord(a, ctx->stream);
+    }
+  }
+  ~ProfScope() {
+    if (a) {
+      cudaEvent_t b = prof_event(ctx);
+      cudaEventRecord(b, ctx->stream);
+      ctx->prof.push_back({kind, a, b});
+      if (kind == PK_INTEGRATE) ctx->prof_integrate_launches++;
+    }
+  }
 };
 
 // ---------------------------------------------------------------- error helpers

@@ -41,6 +41,16 @@ class rp_deposit_info(C.Structure):
     _fields_ = [("n_lost", C.c_int64), ("q_lost", C.c_double), ("q_total", C.c_double)]
 
 
+class rp_profile(C.Structure):
+    _fields_ = [("deposit_ms", C.c_double), ("append_ms", C.c_double), ("clip_ms", C.c_double),
+                ("sort_ms", C.c_double), ("integrate_ms", C.c_double), ("reduce_ms", C.c_double),
+                ("fields_ms", C.c_double), ("push_ms", C.c_double),
+                ("integrate_launches", C.c_int64)]
+
+    def as_dict(self) -> dict:
+        return {k: getattr(self, k) for k, _ in self._fields_}
+
+
 class rp_potential_info(C.Structure):
     _fields_ = [("evals", C.c_int64), ("nodes", C.c_int64), ("segments", C.c_int64),
                 ("leaves", C.c_int64), ("capped", C.c_int64), ("ties", C.c_int64),
@@ -62,6 +72,8 @@ _SIG = {
     "rp_strerror": (C.c_char_p, [C.c_int]),
     "rp_last_error": (C.c_char_p, [_vp]),
     "rp_launch_count": (_i64, [_vp]),
+    "rp_profile_enable": (C.c_int, [_vp, _i32]),
+    "rp_profile_read": (C.c_int, [_vp, _P(rp_profile)]),
     "rp_create": (C.c_int, [_P(rp_config), _P(_vp)]),
     "rp_destroy": (None, [_vp]),
     "rp_set_stream": (C.c_int, [_vp, _vp]),
@@ -163,6 +175,16 @@ def rp_last_error(ctx) -> str:
 
 def rp_launch_count(ctx) -> int:
     return _lib.rp_launch_count(ctx)
+
+
+def rp_profile_enable(ctx, enable=True) -> None:
+    _check(_lib.rp_profile_enable(ctx, int(bool(enable))), ctx, "rp_profile_enable")
+
+
+def rp_profile_read(ctx) -> rp_profile:
+    out = rp_profile()
+    _check(_lib.rp_profile_read(ctx, C.byref(out)), ctx, "rp_profile_read")
+    return out
 
 
 def rp_create(nx, ny, hx, hy, history_depth, c, dt, tau, n_theta=64, max_depth=30, n_root=2,

@@ -1,0 +1,108 @@
+"""One time step of the paper's loop on one GPU per process, optionally sharded
+over ranks (mesh points sharded, history replicated).
+
+Per step k on every rank (torch.distributed is plumbing only; every arithmetic step
+runs in librp's kernels):
+
+  world == 1:  rp_deposit_step -> rp_compute_potentials
+  world  > 1:  rp_deposit(local particle shard) -> all_gather(partial grids)
+               -> rp_history_append(partials in rank order)              [replicated ring]
+               -> rp_compute_potentials_shard(rank)                      [owned points]
+               -> all_gather(shards) -> rp_shard_scatter                 [full mesh]
+  then         rp_compute_fields (replicated) -> rp_push_particles (local shard)
+
+``ops`` defaults to the librp binding; tests substitute a CPU stand-in to exercise the
+multi-process plumbing with the gloo backend.
+"""
+from __future__ import annotations
+
+import numpy as np
+import torch
+
+import workloads as W
+
+
+class Simulation:
+    def __init__(self, cfg: W.Config, device=None, group=None, ops=None, particles=None):
+        if ops is None:
+            from . import rp as ops
+        self.ops = ops
+        self.cfg = cfg
+        self.group = group
+        if group is not None:
+            import torch.distributed as dist
+            self.rank, self.world = dist.get_rank(group), dist.get_world_size(group)
+        else:
+            self.rank, self.world = 0, 1
+        self.device = torch.device("cuda", torch.cuda.current_device()) if device is None else torch.device(device)
+        dev_index = self.device.index if self.device.type == "cuda" else 0
+        self.ctx = ops.rp_create(cfg.nx, cfg.ny, cfg.hx, cfg.hy, cfg.kappa_max, cfg.c, cfg.dt,
+                                 cfg.tau, cfg.n_theta, cfg.max_depth, cfg.n_root, dev_index or 0)
+        if self.device.type == "cuda":
+            ops.rp_set_stream(self.ctx, torch.cuda.current_stream(self.device))
+        ops.rp_history_init(self.ctx, cfg.n_pre, W.frames(cfg, range(-cfg.n_pre, 0)), None, True)
+        x, y, ux, uy = W.particles(cfg) if particles is None else particles
+        n = len(x)
+        lo, hi = (n * self.rank) // self.world, (n * (self.rank + 1)) // self.world
+        f64 = dict(dtype=torch.float64, device=self.device)
+        self.x, self.y, self.ux, self.uy = (torch.tensor(np.ascontiguousarray(a[lo:hi]), **f64)
+                                            for a in (x, y, ux, uy))
+        self.q = 1.0 / n
+        npts = cfg.nx * cfg.ny
+        self.npts = npts
+        self.phi, self.err, self.ex, self.ey, self.bz = (torch.zeros(npts, **f64) for _ in range(5))
+        self.A = [(torch.zeros(npts, **f64), torch.zeros(npts, **f64)) for _ in range(2)]
+        self.nseg = torch.zeros(npts, dtype=torch.int32, device=self.device)
+        self.k = 0
+        if self.world > 1:
+            self.partial = torch.zeros((cfg.ny, cfg.nx, 4), **f64)
+            self.partials = torch.zeros((self.world, cfg.ny, cfg.nx, 4), **f64)
+            cap = ops.rp_shard_capacity(self.ctx, self.world)
+            self.shard = torch.zeros((cap, 6), **f64)
+            self.shards = torch.zeros((self.world, cap, 6), **f64)
+
+    # ------------------------------------------------------------------
+    @property
+    def ax(self):
+        """A_x of the last completed step."""
+        return self.A[(self.k - 1) % 2][0]
+
+    @property
+    def ay(self):
+        return self.A[(self.k - 1) % 2][1]
+
+    def step(self, info: bool = False):
+        """Advance one step; returns rp_potential_info (syncs) when info=True."""
+        import torch.distributed as dist
+        ops, cfg = self.ops, self.cfg
+        fk = W.frame(cfg, self.k)
+        ax, ay = self.A[self.k % 2]
+        axp, ayp = self.A[(self.k + 1) % 2]
+        if self.world == 1:
+            ops.rp_deposit_step(self.ctx, self.x, self.y, self.ux, self.uy, self.q, fk)
+            inf = ops.rp_compute_potentials(self.ctx, self.phi, ax, ay, self.err, self.nseg, info=info)
+        else:
+            ops.rp_deposit(self.ctx, self.x, self.y, self.ux, self.uy, self.q, fk, self.partial)
+            dist.all_gather_into_tensor(self.partials, self.partial, group=self.group)
+            ops.rp_history_append(self.ctx, self.partials, self.world, fk)
+            _, inf = ops.rp_compute_potentials_shard(self.ctx, self.rank, self.world, self.shard, info=info)
+            dist.all_gather_into_tensor(self.shards, self.shard, group=self.group)
+            ops.rp_shard_scatter(self.ctx, self.shards, self.world, self.phi, ax, ay, self.err, self.nseg)
+        first = self.k == 0
+        ops.rp_compute_fields(self.ctx, self.phi, ax, ay, None if first else axp,
+                              None if first else ayp, self.ex, self.ey, self.bz)
+        ops.rp_push_particles(self.ctx, self.x, self.y, self.ux, self.uy, cfg.q_over_mc, cfg.bz_ext,
+                              self.ex, self.ey, self.bz)
+        self.k += 1
+        return inf
+
+    def close(self):
+        if self.ctx is not None:
+            self.ops.rp_destroy(self.ctx)
+            self.ctx = None
+
+    def __del__(self):  # pragma: no cover
+        try:
+            self.close()
+        except Exception:
+            pass
