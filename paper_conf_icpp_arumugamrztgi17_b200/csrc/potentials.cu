@@ -286,15 +286,36 @@ __device__ __forceinline__ void integrand(const Item& it, const Params& P, doubl
   f2 = rho * P.sby;
 }
 
+// ------------------------------------------------------------- bounded sincos
+// sin/cos for |x| <= 8 pi: Cody-Waite reduction by pi/2 with a two-term constant (k <= 16 is
+// exact enough for ulp-level accuracy) and the classic fdlibm minimax kernels on
+// [-pi/4, pi/4].  No Payne-Hanek slow path, so it inlines small.
+__device__ __forceinline__ void sincos_b(double x, double* s, double* c) {
+  const double k = rint(x * 0.63661977236758134308);  // 2/pi
+  double r = fma(-k, 1.5707963267948965580, x);
+  r = fma(-k, 6.1232339957367658e-17, r);
+  const double z = r * r;
+  double ps = fma(z, 1.58969099521155010221e-10, -2.50507602534068634195e-08);
+  ps = fma(z, ps, 2.75573137070700676789e-06);
+  ps = fma(z, ps, -1.98412698298579493134e-04);
+  ps = fma(z, ps, 8.33333333332248946124e-03);
+  ps = fma(z, ps, -1.66666666666666324348e-01);
+  const double sr = fma(r * z, ps, r);
+  double pc = fma(z, -1.13596475577881948265e-11, 2.08757232129817482790e-09);
+  pc = fma(z, pc, -2.75573143513906633035e-07);
+  pc = fma(z, pc, 2.48015872894767294178e-05);
+  pc = fma(z, pc, -1.38888888888741095749e-03);
+  pc = fma(z, pc, 4.16666666666666019037e-02);
+  const double cr = fma(z * z, pc, fma(-0.5, z, 1.0));
+  const int q = (int)k & 3;
+  const double ss = (q & 1) ? cr : sr, cc = (q & 1) ? sr : cr;
+  *s = (q & 2) ? -ss : ss;
+  *c = ((q + 1) & 2) ? -cc : cc;
+}
+
 // ------------------------------------------------------------- arcs (R-5)
 __device__ __forceinline__ bool in_rect(double u, double v, const Item& it) {
   return u >= it.U0 && u <= it.U1 && v >= it.V0 && v <= it.V1;
-}
-
-__device__ __forceinline__ void cswap(double& a, double& b) {
-  double lo = fmin(a, b), hi = fmax(a, b);
-  a = lo;
-  b = hi;
 }
 
 // arcs of circle (cu, cv; r) inside the support; returns -1 (full circle) or the count,
@@ -314,86 +335,69 @@ __device__ int arcs(const Item& it, const Params& P, double cu, double cv, doubl
     dth[0] = ((ph + al) - (ph - al)) / N;
     return 1;
   }
-  const double inf = __longlong_as_double(0x7ff0000000000000LL);
+  // Crossings of the circle with the 4 edge lines that lie on the edge (kept compact: the
+  // node phase runs on 15 lanes once per segment, so code size matters more than ILP).
   double t[8];
-#pragma unroll
-  for (int i = 0; i < 8; ++i) t[i] = inf;
-  {
-    double d = (it.U0 - cu) / r;
-    if (fabs(d) < 1.0) {
-      double al = acos(d), c2 = kTwoPi - al;
-      double v1 = cv + r * sin(al), v2 = cv + r * sin(c2);
-      if (v1 >= it.V0 && v1 <= it.V1) t[0] = al;
-      if (v2 >= it.V0 && v2 <= it.V1) t[1] = c2;
+  int n = 0;
+#pragma unroll 1
+  for (int e = 0; e < 4; ++e) {
+    const bool vert = e < 2;
+    const double edge = e == 0 ? it.U0 : e == 1 ? it.U1 : e == 2 ? it.V0 : it.V1;
+    const double d = (edge - (vert ? cu : cv)) / r;
+    if (!(fabs(d) < 1.0)) continue;
+    const double h = r * sqrt(1.0 - d * d);  // r sin(acos d) = r cos(asin d)
+    const double lo = vert ? it.V0 : it.U0, hi = vert ? it.V1 : it.U1;
+    const double o1 = (vert ? cv : cu) + h, o2 = (vert ? cv : cu) - h;
+    double c1, c2;
+    if (vert) {
+      c1 = acos(d);
+      c2 = kTwoPi - c1;
+    } else {
+      const double be = asin(d);
+      c1 = be < 0.0 ? be + kTwoPi : be;
+      c2 = M_PI - be;
     }
-    d = (it.U1 - cu) / r;
-    if (fabs(d) < 1.0) {
-      double al = acos(d), c2 = kTwoPi - al;
-      double v1 = cv + r * sin(al), v2 = cv + r * sin(c2);
-      if (v1 >= it.V0 && v1 <= it.V1) t[2] = al;
-      if (v2 >= it.V0 && v2 <= it.V1) t[3] = c2;
-    }
-    d = (it.V0 - cv) / r;
-    if (fabs(d) < 1.0) {
-      double be = asin(d);
-      double c1 = be < 0.0 ? be + kTwoPi : be, c2 = M_PI - be;
-      double u1 = cu + r * cos(c1), u2 = cu + r * cos(c2);
-      if (u1 >= it.U0 && u1 <= it.U1) t[4] = c1;
-      if (u2 >= it.U0 && u2 <= it.U1) t[5] = c2;
-    }
-    d = (it.V1 - cv) / r;
-    if (fabs(d) < 1.0) {
-      double be = asin(d);
-      double c1 = be < 0.0 ? be + kTwoPi : be, c2 = M_PI - be;
-      double u1 = cu + r * cos(c1), u2 = cu + r * cos(c2);
-      if (u1 >= it.U0 && u1 <= it.U1) t[6] = c1;
-      if (u2 >= it.U0 && u2 <= it.U1) t[7] = c2;
-    }
+    if (o1 >= lo && o1 <= hi) t[n++] = c1;
+    if (o2 >= lo && o2 <= hi) t[n++] = c2;
   }
-  // sorting network (19 comparators) on 8 keys, +inf = absent
-  cswap(t[0], t[1]); cswap(t[2], t[3]); cswap(t[4], t[5]); cswap(t[6], t[7]);
-  cswap(t[0], t[2]); cswap(t[1], t[3]); cswap(t[4], t[6]); cswap(t[5], t[7]);
-  cswap(t[1], t[2]); cswap(t[5], t[6]); cswap(t[0], t[4]); cswap(t[3], t[7]);
-  cswap(t[1], t[5]); cswap(t[2], t[6]);
-  cswap(t[1], t[4]); cswap(t[3], t[6]);
-  cswap(t[2], t[4]); cswap(t[3], t[5]);
-  cswap(t[3], t[4]);
-  if (t[0] == inf) return in_rect(cu + r, cv, it) ? -1 : 0;
-  // unique crossings u_0 < u_1 < ... ; intervals (u_i, u_{i+1}) and (u_last, u_0 + 2 pi)
+  if (n == 0) return in_rect(cu + r, cv, it) ? -1 : 0;
+#pragma unroll 1
+  for (int i = 1; i < n; ++i) {  // insertion sort (n <= 8)
+    double x = t[i];
+    int k = i - 1;
+    while (k >= 0 && t[k] > x) {
+      t[k + 1] = t[k];
+      --k;
+    }
+    t[k + 1] = x;
+  }
+  // unique crossings u_0 < u_1 < ...; keep the intervals (u_i, u_{i+1}) and
+  // (u_last, u_0 + 2 pi) whose midpoint lies inside the rectangle
   int na = 0;
-  double first = t[0], prev = t[0];
-#pragma unroll
-  for (int i = 1; i < 8; ++i) {
-    double cur = t[i];
-    if (cur != inf && cur != prev) {
-      double mid = 0.5 * (prev + cur);
-      double sm, cm;
-      sincos(mid, &sm, &cm);
-      if (in_rect(cu + r * cm, cv + r * sm, it)) {
-        th1[na] = prev;
-        dth[na] = (cur - prev) / N;
-        ++na;
-      }
-      prev = cur;
-    }
-  }
-  {
-    double cur = first + kTwoPi;
-    double mid = 0.5 * (prev + cur);
+  double prev = t[0];
+#pragma unroll 1
+  for (int i = 1; i <= n; ++i) {
+    const double cur = i < n ? t[i] : t[0] + kTwoPi;
+    if (i < n && cur == prev) continue;
     double sm, cm;
-    sincos(mid, &sm, &cm);
+    sincos_b(0.5 * (prev + cur), &sm, &cm);
     if (in_rect(cu + r * cm, cv + r * sm, it)) {
       th1[na] = prev;
       dth[na] = (cur - prev) / N;
       ++na;
     }
+    prev = cur;
   }
   return na;
 }
 
 // ------------------------------------------------------------- k_integrate
+struct __align__(16) NodeRec {
+  double r, cu, cv, w0, w1, w2, wk, wg;  // r', frame-local centre, time weights, hw*w_GK, hw*w_G7
+};
+
 struct WarpSmem {
-  double r[16], cu[16], cv[16], w0[16], w1[16], w2[16], wk[16], wg[16];
+  NodeRec node[16];
   double th1[16][kMaxArcs], dth[16][kMaxArcs];
   int na[16], cnt[16];
 };
@@ -408,16 +412,14 @@ __device__ __forceinline__ void eval_chunk(const Item& it, const Params& P, cons
                                            double& k1, double& k2, double& g0, double& g1,
                                            double& g2) {
   int cix = -1000000, ciy = -1000000;
-  double st[3][9][3];  // [level][3*b + a][component] of the cached stencil
-#pragma unroll
-  for (int l = 0; l < 3; ++l)
-#pragma unroll
-    for (int i = 0; i < 9; ++i) st[l][i][0] = st[l][i][1] = st[l][i][2] = 0.0;
-#pragma unroll
+  double st[3][9][3];  // [level][3*b + a][component] of the cached stencil (loaded at t = 0)
+  const size_t rs = (size_t)4 * P.PX;  // padded row stride in doubles
+#pragma unroll 1
   for (int t = 0; t < kChunk; ++t) {
     const int n = kChunk * ch + t;
     if (e >= S.cnt[n]) continue;
     const int na = S.na[n];
+    const NodeRec nd = S.node[n];
     double cs, sn, w;
     if (na < 0) {
       const double2 tr = trig_full[e];
@@ -425,15 +427,17 @@ __device__ __forceinline__ void eval_chunk(const Item& it, const Params& P, cons
       sn = tr.y;
       w = wfull;
     } else {
-      const int q = e / (N + 1);
-      const int mm = e - q * (N + 1);
+      int q = 0, mm = e;
+      while (mm > N) {  // arc index without a division (one arc in the common case)
+        mm -= N + 1;
+        ++q;
+      }
       const double d = S.dth[n][q];
-      sincos(S.th1[n][q] + (double)mm * d, &sn, &cs);
+      sincos_b(S.th1[n][q] + (double)mm * d, &sn, &cs);
       const double coef = (mm == 0 || mm == N) ? 1.0 : ((mm & 1) ? 4.0 : 2.0);
       w = coef * d * third;
     }
-    const double r = S.r[n];
-    const double u = S.cu[n] + r * cs, v = S.cv[n] + r * sn;
+    const double u = nd.cu + nd.r * cs, v = nd.cv + nd.r * sn;
     double f0, f1, f2;
     if (KIND == RP_SRC_GRID) {
       const double tx = u * P.inv_hx, ty = v * P.inv_hy;
@@ -443,25 +447,26 @@ __device__ __forceinline__ void eval_chunk(const Item& it, const Params& P, cons
       const double wx[3] = {0.5 * ax * ax, 0.75 - dx * dx, 0.5 * bx * bx};
       const double wy[3] = {0.5 * ay * ay, 0.75 - dy * dy, 0.5 * by * by};
       // clamp keeps every stencil inside the zero border (memory guard only)
-      const int ix = (int)fmin(fmax(fx, -2.0), (double)(P.nx + 1));
-      const int iy = (int)fmin(fmax(fy, -2.0), (double)(P.ny + 1));
+      const int ix = min(max(__double2int_rz(fx), -2), P.nx + 1);
+      const int iy = min(max(__double2int_rz(fy), -2), P.ny + 1);
       if (ix != cix || iy != ciy) {
         cix = ix;
         ciy = iy;
         const size_t base = (size_t)4 * ((iy - 1) * P.PX + (ix - 1));
-        const double* g[3] = {it.g0, it.g1, it.g2};
+        const double* g[3] = {it.g0 + base, it.g1 + base, it.g2 + base};
 #pragma unroll
         for (int l = 0; l < 3; ++l)
 #pragma unroll
-          for (int b = 0; b < 3; ++b)
+          for (int b = 0; b < 3; ++b) {
+            const double* row = g[l] + b * rs;
 #pragma unroll
             for (int a = 0; a < 3; ++a) {
-              const size_t o = base + (size_t)4 * (b * P.PX + a);
-              const double2 m01 = __ldg(reinterpret_cast<const double2*>(g[l] + o));
+              const double2 m01 = __ldg(reinterpret_cast<const double2*>(row + 4 * a));
               st[l][3 * b + a][0] = m01.x;
               st[l][3 * b + a][1] = m01.y;
-              st[l][3 * b + a][2] = __ldg(g[l] + o + 2);
+              st[l][3 * b + a][2] = __ldg(row + 4 * a + 2);
             }
+          }
       }
       double s[3][3];
 #pragma unroll
@@ -477,14 +482,13 @@ __device__ __forceinline__ void eval_chunk(const Item& it, const Params& P, cons
             s[l][2] += ww * st[l][3 * b + a][2];
           }
       }
-      const double w0 = S.w0[n], w1 = S.w1[n], w2 = S.w2[n];
-      f0 = w0 * s[0][0] + w1 * s[1][0] + w2 * s[2][0];
-      f1 = w0 * s[0][1] + w1 * s[1][1] + w2 * s[2][1];
-      f2 = w0 * s[0][2] + w1 * s[1][2] + w2 * s[2][2];
+      f0 = nd.w0 * s[0][0] + nd.w1 * s[1][0] + nd.w2 * s[2][0];
+      f1 = nd.w0 * s[0][1] + nd.w1 * s[1][1] + nd.w2 * s[2][1];
+      f2 = nd.w0 * s[0][2] + nd.w1 * s[1][2] + nd.w2 * s[2][2];
     } else {
-      integrand<KIND>(it, P, u, v, S.w0[n], S.w1[n], S.w2[n], f0, f1, f2);
+      integrand<KIND>(it, P, u, v, nd.w0, nd.w1, nd.w2, f0, f1, f2);
     }
-    const double wk = w * S.wk[n], wg = w * S.wg[n];
+    const double wk = w * nd.wk, wg = w * nd.wg;
     k0 += wk * f0; k1 += wk * f1; k2 += wk * f2;
     g0 += wg * f0; g1 += wg * f1; g2 += wg * f2;
   }
@@ -543,10 +547,11 @@ __global__ void __launch_bounds__(32 * kWarps) k_integrate(
         centre_at(it, P, r, cu, cv, w0, w1, w2);
         double th1[kMaxArcs], dth[kMaxArcs];
         int na = arcs<KIND>(it, P, cu, cv, r, th1, dth);
-        S.r[lane] = r; S.cu[lane] = cu; S.cv[lane] = cv;
-        S.w0[lane] = w0; S.w1[lane] = w1; S.w2[lane] = w2;
-        S.wk[lane] = hw * c_wgk[i];
-        S.wg[lane] = (i & 1) ? hw * c_wg[i >> 1] : (i == 7 ? hw * c_wg[3] : 0.0);
+        NodeRec nr;
+        nr.r = r; nr.cu = cu; nr.cv = cv; nr.w0 = w0; nr.w1 = w1; nr.w2 = w2;
+        nr.wk = hw * c_wgk[i];
+        nr.wg = (i & 1) ? hw * c_wg[i >> 1] : 0.0;  // Gauss nodes are the odd i (i = 7 centre)
+        S.node[lane] = nr;
         S.na[lane] = na;
         for (int q = 0; q < (na > 0 ? na : 0); ++q) {
           S.th1[lane][q] = th1[q];
