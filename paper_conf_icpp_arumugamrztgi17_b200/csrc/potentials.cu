@@ -397,12 +397,20 @@ struct __align__(16) NodeRec {
 };
 
 struct WarpSmem {
+  Item it;  // per-item geometry, kept in shared memory to free registers for the eval loop
   NodeRec node[16];
   double th1[16][kMaxArcs], dth[16][kMaxArcs];
   int na[16], cnt[16];
 };
 
-constexpr int kChunk = 5, kNChunks = 3;  // 15 r' nodes = 3 chunks of 5
+constexpr int kChunk = 5, kNChunks = 3;
+
+// 256-bit read-only load of one padded node record (rho, rho*bx, rho*by, 0): sm_100
+// LDG.E.ENL2.256, one instruction per stencil node.
+__device__ __forceinline__ void ldg_node(const double* p, double& a, double& b, double& c) {
+  double d;
+  asm("ld.global.nc.v4.f64 {%0,%1,%2,%3}, [%4];" : "=d"(a), "=d"(b), "=d"(c), "=d"(d) : "l"(p));
+}  // 15 r' nodes = 3 chunks of 5
 
 // One theta slot e of the r' nodes 5*ch .. 5*ch+4 of the current segment.
 template <int KIND>
@@ -460,12 +468,8 @@ __device__ __forceinline__ void eval_chunk(const Item& it, const Params& P, cons
           for (int b = 0; b < 3; ++b) {
             const double* row = g[l] + b * rs;
 #pragma unroll
-            for (int a = 0; a < 3; ++a) {
-              const double2 m01 = __ldg(reinterpret_cast<const double2*>(row + 4 * a));
-              st[l][3 * b + a][0] = m01.x;
-              st[l][3 * b + a][1] = m01.y;
-              st[l][3 * b + a][2] = __ldg(row + 4 * a + 2);
-            }
+            for (int a = 0; a < 3; ++a)
+              ldg_node(row + 4 * a, st[l][3 * b + a][0], st[l][3 * b + a][1], st[l][3 * b + a][2]);
           }
       }
       double s[3][3];
@@ -523,8 +527,10 @@ __global__ void __launch_bounds__(32 * kWarps) k_integrate(
     const int p = item / P.kmax, j = item % P.kmax;
     const double2 ab = AB[item];
     const double A = ab.x, BA = __dsub_rn(ab.y, ab.x);
-    Item it;
-    setup_item<KIND>(it, P, p, j);
+    __syncwarp();
+    if (lane == 0) setup_item<KIND>(S.it, P, p, j);
+    __syncwarp();
+    const Item& it = S.it;
 
     double s_phi = 0.0, s_ax = 0.0, s_ay = 0.0, s_err = 0.0;
     int nseg = 0, nleaf = 0, capped = 0, ties = 0, maxlev = 0;
