@@ -403,7 +403,10 @@ struct WarpSmem {
   int na[16], cnt[16];
 };
 
-constexpr int kChunk = 5, kNChunks = 3;
+#ifndef RP_CHUNK
+#define RP_CHUNK 5
+#endif
+constexpr int kChunk = RP_CHUNK, kNChunks = 15 / RP_CHUNK;  // 15 r' nodes = kNChunks chunks
 
 // 256-bit read-only load of one padded node record (rho, rho*bx, rho*by, 0): sm_100
 // LDG.E.ENL2.256, one instruction per stencil node.
@@ -427,7 +430,7 @@ __device__ __forceinline__ void eval_chunk(const Item& it, const Params& P, cons
     const int n = kChunk * ch + t;
     if (e >= S.cnt[n]) continue;
     const int na = S.na[n];
-    const NodeRec nd = S.node[n];
+    const NodeRec& nd = S.node[n];  // read at the point of use (register pressure)
     double cs, sn, w;
     if (na < 0) {
       const double2 tr = trig_full[e];
