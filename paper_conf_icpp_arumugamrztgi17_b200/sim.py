@@ -83,10 +83,10 @@ class Simulation:
             inf = ops.rp_compute_potentials(self.ctx, self.phi, ax, ay, self.err, self.nseg, info=info)
         else:
             ops.rp_deposit(self.ctx, self.x, self.y, self.ux, self.uy, self.q, fk, self.partial)
-            dist.all_gather_into_tensor(self.partials, self.partial, group=self.group)
+            dist.all_gather_into_tensor(self.partials.view(-1), self.partial.view(-1), group=self.group)
             ops.rp_history_append(self.ctx, self.partials, self.world, fk)
             _, inf = ops.rp_compute_potentials_shard(self.ctx, self.rank, self.world, self.shard, info=info)
-            dist.all_gather_into_tensor(self.shards, self.shard, group=self.group)
+            dist.all_gather_into_tensor(self.shards.view(-1), self.shard.view(-1), group=self.group)
             ops.rp_shard_scatter(self.ctx, self.shards, self.world, self.phi, ax, ay, self.err, self.nseg)
         first = self.k == 0
         ops.rp_compute_fields(self.ctx, self.phi, ax, ay, None if first else axp,
