@@ -20,7 +20,7 @@ int main() {
   cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
   cudaDeviceGetAttribute(&clk, cudaDevAttrClockRate, dev);
   double* out; cudaMalloc(&out, 8);
-  int blocks = sms * 8, threads = 256, iters = 4096;
+  int blocks = sms * 4, threads = 256, iters = 4096;  // 32 warps / SM
   cudaEvent_t e0, e1; cudaEventCreate(&e0); cudaEventCreate(&e1);
   for (int w = 0; w < 3; ++w) dfma_loop<<<blocks, threads>>>(out, iters, 0.999999, 1e-7);
   float best = 1e30f;
