@@ -425,6 +425,8 @@ __device__ __forceinline__ void eval_chunk(const Item& it, const Params& P, cons
   int cix = -1000000, ciy = -1000000;
   double st[3][9][3];  // [level][3*b + a][component] of the cached stencil (loaded at t = 0)
   const size_t rs = (size_t)4 * P.PX;  // padded row stride in doubles
+  // the full-circle node of slot e is the same for every r' node: one load per unit
+  const double2 trf = __ldg(trig_full + (e < N ? e : 0));
 #pragma unroll 1
   for (int t = 0; t < kChunk; ++t) {
     const int n = kChunk * ch + t;
@@ -433,9 +435,8 @@ __device__ __forceinline__ void eval_chunk(const Item& it, const Params& P, cons
     const NodeRec& nd = S.node[n];  // read at the point of use (register pressure)
     double cs, sn, w;
     if (na < 0) {
-      const double2 tr = trig_full[e];
-      cs = tr.x;
-      sn = tr.y;
+      cs = trf.x;
+      sn = trf.y;
       w = wfull;
     } else {
       int q = 0, mm = e;
