@@ -398,3 +398,54 @@ def test_call_order_errors(torch):
         assert e.value.code == -5
     finally:
         rp.rp_destroy(ctx)
+
+
+# ------------------------------------------------------------------ more product-path cases
+def test_history_init_explicit_grids_and_empty_deposit(torch):
+    """rp_history_init with explicit pre-history grids (rigid = 0), then a step whose local
+    deposit is empty (0 particles): the potentials come from the pre-history alone."""
+    from paper_conf_icpp_arumugamrztgi17_b200 import rp
+    cfg = _bend_small(n=20, kap=12)
+    ring = W.node_gaussian_ring(cfg, k=0, beta=(cfg.beta0, 0.0), amp_of_level=lambda l: 1.0 + 0.02 * l)
+    n_pre = cfg.kappa_max + 1
+    pre_levels = list(range(-n_pre, 0))
+    grids = np.stack([ring[l % cfg.H] for l in pre_levels])
+    ctx = G.make_ctx(cfg)
+    try:
+        rp.rp_history_init(ctx, n_pre, W.frames(cfg, pre_levels),
+                           torch.tensor(grids, dtype=torch.float64, device="cuda"), False)
+        z = torch.zeros(0, dtype=torch.float64, device="cuda")
+        info = rp.rp_deposit_step(ctx, z, z, z, z, 1.0, W.frame(cfg, 0), info=True)
+        assert info.n_lost == 0 and info.q_total == 0.0
+        gpu, _ = G.gpu_potentials(ctx, cfg.nx * cfg.ny)
+        full = ring.copy()
+        full[0 % cfg.H] = 0.0  # step 0 grid is empty
+        pts = np.arange(cfg.nx * cfg.ny)
+        orc = G.oracle_problem(cfg, full, W.ring_frames(cfg, 0), 0, n_pre).potentials(pts)
+        fail, worst, _ = G.compare_potentials(gpu, orc, pts)
+        assert not fail.any(), worst
+    finally:
+        rp.rp_destroy(ctx)
+
+
+@pytest.mark.slow
+def test_potentials_bend_cfg3_full_size_sampled(torch):
+    """Config 3 (128x128, 1e7 particles, full history kappa = 500) through the product path;
+    the oracle computes a stratified sample of 24 points from its own deposit."""
+    from paper_conf_icpp_arumugamrztgi17_b200 import rp
+    cfg = W.config(3)
+    ring, (x, y, ux, uy, q) = _deposit_rigid_ring(cfg)
+    pts = W.sample_points(cfg.nx, cfg.ny, 24, seed=9)
+    orc = G.oracle_problem(cfg, ring, W.ring_frames(cfg, 0), 0, cfg.n_pre).potentials(pts)
+    del ring
+    ctx = G.make_ctx(cfg)
+    try:
+        rp.rp_history_init(ctx, cfg.n_pre, W.frames(cfg, range(-cfg.n_pre, 0)), None, True)
+        xd, yd, uxd, uyd = _dev_arrays(torch, x, y, ux, uy)
+        rp.rp_deposit_step(ctx, xd, yd, uxd, uyd, q, W.frame(cfg, 0))
+        gpu, info = G.gpu_potentials(ctx, cfg.nx * cfg.ny)
+        fail, worst, _ = G.compare_potentials(gpu, orc, pts)
+        assert not fail.any(), (pts[fail][:10], worst)
+        assert info.kappa == cfg.kappa_max
+    finally:
+        rp.rp_destroy(ctx)
