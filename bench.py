@@ -154,6 +154,11 @@ def run_ours(args):
         group = dist.group.WORLD
     cfg = W.config(args.config)
     sim = Simulation(cfg, group=group)
+    sched = args.schedule
+    if sched == "index":
+        rp.rp_set_schedule(sim.ctx, rp.RP_SCHED_INDEX, 1)
+    elif sched.startswith("knn"):
+        rp.rp_set_schedule(sim.ctx, rp.RP_SCHED_KNN, int(sched[3:]))
     dev = torch.device("cuda", local)
     flush = torch.empty(512 * 1024 * 1024 // 8, dtype=torch.float64, device=dev)  # 512 MB > L2
 
@@ -235,7 +240,8 @@ def run_ours(args):
                        "particles": cfg.n_particles, "history_depth": cfg.kappa_max,
                        "tau": cfg.tau, "n_theta": cfg.n_theta, "n_root": cfg.n_root,
                        "parallelism": f"mesh-point shards x{world}, history replicated",
-                       "l2": "flushed between timed steps (512 MB write)"},
+                       "l2": "flushed between timed steps (512 MB write)",
+                       "schedule": args.schedule},
             "fp64_gflops": gflops,
             "work_per_step": {k2: v / args.steps for k2, v in totals.items()},
             "roofline": {"kernel": "k_integrate (GK15 tree integrator)", "bound": "alu",
@@ -384,6 +390,8 @@ def main():
     ap.add_argument("--impl", choices=["ours", "reference"], default="ours")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--schedule", default="persistence",
+                    help="work-order forecast: index | persistence | knn5 | knn9 | knn25")
     args = ap.parse_args()
     if args.warmup < 3 and args.impl == "ours":
         print("warning: fewer than 3 warm-up steps", file=sys.stderr)

@@ -202,6 +202,19 @@ int rp_debug_potentials_analytic(rp_ctx* ctx, int32_t kind, double x0, double y0
                                  const double* amp_host, double* phi, double* ax, double* ay,
                                  double* err, int32_t* nseg, rp_potential_info* info);
 
+/* Work-scheduling forecast (the paper's predictor g, used ONLY to order work; the
+ * results are bit-identical for every policy, R-17):
+ *   RP_SCHED_INDEX        no forecast: (point, subregion) items in index order;
+ *   RP_SCHED_PERSISTENCE  (default) predicted cost of (p, j) = segments it took last step;
+ *   RP_SCHED_KNN          kNN regression over mesh points: predicted cost of (p, j) =
+ *                         mean of last step's cost of (q, j) over the k nearest mesh points q
+ *                         of the comoving mesh (k in {1, 5, 9, 25}; 1 = persistence).
+ * Items are then run longest-predicted-first (LPT). */
+#define RP_SCHED_INDEX 0
+#define RP_SCHED_PERSISTENCE 1
+#define RP_SCHED_KNN 2
+int rp_set_schedule(rp_ctx* ctx, int32_t policy, int32_t k);
+
 /* Per-kernel device time, measured with CUDA events recorded on the context's stream around
  * each launch while profiling is enabled (bench.py's live roofline numbers). */
 typedef struct {

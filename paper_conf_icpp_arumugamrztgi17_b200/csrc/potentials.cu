@@ -166,9 +166,29 @@ __device__ void setup_item(Item& it, const Params& P, int p, int j) {
 }
 
 // ------------------------------------------------------------- k_clip
+// Forecast of the segments of item (p, j) from last step's counts (scheduling only).
+__device__ __forceinline__ unsigned forecast(const uint16_t* __restrict__ cost, int p, int j,
+                                             int nx, int ny, int kmax, int policy, int knn) {
+  if (policy != RP_SCHED_KNN || knn <= 1) return cost[(size_t)p * kmax + j];
+  // kNN regression over the comoving mesh: k nearest nodes in index space
+  const int ix = p % nx, iy = p / nx;
+  const int rad = knn >= 25 ? 2 : 1;
+  unsigned sum = 0, cnt = 0;
+  for (int dy = -rad; dy <= rad; ++dy)
+    for (int dx = -rad; dx <= rad; ++dx) {
+      if (knn == 5 && dx != 0 && dy != 0) continue;  // 4-neighbour cross + centre
+      const int x = ix + dx, y = iy + dy;
+      if (x < 0 || x >= nx || y < 0 || y >= ny) continue;
+      sum += cost[((size_t)y * nx + x) * kmax + j];
+      ++cnt;
+    }
+  return cnt ? (sum + cnt / 2) / cnt : 0u;
+}
+
 template <int KIND>
 __global__ void k_clip(Params P, const int32_t* __restrict__ owner, int rank,
-                       const uint16_t* __restrict__ cost_prev, double2* __restrict__ AB,
+                       const uint16_t* __restrict__ cost_prev, int policy, int knn,
+                       double2* __restrict__ AB,
                        uint16_t* __restrict__ key, int32_t* __restrict__ iota,
                        unsigned long long* __restrict__ counters) {
   int64_t id = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
@@ -215,7 +235,7 @@ __global__ void k_clip(Params P, const int32_t* __restrict__ owner, int rank,
         B = lo;
       }
       if (A < B) {
-        unsigned c = cost_prev ? cost_prev[id] : 0u;
+        unsigned c = cost_prev ? forecast(cost_prev, p, j, P.nx, P.ny, P.kmax, policy, knn) : 0u;
         kk = (uint16_t)(0xFFFEu - (c < 0xFFFEu ? c : 0xFFFEu));
       }
     }
@@ -787,7 +807,9 @@ static int run_potentials(rp_ctx* ctx, const Params& P, int32_t rank, int32_t wo
     {
       ProfScope ps(ctx, PK_CLIP);
       k_clip<KIND><<<(unsigned)((nd + 255) / 256), 256, 0, st>>>(
-          P, owner, rank, ctx->has_forecast ? ctx->cost_prev : nullptr, ctx->clipAB,
+          P, owner, rank,
+          (ctx->has_forecast && ctx->sched_policy != RP_SCHED_INDEX) ? ctx->cost_prev : nullptr,
+          ctx->sched_policy, ctx->sched_k, ctx->clipAB,
           ctx->sched_key, ctx->sched_idx, ctx->counters);
       RP_CHECK_LAUNCH();
     }

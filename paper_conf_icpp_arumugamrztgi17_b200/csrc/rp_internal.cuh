@@ -59,6 +59,8 @@ struct rp_ctx {
   double* amp_dev = nullptr;        // [H] analytic amplitudes
   double2* trig_full = nullptr;     // [n_theta] (cos, sin)(2 pi m / n_theta)
   int has_forecast = 0;
+  int sched_policy = 1;             // RP_SCHED_*
+  int sched_k = 9;                  // kNN neighbours
 
   // sharding scratch
   int32_t* point_key = nullptr;     // per point predicted work key

@@ -17,6 +17,7 @@ _HERE = os.path.dirname(os.path.abspath(__file__))
 LIB_PATH = os.path.join(_HERE, "librp.so")
 
 RP_SRC_GRID, RP_SRC_GAUSS, RP_SRC_DISK = 0, 1, 2
+RP_SCHED_INDEX, RP_SCHED_PERSISTENCE, RP_SCHED_KNN = 0, 1, 2
 
 
 class RpError(RuntimeError):
@@ -73,6 +74,7 @@ _SIG = {
     "rp_last_error": (C.c_char_p, [_vp]),
     "rp_launch_count": (_i64, [_vp]),
     "rp_profile_enable": (C.c_int, [_vp, _i32]),
+    "rp_set_schedule": (C.c_int, [_vp, _i32, _i32]),
     "rp_profile_read": (C.c_int, [_vp, _P(rp_profile)]),
     "rp_create": (C.c_int, [_P(rp_config), _P(_vp)]),
     "rp_destroy": (None, [_vp]),
@@ -175,6 +177,10 @@ def rp_last_error(ctx) -> str:
 
 def rp_launch_count(ctx) -> int:
     return _lib.rp_launch_count(ctx)
+
+
+def rp_set_schedule(ctx, policy, k=9) -> None:
+    _check(_lib.rp_set_schedule(ctx, int(policy), int(k)), ctx, "rp_set_schedule")
 
 
 def rp_profile_enable(ctx, enable=True) -> None:

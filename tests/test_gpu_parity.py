@@ -449,3 +449,23 @@ def test_potentials_bend_cfg3_full_size_sampled(torch):
         assert info.kappa == cfg.kappa_max
     finally:
         rp.rp_destroy(ctx)
+
+
+@pytest.mark.parametrize("policy,k", [(0, 1), (2, 9), (2, 25), (2, 5)])
+def test_schedule_policies_bit_identical(torch, policy, k):
+    """The forecast (paper's predictor g) only orders the work: every policy gives
+    bit-identical results to the default persistence forecast over several steps."""
+    from paper_conf_icpp_arumugamrztgi17_b200 import rp
+    from paper_conf_icpp_arumugamrztgi17_b200.sim import Simulation
+    cfg = W.config(1)
+    a, b = Simulation(cfg), Simulation(cfg)
+    try:
+        rp.rp_set_schedule(b.ctx, policy, k)
+        for _ in range(3):
+            a.step()
+            b.step()
+            for t1, t2 in ((a.phi, b.phi), (a.ax, b.ax), (a.ay, b.ay), (a.nseg, b.nseg), (a.ex, b.ex)):
+                assert torch.equal(t1, t2)
+    finally:
+        a.close()
+        b.close()
