@@ -435,21 +435,21 @@ __device__ __forceinline__ void ldg_node(const double* p, double& a, double& b, 
   asm("ld.global.nc.v4.f64 {%0,%1,%2,%3}, [%4];" : "=d"(a), "=d"(b), "=d"(c), "=d"(d) : "l"(p));
 }  // 15 r' nodes = 3 chunks of 5
 
-// One theta slot e of the r' nodes 5*ch .. 5*ch+4 of the current segment.
+// Theta slot e of the r' nodes n0 .. n1-1 of the current segment.  The 27-node x 3-component
+// stencil cache (st, cix, ciy) belongs to the caller, so it survives across calls: a lane that
+// evaluates the same slot in consecutive (radially adjacent) deep segments keeps its cell.
 template <int KIND>
-__device__ __forceinline__ void eval_chunk(const Item& it, const Params& P, const WarpSmem& S,
-                                           const double2* __restrict__ trig_full, int e, int ch,
-                                           int N, double wfull, double third, double& k0,
+__device__ __forceinline__ void eval_nodes(const Item& it, const Params& P, const WarpSmem& S,
+                                           const double2* __restrict__ trig_full, int e, int n0,
+                                           int n1, int N, double wfull, double third,
+                                           double (&st)[3][9][3], int& cix, int& ciy, double& k0,
                                            double& k1, double& k2, double& g0, double& g1,
                                            double& g2) {
-  int cix = -1000000, ciy = -1000000;
-  double st[3][9][3];  // [level][3*b + a][component] of the cached stencil (loaded at t = 0)
   const size_t rs = (size_t)4 * P.PX;  // padded row stride in doubles
-  // the full-circle node of slot e is the same for every r' node: one load per unit
+  // the full-circle node of slot e is the same for every r' node: one load per call
   const double2 trf = __ldg(trig_full + (e < N ? e : 0));
 #pragma unroll 1
-  for (int t = 0; t < kChunk; ++t) {
-    const int n = kChunk * ch + t;
+  for (int n = n0; n < n1; ++n) {
     if (e >= S.cnt[n]) continue;
     const int na = S.na[n];
     const NodeRec& nd = S.node[n];  // read at the point of use (register pressure)
@@ -557,6 +557,8 @@ __global__ void __launch_bounds__(32 * kWarps) k_integrate(
     const Item& it = S.it;
 
     double s_phi = 0.0, s_ax = 0.0, s_ay = 0.0, s_err = 0.0;
+    double st[3][9][3];                      // per-lane stencil cache (valid for this item's levels)
+    int cix = -1000000, ciy = -1000000;
     int nseg = 0, nleaf = 0, capped = 0, ties = 0, maxlev = 0;
     unsigned evals = 0;
     int lev = P.n_root == 2 ? 1 : 0;
@@ -606,10 +608,21 @@ __global__ void __launch_bounds__(32 * kWarps) k_integrate(
 #pragma unroll
       for (int o = 16; o > 0; o >>= 1) emax = max(emax, __shfl_xor_sync(0xffffffffu, emax, o));
       double k0 = 0.0, k1 = 0.0, k2 = 0.0, g0 = 0.0, g1 = 0.0, g2 = 0.0;
-      const int units = emax * kNChunks;
-      for (int u = lane; u < units; u += 32) {
-        const int e = u / kNChunks, ch = u - e * kNChunks;
-        eval_chunk<KIND>(it, P, S, trig_full, e, ch, N, wfull, third, k0, k1, k2, g0, g1, g2);
+      // Lane <-> theta slot: full rounds of 32 slots, each lane running all 15 r' nodes of
+      // its slot with the register stencil cache.  The round order alternates from segment
+      // to segment, so the first round of a segment finds the cell left by the last round of
+      // the previous (radially adjacent) segment.  Leftover slots (65-node arcs) go last as
+      // (slot, node) units.
+      const int rounds = emax >> 5, left = emax - 32 * rounds;
+      for (int rr = 0; rr < rounds; ++rr) {
+        const int r = (nseg & 1) ? rounds - 1 - rr : rr;
+        eval_nodes<KIND>(it, P, S, trig_full, 32 * r + lane, 0, 15, N, wfull, third, st, cix, ciy,
+                         k0, k1, k2, g0, g1, g2);
+      }
+      for (int u = lane; u < 15 * left; u += 32) {
+        const int e = 32 * rounds + u / 15, n = u - 15 * (u / 15);
+        eval_nodes<KIND>(it, P, S, trig_full, e, n, n + 1, N, wfull, third, st, cix, ciy, k0, k1,
+                         k2, g0, g1, g2);
       }
       k0 = warp_sum(k0); k1 = warp_sum(k1); k2 = warp_sum(k2);
       g0 = warp_sum(g0); g1 = warp_sum(g1); g2 = warp_sum(g2);
