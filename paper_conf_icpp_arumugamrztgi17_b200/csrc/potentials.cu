@@ -438,7 +438,7 @@ __device__ __forceinline__ void ldg_node(const double* p, double& a, double& b, 
 // Theta slot e of the r' nodes n0 .. n1-1 of the current segment.  The 27-node x 3-component
 // stencil cache (st, cix, ciy) belongs to the caller, so it survives across calls: a lane that
 // evaluates the same slot in consecutive (radially adjacent) deep segments keeps its cell.
-template <int KIND>
+template <int KIND, bool CACHE = true>
 __device__ __forceinline__ void eval_nodes(const Item& it, const Params& P, const WarpSmem& S,
                                            const double2* __restrict__ trig_full, int e, int n0,
                                            int n1, int N, double wfull, double third,
@@ -481,6 +481,8 @@ __device__ __forceinline__ void eval_nodes(const Item& it, const Params& P, cons
       // clamp keeps every stencil inside the zero border (memory guard only)
       const int ix = min(max(__double2int_rz(fx), -2), P.nx + 1);
       const int iy = min(max(__double2int_rz(fy), -2), P.ny + 1);
+      double s[3][3];
+      if (CACHE) {
       if (ix != cix || iy != ciy) {
         cix = ix;
         ciy = iy;
@@ -496,7 +498,6 @@ __device__ __forceinline__ void eval_nodes(const Item& it, const Params& P, cons
               ldg_node(row + 4 * a, st[l][3 * b + a][0], st[l][3 * b + a][1], st[l][3 * b + a][2]);
           }
       }
-      double s[3][3];
 #pragma unroll
       for (int l = 0; l < 3; ++l) {
         s[l][0] = s[l][1] = s[l][2] = 0.0;
@@ -508,6 +509,28 @@ __device__ __forceinline__ void eval_nodes(const Item& it, const Params& P, cons
             s[l][0] += ww * st[l][3 * b + a][0];
             s[l][1] += ww * st[l][3 * b + a][1];
             s[l][2] += ww * st[l][3 * b + a][2];
+          }
+      }
+      } else {
+        // leftover slots: stream the stencil node by node (no cache; the lane's cache is
+        // kept for the next segment)
+        const size_t base = (size_t)4 * ((iy - 1) * P.PX + (ix - 1));
+        const double* g[3] = {it.g0 + base, it.g1 + base, it.g2 + base};
+#pragma unroll
+        for (int l = 0; l < 3; ++l) s[l][0] = s[l][1] = s[l][2] = 0.0;
+#pragma unroll
+        for (int b = 0; b < 3; ++b)
+#pragma unroll
+          for (int a = 0; a < 3; ++a) {
+            const double ww = wx[a] * wy[b];
+#pragma unroll
+            for (int l = 0; l < 3; ++l) {
+              double m0, m1, m2;
+              ldg_node(g[l] + b * rs + 4 * a, m0, m1, m2);
+              s[l][0] = fma(ww, m0, s[l][0]);
+              s[l][1] = fma(ww, m1, s[l][1]);
+              s[l][2] = fma(ww, m2, s[l][2]);
+            }
           }
       }
       f0 = nd.w0 * s[0][0] + nd.w1 * s[1][0] + nd.w2 * s[2][0];
@@ -621,8 +644,8 @@ __global__ void __launch_bounds__(32 * kWarps) k_integrate(
       }
       for (int u = lane; u < 15 * left; u += 32) {
         const int e = 32 * rounds + u / 15, n = u - 15 * (u / 15);
-        eval_nodes<KIND>(it, P, S, trig_full, e, n, n + 1, N, wfull, third, st, cix, ciy, k0, k1,
-                         k2, g0, g1, g2);
+        eval_nodes<KIND, false>(it, P, S, trig_full, e, n, n + 1, N, wfull, third, st, cix, ciy,
+                                k0, k1, k2, g0, g1, g2);
       }
       k0 = warp_sum(k0); k1 = warp_sum(k1); k2 = warp_sum(k2);
       g0 = warp_sum(g0); g1 = warp_sum(g1); g2 = warp_sum(g2);
