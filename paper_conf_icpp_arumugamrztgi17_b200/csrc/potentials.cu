@@ -498,18 +498,22 @@ __device__ __forceinline__ void eval_nodes(const Item& it, const Params& P, cons
               ldg_node(row + 4 * a, st[l][3 * b + a][0], st[l][3 * b + a][1], st[l][3 * b + a][2]);
           }
       }
+      // 9 independent chains (level x component) advanced node by node: covers the DFMA
+      // latency at 2 warps per scheduler
+      {
+        const double w00 = wx[0] * wy[0];
 #pragma unroll
-      for (int l = 0; l < 3; ++l) {
-        s[l][0] = s[l][1] = s[l][2] = 0.0;
+        for (int l = 0; l < 3; ++l)
 #pragma unroll
-        for (int b = 0; b < 3; ++b)
+          for (int c = 0; c < 3; ++c) s[l][c] = w00 * st[l][0][c];
 #pragma unroll
-          for (int a = 0; a < 3; ++a) {
-            const double ww = wx[a] * wy[b];
-            s[l][0] += ww * st[l][3 * b + a][0];
-            s[l][1] += ww * st[l][3 * b + a][1];
-            s[l][2] += ww * st[l][3 * b + a][2];
-          }
+        for (int i = 1; i < 9; ++i) {
+          const double ww = wx[i % 3] * wy[i / 3];
+#pragma unroll
+          for (int l = 0; l < 3; ++l)
+#pragma unroll
+            for (int c = 0; c < 3; ++c) s[l][c] = fma(ww, st[l][i][c], s[l][c]);
+        }
       }
       } else {
         // leftover slots: stream the stencil node by node (no cache; the lane's cache is
