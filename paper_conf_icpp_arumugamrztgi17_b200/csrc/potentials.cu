@@ -476,8 +476,9 @@ __device__ __forceinline__ void eval_nodes(const Item& it, const Params& P, cons
       const double fx = floor(tx + 0.5), fy = floor(ty + 0.5);
       const double dx = tx - fx, dy = ty - fy;
       const double ax = 0.5 - dx, bx = 0.5 + dx, ay = 0.5 - dy, by = 0.5 + dy;
-      const double wx[3] = {0.5 * ax * ax, 0.75 - dx * dx, 0.5 * bx * bx};
-      const double wy[3] = {0.5 * ay * ay, 0.75 - dy * dy, 0.5 * by * by};
+      // 2 x TSC weights (the factor 1/4 of the products is folded into the node weight)
+      const double wx[3] = {ax * ax, fma(-2.0 * dx, dx, 1.5), bx * bx};
+      const double wy[3] = {ay * ay, fma(-2.0 * dy, dy, 1.5), by * by};
       // clamp keeps every stencil inside the zero border (memory guard only)
       const int ix = min(max(__double2int_rz(fx), -2), P.nx + 1);
       const int iy = min(max(__double2int_rz(fy), -2), P.ny + 1);
@@ -543,9 +544,13 @@ __device__ __forceinline__ void eval_nodes(const Item& it, const Params& P, cons
     } else {
       integrand<KIND>(it, P, u, v, nd.w0, nd.w1, nd.w2, f0, f1, f2);
     }
-    const double wk = w * nd.wk, wg = w * nd.wg;
+    const double ws = KIND == RP_SRC_GRID ? 0.25 * w : w;  // undo the 2 x 2 weight scaling
+    const double wk = ws * nd.wk;
     k0 += wk * f0; k1 += wk * f1; k2 += wk * f2;
-    g0 += wg * f0; g1 += wg * f1; g2 += wg * f2;
+    if (n & 1) {  // Gauss nodes only (warp-uniform: all lanes walk the same n)
+      const double wg = ws * nd.wg;
+      g0 += wg * f0; g1 += wg * f1; g2 += wg * f2;
+    }
   }
 }
 
