@@ -143,14 +143,18 @@ def run_ours(args):
 
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
-    local = int(os.environ.get("LOCAL_RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0")) % max(1, __import__("torch").cuda.device_count())
     if args.gpus != world:
         if world == 1 and args.gpus > 1:
             raise SystemExit("--gpus N > 1 must be launched with torchrun (one rank per GPU)")
-    torch.cuda.set_device(local)
+    torch.cuda.set_device(local % max(1, torch.cuda.device_count()))
     group = None
     if world > 1:
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        backend = os.environ.get("RP_DIST_BACKEND", "nccl")  # gloo: 2 ranks on 1 GPU (tests)
+        if backend == "nccl":
+            dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        else:
+            dist.init_process_group(backend)
         group = dist.group.WORLD
     cfg = W.config(args.config)
     sim = Simulation(cfg, group=group)
@@ -214,8 +218,8 @@ def run_ours(args):
     # ---- end-to-end through the C ABI with host buffers (pinned), every step:
     # H2D of the particles, the whole step, D2H of the pushed particles + six mesh outputs.
     e2e = None
-    if world == 1 and not args.no_e2e:
-        e2e = run_e2e(cfg, args, dev)
+    if not args.no_e2e:
+        e2e = run_e2e(cfg, args, dev) if world == 1 else run_e2e_dist(cfg, args, dev, group)
 
     peaks = measured_peaks()
     if rank == 0:
@@ -263,6 +267,48 @@ def run_ours(args):
     if world > 1:
         dist.barrier()
         dist.destroy_process_group()
+
+
+def run_e2e_dist(cfg, args, dev, group):
+    """N > 1: each rank copies its particle shard from pinned host memory, runs the sharded
+    step, and copies the full-mesh potentials and fields (and its pushed shard) back.  Time is
+    the max over ranks of the CUDA-event time on the step's stream."""
+    import torch
+    import torch.distributed as dist
+
+    from paper_conf_icpp_arumugamrztgi17_b200.sim import Simulation
+    sim = Simulation(cfg, group=group)
+    host = [t.detach().cpu().pin_memory() for t in (sim.x, sim.y, sim.ux, sim.uy)]
+    npts = cfg.nx * cfg.ny
+    mesh = torch.zeros((6, npts), dtype=torch.float64).pin_memory()
+    stream = torch.cuda.current_stream()
+    for _ in range(args.warmup):
+        sim.step()
+    dist.barrier()
+    torch.cuda.synchronize()
+    ms = 0.0
+    for _ in range(args.steps):
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record(stream)
+        for d, h in zip((sim.x, sim.y, sim.ux, sim.uy), host):
+            d.copy_(h, non_blocking=True)
+        sim.step()
+        for i, t in enumerate((sim.phi, sim.ax, sim.ay, sim.ex, sim.ey, sim.bz)):
+            mesh[i].copy_(t, non_blocking=True)
+        for d, h in zip((sim.x, sim.y, sim.ux, sim.uy), host):
+            h.copy_(d, non_blocking=True)
+        e1.record(stream)
+        e1.synchronize()
+        ms += e0.elapsed_time(e1)
+    t = torch.tensor([ms], dtype=torch.float64, device=dev)
+    dist.all_reduce(t, op=dist.ReduceOp.MAX)
+    ms = float(t.item())
+    sim.close()
+    pbytes = 4 * sim.x.numel() * 8
+    return {"value": npts * args.steps / (ms * 1e-3), "unit": "mesh-point potentials/s",
+            "h2d_bytes_per_step": pbytes, "d2h_bytes_per_step": pbytes + 6 * npts * 8,
+            "ms_per_step": ms / args.steps, "bytes_per": "rank 0 (particle shard)",
+            "api": "sim.Simulation.step with pinned host copies (torch) around the C-ABI calls"}
 
 
 def run_e2e(cfg, args, dev):
