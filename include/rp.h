@@ -102,21 +102,25 @@ int rp_set_stream(rp_ctx* ctx, void* stream);
 int rp_history_init(rp_ctx* ctx, int32_t n_pre, const rp_frame* frames_host,
                     const double* grids_dev, int32_t rigid);
 
+/* Bytes of one partial-deposit buffer (16-byte aligned device memory). */
+int64_t rp_partial_bytes(const rp_ctx* ctx);
+
 /* Partial deposition of n local particles (SoA x, y, u_x, u_y with u = gamma*beta) of
- * charge q each on frame_k (TSC, R-14): writes partial_dev [ny][nx][4] =
- * (rho, rho*beta_x, rho*beta_y, 0), overwritten.  Bins are computed without FMA so
- * they are bit-identical to the oracle (R-13).  Atomics-free: particles are radix-sorted
- * by bin and every node sums its 9 neighbour bins in a fixed order.
- * info (nullable) syncs the stream. */
+ * charge q each on frame_k (TSC, R-14) into partial_dev, an opaque buffer of
+ * rp_partial_bytes() bytes holding the EXACT sums of (rho, rho*beta_x, rho*beta_y) per node:
+ * each particle contribution is rounded once to 128-bit fixed point (quantum 2^-s with
+ * 2^s ~ 2^85 (hx hy)/|q|), so sums do not depend on order or grouping.  Bins are computed
+ * without FMA so they are bit-identical to the oracle (R-13).  Atomics-free: particles are
+ * radix-sorted by bin and every node sums its 9 neighbour bins.  info (nullable) syncs. */
 int rp_deposit(rp_ctx* ctx, const double* x, const double* y, const double* ux,
                const double* uy, double q, int64_t n, const rp_frame* frame_k,
-               double* partial_dev, rp_deposit_info* info);
+               void* partial_dev, rp_deposit_info* info);
 
-/* Advance to the next step k (0 at the first call) and store
- * D_k = sum_{i < n_parts} partials_dev[i] (summed in index order = rank order) into ring
- * slot k mod H with frame_k ("stored linearly on the device memory").
- * partials_dev is [n_parts][ny][nx][4]. */
-int rp_history_append(rp_ctx* ctx, const double* partials_dev, int32_t n_parts,
+/* Advance to the next step k (0 at the first call) and store D_k = the exact sum of
+ * n_parts consecutive partial buffers (e.g. all-gathered from the ranks), rounded once to
+ * FP64, into ring slot k mod H with frame_k ("stored linearly on the device memory").
+ * D_k is bit-identical for any split of the particles over ranks. */
+int rp_history_append(rp_ctx* ctx, const void* partials_dev, int32_t n_parts,
                       const rp_frame* frame_k);
 
 /* rp_deposit into context scratch + rp_history_append(n_parts = 1). */

@@ -4,8 +4,12 @@
 //   CUB sort     stable radix sort of (bin, particle id)
 //   k_bin_start  per-bin start offsets (binary search in the sorted keys)
 //   k_gather     particle records into sorted order (coalesced reads below)
-//   k_node_sum   one warp per node: fixed-order sum over its 9 neighbour bins -> M_k
-//   k_append     D_k = sum of per-rank partials in rank order -> ring slot k mod H
+//   k_node_sum   one warp per node: sum over its 9 neighbour bins -> exact partial M_k
+//   k_append     D_k = exact sum of the per-rank partials -> ring slot k mod H
+// Partial sums are exact: every particle contribution is rounded once to a 128-bit fixed-point
+// number (quantum 2^-shift, shift from |q|/(hx hy) so 2^40 particles cannot overflow) and the
+// integer sums are order-independent, so D_k is bit-identical however the particles are split
+// over ranks, lanes or warps.  The one rounding to FP64 happens in k_append.
 #include <cub/device/device_radix_sort.cuh>
 
 #include "rp_internal.cuh"
@@ -58,16 +62,28 @@ __device__ __forceinline__ void tsc(double d, double& wm, double& w0, double& wp
   wp = 0.5 * (b * b);
 }
 
+__device__ __forceinline__ __int128 to_fixed(double v, int shift) {
+  return (__int128)rint(ldexp(v, shift));
+}
+
+__device__ __forceinline__ __int128 shfl_xor_i128(__int128 v, int o) {
+  unsigned long long lo = (unsigned long long)v, hi = (unsigned long long)(v >> 64);
+  lo = __shfl_xor_sync(0xffffffffu, lo, o);
+  hi = __shfl_xor_sync(0xffffffffu, hi, o);
+  return (__int128)(((unsigned __int128)hi << 64) | lo);
+}
+
 // One warp per grid node.  Node (ix, iy) receives from the particles of bin
 // (ix - oa, iy - ob), oa, ob in {-1, 0, 1}, the weight w_oa(dx) w_ob(dy) (TSC).
+// out: [nx*ny][3] 128-bit fixed-point sums (rho, rho*bx, rho*by) x 2^shift.
 __global__ void k_node_sum(int nx, int ny, const int32_t* __restrict__ start,
-                           const double4* __restrict__ rec, double scale,
-                           double* __restrict__ M) {
+                           const double4* __restrict__ rec, double scale, int shift,
+                           __int128* __restrict__ out) {
   int warp = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
   int lane = threadIdx.x & 31;
   if (warp >= nx * ny) return;
   int ix = warp % nx, iy = warp / nx;
-  double s0 = 0.0, s1 = 0.0, s2 = 0.0;
+  __int128 s0 = 0, s1 = 0, s2 = 0;
   for (int ob = -1; ob <= 1; ++ob) {
     int by = iy - ob;
     if (by < 1 || by > ny - 2) continue;
@@ -83,46 +99,53 @@ __global__ void k_node_sum(int nx, int ny, const int32_t* __restrict__ start,
         tsc(r.y, vm, v0, vp);
         double wx = oa < 0 ? wm : (oa == 0 ? w0 : wp);
         double wy = ob < 0 ? vm : (ob == 0 ? v0 : vp);
-        double w = wx * wy;
-        s0 += w;
-        s1 += w * r.z;
-        s2 += w * r.w;
+        double w = scale * (wx * wy);  // q w_a w_b / (hx hy), one rounding per particle
+        s0 += to_fixed(w, shift);
+        s1 += to_fixed(w * r.z, shift);
+        s2 += to_fixed(w * r.w, shift);
       }
     }
   }
   for (int o = 16; o > 0; o >>= 1) {
-    s0 += __shfl_xor_sync(0xffffffffu, s0, o);
-    s1 += __shfl_xor_sync(0xffffffffu, s1, o);
-    s2 += __shfl_xor_sync(0xffffffffu, s2, o);
+    s0 += shfl_xor_i128(s0, o);
+    s1 += shfl_xor_i128(s1, o);
+    s2 += shfl_xor_i128(s2, o);
   }
   if (lane == 0) {
-    double* m = M + 4 * (size_t)warp;
-    m[0] = scale * s0;
-    m[1] = scale * s1;
-    m[2] = scale * s2;
-    m[3] = 0.0;
+    __int128* m = out + 3 * (size_t)warp;
+    m[0] = s0;
+    m[1] = s1;
+    m[2] = s2;
   }
 }
 
-// ring slot (padded) <- sum of n_parts unpadded partial grids, in part order
-__global__ void k_append(int nx, int ny, int PX, const double* __restrict__ parts,
-                         int n_parts, double* __restrict__ slot) {
+// ring slot (padded) <- exact sum of n_parts partial buffers (header + [npts][3] int128)
+__global__ void k_append(int nx, int ny, int PX, const unsigned char* __restrict__ parts,
+                         size_t part_bytes, int n_parts, double* __restrict__ slot) {
   int id = blockIdx.x * blockDim.x + threadIdx.x;
   if (id >= nx * ny) return;
   int ix = id % nx, iy = id / nx;
-  size_t np = (size_t)nx * ny * 4;
-  double a = 0.0, b = 0.0, c = 0.0;
+  __int128 a = 0, b = 0, c = 0;
+  const int shift = (int)reinterpret_cast<const long long*>(parts)[0];
   for (int i = 0; i < n_parts; ++i) {
-    const double* m = parts + i * np + 4 * (size_t)id;
-    a += m[0];
-    b += m[1];
-    c += m[2];
+    const unsigned char* base = parts + i * part_bytes;
+    const int sh = (int)reinterpret_cast<const long long*>(base)[0];
+    const __int128* m = reinterpret_cast<const __int128*>(base + 16) + 3 * (size_t)id;
+    const int d = sh - shift;  // equal shifts in practice (same q on every rank)
+    a += d >= 0 ? (m[0] >> d) : (m[0] << -d);
+    b += d >= 0 ? (m[1] >> d) : (m[1] << -d);
+    c += d >= 0 ? (m[2] >> d) : (m[2] << -d);
   }
-  double* d = slot + 4 * ((size_t)(iy + RP_PAD) * PX + (ix + RP_PAD));
-  d[0] = a;
-  d[1] = b;
-  d[2] = c;
-  d[3] = 0.0;
+  double* dst = slot + 4 * ((size_t)(iy + RP_PAD) * PX + (ix + RP_PAD));
+  dst[0] = ldexp((double)a, -shift);
+  dst[1] = ldexp((double)b, -shift);
+  dst[2] = ldexp((double)c, -shift);
+  dst[3] = 0.0;
+}
+
+__global__ void k_set_header(long long* hdr, long long shift) {
+  hdr[0] = shift;
+  hdr[1] = 0;
 }
 
 int grow_deposit(rp_ctx* ctx, int64_t n) {
@@ -156,9 +179,20 @@ int rp_ensure_cub_tmp(rp_ctx* ctx, size_t bytes) {
   return RP_OK;
 }
 
+int64_t rp_partial_bytes_impl(const rp_ctx* ctx) {
+  return 16 + (int64_t)ctx->cfg.nx * ctx->cfg.ny * 3 * 16;
+}
+
+// quantum of the exact partial sums: |sum| <= |q| N / (hx hy) < 2^126 for N <= 2^40
+static int fixed_shift(double q, double hx, double hy) {
+  double a = fabs(q) / (hx * hy);
+  if (!(a > 0.0) || !isfinite(a)) return 64;
+  return 126 - 40 - 1 - (int)ceil(log2(a));
+}
+
 int rp_deposit_impl(rp_ctx* ctx, const double* x, const double* y, const double* ux,
                     const double* uy, double q, int64_t n, const rp_frame* fk,
-                    double* partial, rp_deposit_info* info) {
+                    void* partial, rp_deposit_info* info) {
   const rp_config& c = ctx->cfg;
   if (n < 0 || n > 0x7fffffffLL || !fk || !partial) return rp_fail(ctx, RP_EINVAL, "deposit: bad args");
   if (n > 0 && (!x || !y || !ux || !uy)) return rp_fail(ctx, RP_EINVAL, "deposit: null particle array");
@@ -191,9 +225,13 @@ int rp_deposit_impl(rp_ctx* ctx, const double* x, const double* y, const double*
     RP_CUDA(cudaMemsetAsync(ctx->bin_start, 0, (nbins + 1) * sizeof(int32_t), st));
   }
   double scale = q / (c.hx * c.hy);
+  const int shift = fixed_shift(q, c.hx, c.hy);
+  k_set_header<<<1, 1, 0, st>>>(reinterpret_cast<long long*>(partial), shift);
+  RP_CHECK_LAUNCH();
   int warps_per_block = 8;
   k_node_sum<<<(nbins + warps_per_block - 1) / warps_per_block, 32 * warps_per_block, 0, st>>>(
-      c.nx, c.ny, ctx->bin_start, ctx->rec_sorted, scale, partial);
+      c.nx, c.ny, ctx->bin_start, ctx->rec_sorted, scale, shift,
+      reinterpret_cast<__int128*>(reinterpret_cast<unsigned char*>(partial) + 16));
   RP_CHECK_LAUNCH();
   if (info) {
     int32_t kept = 0;
@@ -207,7 +245,7 @@ int rp_deposit_impl(rp_ctx* ctx, const double* x, const double* y, const double*
   return RP_OK;
 }
 
-int rp_append_impl(rp_ctx* ctx, const double* parts, int32_t n_parts, const rp_frame* fk) {
+int rp_append_impl(rp_ctx* ctx, const void* parts, int32_t n_parts, const rp_frame* fk) {
   const rp_config& c = ctx->cfg;
   if (!parts || n_parts < 1 || !fk) return rp_fail(ctx, RP_EINVAL, "append: bad args");
   cudaStream_t st = ctx->stream;
@@ -216,7 +254,9 @@ int rp_append_impl(rp_ctx* ctx, const double* parts, int32_t n_parts, const rp_f
   double* slot = ctx->ring + (size_t)s * ctx->slot_doubles;
   int npts = c.nx * c.ny;
   ProfScope ps(ctx, PK_APPEND);
-  k_append<<<(npts + 255) / 256, 256, 0, st>>>(c.nx, c.ny, ctx->PX, parts, n_parts, slot);
+  k_append<<<(npts + 255) / 256, 256, 0, st>>>(c.nx, c.ny, ctx->PX,
+                                                reinterpret_cast<const unsigned char*>(parts),
+                                                (size_t)rp_partial_bytes_impl(ctx), n_parts, slot);
   RP_CHECK_LAUNCH();
   ctx->fh[s] = *fk;
   RP_CUDA(cudaMemcpyAsync(ctx->frames_dev + s, fk, sizeof(rp_frame), cudaMemcpyHostToDevice, st));

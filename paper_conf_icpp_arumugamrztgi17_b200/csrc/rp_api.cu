@@ -165,7 +165,7 @@ int rp_create(const rp_config* cfg, rp_ctx** out) {
     return fail(RP_ECUDA);
   size_t npts = (size_t)cfg->nx * cfg->ny;
   if (cudaMalloc(&ctx->bin_start, (npts + 2) * sizeof(int32_t)) != cudaSuccess) return fail(RP_ENOMEM);
-  if (cudaMalloc(&ctx->partial, npts * 4 * sizeof(double)) != cudaSuccess) return fail(RP_ENOMEM);
+  if (cudaMalloc(&ctx->partial, rp_partial_bytes_impl(ctx)) != cudaSuccess) return fail(RP_ENOMEM);
   int rc = rp_alloc_potential_scratch(ctx);
   if (rc) return fail(rc);
   // analytic amplitudes default to 1
@@ -221,13 +221,15 @@ int rp_history_init(rp_ctx* ctx, int32_t n_pre, const rp_frame* frames_host,
 }
 
 int rp_deposit(rp_ctx* ctx, const double* x, const double* y, const double* ux, const double* uy,
-               double q, int64_t n, const rp_frame* frame_k, double* partial_dev,
+               double q, int64_t n, const rp_frame* frame_k, void* partial_dev,
                rp_deposit_info* info) {
   if (!ctx) return RP_EINVAL;
   return rp_deposit_impl(ctx, x, y, ux, uy, q, n, frame_k, partial_dev, info);
 }
 
-int rp_history_append(rp_ctx* ctx, const double* partials_dev, int32_t n_parts,
+int64_t rp_partial_bytes(const rp_ctx* ctx) { return ctx ? rp_partial_bytes_impl(ctx) : 0; }
+
+int rp_history_append(rp_ctx* ctx, const void* partials_dev, int32_t n_parts,
                       const rp_frame* frame_k) {
   if (!ctx) return RP_EINVAL;
   return rp_append_impl(ctx, partials_dev, n_parts, frame_k);

@@ -41,7 +41,7 @@ struct rp_ctx {
   double4* rec_sorted = nullptr;
   int32_t* bin_start = nullptr; // [nx*ny + 1]
   int64_t last_n = 0;
-  double* partial = nullptr;    // [ny][nx][4] scratch for rp_deposit_step
+  void* partial = nullptr;      // exact partial buffer (rp_partial_bytes) for rp_deposit_step
   void* cub_tmp = nullptr;
   size_t cub_tmp_bytes = 0;
 
@@ -160,8 +160,9 @@ static inline int kappa_of(const rp_ctx* ctx) {
 // internal entry points implemented in the .cu files
 int rp_deposit_impl(rp_ctx* ctx, const double* x, const double* y, const double* ux,
                     const double* uy, double q, int64_t n, const rp_frame* frame_k,
-                    double* partial_dev, rp_deposit_info* info);
-int rp_append_impl(rp_ctx* ctx, const double* partials, int32_t n_parts, const rp_frame* fk);
+                    void* partial_dev, rp_deposit_info* info);
+int rp_append_impl(rp_ctx* ctx, const void* partials, int32_t n_parts, const rp_frame* fk);
+int64_t rp_partial_bytes_impl(const rp_ctx* ctx);
 int rp_potentials_impl(rp_ctx* ctx, int src_kind, const double src[6], int32_t rank,
                        int32_t world, double* phi, double* ax, double* ay, double* err,
                        int32_t* nseg, double* shard_out, int64_t cap, int64_t* n_out,

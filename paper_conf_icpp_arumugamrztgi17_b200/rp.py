@@ -83,6 +83,7 @@ _SIG = {
     "rp_deposit": (C.c_int, [_vp, _vp, _vp, _vp, _vp, _d, _i64, _P(rp_frame), _vp,
                              _P(rp_deposit_info)]),
     "rp_history_append": (C.c_int, [_vp, _vp, _i32, _P(rp_frame)]),
+    "rp_partial_bytes": (_i64, [_vp]),
     "rp_deposit_step": (C.c_int, [_vp, _vp, _vp, _vp, _vp, _d, _i64, _P(rp_frame),
                                   _P(rp_deposit_info)]),
     "rp_compute_potentials": (C.c_int, [_vp, _vp, _vp, _vp, _vp, _vp, _P(rp_potential_info)]),
@@ -218,16 +219,25 @@ def rp_history_init(ctx, n_pre, frames, grids=None, rigid=True) -> None:
            "rp_history_init")
 
 
+def rp_partial_bytes(ctx) -> int:
+    return _lib.rp_partial_bytes(ctx)
+
+
 def rp_deposit(ctx, x, y, ux, uy, q, frame_k, partial, info=False):
+    """partial: uint8 CUDA tensor of rp_partial_bytes(ctx) bytes (opaque exact sums)."""
     inf = rp_deposit_info() if info else None
+    if partial.numel() * partial.element_size() < rp_partial_bytes(ctx):
+        raise ValueError("partial: smaller than rp_partial_bytes(ctx)")
     _check(_lib.rp_deposit(ctx, _f64(x, "x"), _f64(y, "y"), _f64(ux, "ux"), _f64(uy, "uy"),
-                           float(q), x.numel(), C.byref(frame(frame_k)), _f64(partial, "partial"),
+                           float(q), x.numel(), C.byref(frame(frame_k)), _dev(partial, None, "partial"),
                            C.byref(inf) if inf is not None else None), ctx, "rp_deposit")
     return inf
 
 
 def rp_history_append(ctx, partials, n_parts, frame_k) -> None:
-    _check(_lib.rp_history_append(ctx, _f64(partials, "partials"), n_parts, C.byref(frame(frame_k))),
+    """partials: n_parts consecutive partial buffers (uint8 CUDA tensor)."""
+    _check(_lib.rp_history_append(ctx, _dev(partials, None, "partials"), n_parts,
+                                  C.byref(frame(frame_k))),
            ctx, "rp_history_append")
 
 

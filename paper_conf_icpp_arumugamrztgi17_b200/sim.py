@@ -55,8 +55,9 @@ class Simulation:
         self.nseg = torch.zeros(npts, dtype=torch.int32, device=self.device)
         self.k = 0
         if self.world > 1:
-            self.partial = torch.zeros((cfg.ny, cfg.nx, 4), **f64)
-            self.partials = torch.zeros((self.world, cfg.ny, cfg.nx, 4), **f64)
+            pb = ops.rp_partial_bytes(self.ctx)  # opaque exact partial sums
+            self.partial = torch.zeros(pb, dtype=torch.uint8, device=self.device)
+            self.partials = torch.zeros(self.world * pb, dtype=torch.uint8, device=self.device)
             cap = ops.rp_shard_capacity(self.ctx, self.world)
             self.shard = torch.zeros((cap, 6), **f64)
             self.shards = torch.zeros((self.world, cap, 6), **f64)

@@ -53,15 +53,19 @@ class OracleOps:
             ctx.frames[(-n_pre + i) % ctx.H] = f
         ctx.n_pre, ctx.rigid = n_pre, rigid
 
+    def rp_partial_bytes(self, ctx):
+        return ctx.ny * ctx.nx * 4 * 8  # the stand-in keeps FP64 partials
+
     def rp_deposit(self, ctx, x, y, ux, uy, q, fk, partial, info=False):
         M, _, _ = oracle.deposit(x.numpy(), y.numpy(), ux.numpy(), uy.numpy(), q, fk, ctx.nx, ctx.ny,
                                  ctx.hx, ctx.hy)
-        partial.copy_(torch.from_numpy(M))
+        partial.view(torch.float64).copy_(torch.from_numpy(M).view(-1))
 
     def rp_history_append(self, ctx, partials, n_parts, fk):
         tot = np.zeros((ctx.ny, ctx.nx, 4))
+        parts = partials.view(torch.float64).view(n_parts, ctx.ny, ctx.nx, 4)
         for i in range(n_parts):  # rank order
-            tot = tot + partials[i].numpy()
+            tot = tot + parts[i].numpy()
         ctx.k += 1
         ctx.ring[ctx.k % ctx.H] = tot
         ctx.frames[ctx.k % ctx.H] = fk
@@ -70,8 +74,8 @@ class OracleOps:
                 ctx.ring[l % ctx.H] = tot
 
     def rp_deposit_step(self, ctx, x, y, ux, uy, q, fk, info=False):
-        part = torch.zeros((1, ctx.ny, ctx.nx, 4), dtype=torch.float64)
-        self.rp_deposit(ctx, x, y, ux, uy, q, fk, part[0])
+        part = torch.zeros(self.rp_partial_bytes(ctx), dtype=torch.uint8)
+        self.rp_deposit(ctx, x, y, ux, uy, q, fk, part)
         self.rp_history_append(ctx, part, 1, fk)
 
     def _problem(self, ctx):

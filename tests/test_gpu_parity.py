@@ -29,6 +29,18 @@ def _dev_arrays(torch, *arrs):
 
 
 # ------------------------------------------------------------------ deposition
+def _partial(torch, ctx, n=1):
+    from paper_conf_icpp_arumugamrztgi17_b200 import rp
+    return torch.zeros(n * rp.rp_partial_bytes(ctx), dtype=torch.uint8, device="cuda")
+
+
+def _slot_moments(torch, ctx, cfg, slot):
+    from paper_conf_icpp_arumugamrztgi17_b200 import rp
+    ring = torch.zeros((cfg.H, cfg.ny, cfg.nx, 4), dtype=torch.float64, device="cuda")
+    rp.rp_save_state(ctx, ring)
+    return ring[slot].cpu().numpy()
+
+
 @pytest.mark.parametrize("cfgno", [1, 2])
 def test_deposit_bins_bit_exact_and_moments(torch, cfgno):
     from paper_conf_icpp_arumugamrztgi17_b200 import rp
@@ -41,13 +53,14 @@ def test_deposit_bins_bit_exact_and_moments(torch, cfgno):
     ctx = G.make_ctx(cfg)
     try:
         xd, yd, uxd, uyd = _dev_arrays(torch, x, y, ux, uy)
-        part = torch.zeros((cfg.ny, cfg.nx, 4), dtype=torch.float64, device="cuda")
+        part = _partial(torch, ctx)
         info = rp.rp_deposit(ctx, xd, yd, uxd, uyd, cfg.q_particle, W.frame(cfg, 0), part, info=True)
         b = torch.zeros(len(x), dtype=torch.int32, device="cuda")
         rp.rp_debug_bins(ctx, b)
         torch.cuda.synchronize()
         np.testing.assert_array_equal(b.cpu().numpy(), bins)
-        Mg = part.cpu().numpy()
+        rp.rp_history_append(ctx, part, 1, W.frame(cfg, 0))
+        Mg = _slot_moments(torch, ctx, cfg, 0)
         scale = np.abs(M).max()
         assert np.abs(Mg - M).max() <= 1e-12 * scale
         assert info.n_lost == int((bins < 0).sum())
@@ -56,6 +69,35 @@ def test_deposit_bins_bit_exact_and_moments(torch, cfgno):
         assert abs(tot - 1.0) < 1e-12
     finally:
         rp.rp_destroy(ctx)
+
+
+def test_deposit_exact_for_any_particle_split(torch):
+    """Exact fixed-point partial sums: depositing the bunch in one piece or
+    split into 3 unequal rank shards and appending the partials gives a bit-identical D_k."""
+    from paper_conf_icpp_arumugamrztgi17_b200 import rp
+    cfg = W.config(2)
+    x, y, ux, uy = W.particles(cfg, n=200_000, seed=11)
+    q = 1.0 / len(x)
+    fk = W.frame(cfg, 0)
+    ctx1, ctx3 = G.make_ctx(cfg), G.make_ctx(cfg)
+    try:
+        d = _dev_arrays(torch, x, y, ux, uy)
+        p1 = _partial(torch, ctx1)
+        rp.rp_deposit(ctx1, *d, q, fk, p1)
+        rp.rp_history_append(ctx1, p1, 1, fk)
+        pb = rp.rp_partial_bytes(ctx3)
+        p3 = _partial(torch, ctx3, 3)
+        cuts = [0, 31_337, 150_001, len(x)]
+        for r in range(3):
+            sl = [t[cuts[r]:cuts[r + 1]].contiguous() for t in d]
+            rp.rp_deposit(ctx3, *sl, q, fk, p3[r * pb:(r + 1) * pb])
+        rp.rp_history_append(ctx3, p3, 3, fk)
+        a, b = _slot_moments(torch, ctx1, cfg, 0), _slot_moments(torch, ctx3, cfg, 0)
+        np.testing.assert_array_equal(a, b)
+        assert np.abs(a).max() > 0
+    finally:
+        rp.rp_destroy(ctx1)
+        rp.rp_destroy(ctx3)
 
 
 def test_deposit_golden_ties(torch):
@@ -68,7 +110,7 @@ def test_deposit_golden_ties(torch):
     ctx = rp.rp_create(g["nx"], g["ny"], g["hx"], g["hy"], 2, 1.0, 1.0, 1e-6)
     try:
         xd, yd, zd, zd2 = _dev_arrays(torch, x, y, z, z)
-        part = torch.zeros((g["ny"], g["nx"], 4), dtype=torch.float64, device="cuda")
+        part = _partial(torch, ctx)
         rp.rp_deposit(ctx, xd, yd, zd, zd2, 1.0, g["frame"], part)
         b = torch.zeros(len(x), dtype=torch.int32, device="cuda")
         rp.rp_debug_bins(ctx, b)
