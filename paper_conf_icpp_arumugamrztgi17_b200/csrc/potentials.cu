@@ -448,7 +448,7 @@ __device__ __forceinline__ void eval_nodes(const Item& it, const Params& P, cons
   const size_t rs = (size_t)4 * P.PX;  // padded row stride in doubles
   // the full-circle node of slot e is the same for every r' node: one load per call
   const double2 trf = __ldg(trig_full + (e < N ? e : 0));
-#pragma unroll 1
+#pragma unroll 3
   for (int n = n0; n < n1; ++n) {
     if (e >= S.cnt[n]) continue;
     const int na = S.na[n];
