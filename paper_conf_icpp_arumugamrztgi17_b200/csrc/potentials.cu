@@ -235,7 +235,10 @@ __global__ void k_clip(Params P, const int32_t* __restrict__ owner, int rank,
         B = lo;
       }
       if (A < B) {
-        unsigned c = cost_prev ? forecast(cost_prev, p, j, P.nx, P.ny, P.kmax, policy, knn) : 0u;
+        // no forecast yet (first step): the near-field subregion S_0 carries most of the work
+        // (DESIGN.md sec. 3), so run it first; later steps use last step's counts
+        unsigned c = cost_prev ? forecast(cost_prev, p, j, P.nx, P.ny, P.kmax, policy, knn)
+                               : (policy == RP_SCHED_INDEX ? 0u : (j == 0 ? 1u : 0u));
         kk = (uint16_t)(0xFFFEu - (c < 0xFFFEu ? c : 0xFFFEu));
       }
     }
