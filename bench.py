@@ -157,6 +157,7 @@ def run_ours(args):
             dist.init_process_group(backend)
         group = dist.group.WORLD
     cfg = W.config(args.config)
+    cfg.rule = 1 if args.rule == "simpson" else 0
     sim = Simulation(cfg, group=group)
     sched = args.schedule
     if sched == "index":
@@ -245,7 +246,7 @@ def run_ours(args):
                        "tau": cfg.tau, "n_theta": cfg.n_theta, "n_root": cfg.n_root,
                        "parallelism": f"mesh-point shards x{world}, history replicated",
                        "l2": "flushed between timed steps (512 MB write)",
-                       "schedule": args.schedule},
+                       "schedule": args.schedule, "outer_rule": args.rule},
             "fp64_gflops": gflops,
             "work_per_step": {k2: v / args.steps for k2, v in totals.items()},
             "roofline": {"kernel": "k_integrate (GK15 tree integrator)", "bound": "alu",
@@ -436,6 +437,8 @@ def main():
     ap.add_argument("--impl", choices=["ours", "reference"], default="ours")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--rule", default="gk15", choices=["gk15", "simpson"],
+                    help="outer segment rule (simpson = the paper's RP-QUADRULE, a variant)")
     ap.add_argument("--schedule", default="persistence",
                     help="work-order forecast: index | persistence | knn5 | knn9 | knn25")
     args = ap.parse_args()

@@ -63,7 +63,12 @@ typedef struct {
   int32_t max_depth;       /* 1..60 bisection cap of the outer tree (R-12)                       */
   int32_t n_root;          /* 2: roots are the two halves of each clipped S_j (R-12b); or 1     */
   int32_t device;          /* CUDA ordinal                                                       */
+  int32_t outer_rule;      /* RP_RULE_GK15 (default, R-8) or RP_RULE_SIMPSON: the paper's own   */
+                           /* rule (P:155 RP-QUADRULE), Boole value + |S2 - S1|/15 estimate (R-22) */
 } rp_config;
+
+#define RP_RULE_GK15 0
+#define RP_RULE_SIMPSON 1
 
 typedef struct {
   int64_t n_lost;          /* particles whose 3x3 stencil leaves the grid (R-14)                 */

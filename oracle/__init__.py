@@ -43,7 +43,7 @@ class Params(C.Structure):
     _fields_ = [("nx", C.c_int32), ("ny", C.c_int32), ("hx", C.c_double), ("hy", C.c_double),
                 ("c", C.c_double), ("dt", C.c_double), ("tau", C.c_double),
                 ("n_theta", C.c_int32), ("max_depth", C.c_int32), ("n_root", C.c_int32),
-                ("kappa_max", C.c_int32)]
+                ("kappa_max", C.c_int32), ("rule", C.c_int32)]
 
 
 class Hist(C.Structure):
@@ -127,9 +127,11 @@ class Problem:
 
     def __init__(self, *, nx, ny, hx, hy, c, dt, tau, kappa_max, k, n_pre,
                  ring=None, frames=None, n_theta=64, max_depth=30, n_root=2,
-                 source=SRC_GRID, x0=0.0, y0=0.0, width=1.0, q=1.0, bx=0.0, by=0.0, amp=None):
+                 source=SRC_GRID, x0=0.0, y0=0.0, width=1.0, q=1.0, bx=0.0, by=0.0, amp=None,
+                 rule=0):
         H = kappa_max + 2
-        self.params = Params(nx, ny, hx, hy, c, dt, tau, n_theta, max_depth, n_root, kappa_max)
+        self.params = Params(nx, ny, hx, hy, c, dt, tau, n_theta, max_depth, n_root, kappa_max,
+                             rule)
         self.ring = None if ring is None else np.ascontiguousarray(ring, dtype=np.float64)
         if self.ring is not None:
             assert self.ring.shape == (H, ny, nx, 4), self.ring.shape
@@ -250,7 +252,7 @@ def arcs_disk(cu, cv, r, x0, y0, a):
 
 
 def fields(nx, ny, hx, hy, c, dt, fk, fkm1, phi, ax, ay, ax_prev=None, ay_prev=None):
-    P = Params(nx, ny, hx, hy, c, dt, 1.0, 64, 30, 2, 1)
+    P = Params(nx, ny, hx, hy, c, dt, 1.0, 64, 30, 2, 1, 0)
     phi, ax, ay = (np.ascontiguousarray(a, dtype=np.float64) for a in (phi, ax, ay))
     if ax_prev is not None:
         ax_prev = np.ascontiguousarray(ax_prev, dtype=np.float64)
@@ -264,7 +266,7 @@ def fields(nx, ny, hx, hy, c, dt, fk, fkm1, phi, ax, ay, ax_prev=None, ay_prev=N
 
 def push(nx, ny, hx, hy, c, dt, fk, x, y, ux, uy, q_over_mc, bz_ext, ex, ey, bz):
     """In-place Boris push on copies; returns (x, y, ux, uy)."""
-    P = Params(nx, ny, hx, hy, c, dt, 1.0, 64, 30, 2, 1)
+    P = Params(nx, ny, hx, hy, c, dt, 1.0, 64, 30, 2, 1, 0)
     x, y, ux, uy = (np.array(a, dtype=np.float64, copy=True) for a in (x, y, ux, uy))
     ex, ey, bz = (np.ascontiguousarray(a, dtype=np.float64) for a in (ex, ey, bz))
     lib().orc_push(C.byref(P), C.byref(frame(fk)), len(x), _pd(x), _pd(y), _pd(ux), _pd(uy),

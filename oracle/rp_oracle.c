@@ -49,6 +49,7 @@ typedef struct {
   int32_t max_depth; /* bisection cap (R-12)                                 */
   int32_t n_root;    /* 2: start from both halves of [A,B]; 1: from [A,B]   */
   int32_t kappa_max; /* history depth (R-4)                                  */
+  int32_t rule;      /* outer segment rule: 0 = GK15 (R-8), 1 = Simpson/Boole (R-22) */
 } orc_params;
 
 typedef struct {
@@ -486,6 +487,39 @@ static void gk15(subctx* X, double a, double b, double* K, double* G, double* er
   }
 }
 
+/* The paper's own outer rule (P:155 RP-QUADRULE "standard Simpson's quadrature rule",
+ * P:157 Simpson adaptive quadrature; reading R-22): on five equispaced nodes
+ * r_0 = a, r_2 = (a+b)/2, r_1 = (r_0+r_2)/2, r_3 = (r_2+r_4)/2, r_4 = b, the composite
+ * Simpson estimate S2 = h/12 (1,4,2,4,1) and the single-panel S1 = h/6 (1,0,4,0,1) give the
+ * standard error estimate |S2 - S1| / 15 and the Richardson value S2 + (S2 - S1)/15, which
+ * is Boole's rule h/90 (7,32,12,32,7).  Returned as K = Boole, G = S2: err = |K - G|. */
+static void simpson5(subctx* X, double a, double b, double* K, double* G, double* err) {
+  double r[5];
+  r[0] = a;
+  r[4] = b;
+  r[2] = 0.5 * (a + b);
+  r[1] = 0.5 * (r[0] + r[2]);
+  r[3] = 0.5 * (r[2] + r[4]);
+  static const double wb[5] = {7.0, 32.0, 12.0, 32.0, 7.0};
+  static const double ws[5] = {1.0, 4.0, 2.0, 4.0, 1.0};
+  double h = b - a;
+  double kb[3] = {0, 0, 0}, ks[3] = {0, 0, 0}, v[3];
+  for (int i = 0; i < 5; ++i) {
+    orc_inner_ctx(X, r[i], v);
+    for (int c = 0; c < 3; ++c) {
+      kb[c] += wb[i] * v[c];
+      ks[c] += ws[i] * v[c];
+    }
+  }
+  *err = 0.0;
+  for (int c = 0; c < 3; ++c) {
+    K[c] = h / 90.0 * kb[c];
+    G[c] = h / 12.0 * ks[c];
+    double e = fabs(K[c] - G[c]);
+    if (e > *err) *err = e;
+  }
+}
+
 /* depth-first, left to right: visit (level, index) on [A,B] */
 static void tree(subctx* X, double A, double B, double R, int32_t lev, int64_t idx,
                  orc_result* res) {
@@ -493,9 +527,12 @@ static void tree(subctx* X, double A, double B, double R, int32_t lev, int64_t i
   double fa = ldexp((double)idx, -lev), fb = ldexp((double)(idx + 1), -lev);
   double a = A + (B - A) * fa, b = A + (B - A) * fb;
   double K[3], G[3], err;
-  gk15(X, a, b, K, G, &err);
+  if (P->rule == 1)
+    simpson5(X, a, b, K, G, &err);
+  else
+    gk15(X, a, b, K, G, &err);
   res->nseg++;
-  res->nodes += 15;
+  res->nodes += P->rule == 1 ? 5 : 15;
   double tol = P->tau * ldexp(B - A, -lev) / R;
   double margin = fabs(err - tol) / tol;
   if (margin < res->min_margin) res->min_margin = margin;

@@ -48,7 +48,7 @@ constexpr int kMaxArcs = 8;
 constexpr int kWarps = 4;  // warps per CTA of k_integrate
 
 struct Params {
-  int nx, ny, PX, npts, kmax, kap, k, H, n_theta, max_depth, n_root;
+  int nx, ny, PX, npts, kmax, kap, k, H, n_theta, max_depth, n_root, rule;
   double hx, hy, inv_hx, inv_hy, cdt, tau, R;
   size_t slot_doubles;
   const double* ring;        // padded ring, slot 0 node (-PAD, -PAD)
@@ -550,7 +550,7 @@ __device__ __forceinline__ void eval_nodes(const Item& it, const Params& P, cons
     const double ws = KIND == RP_SRC_GRID ? 0.25 * w : w;  // undo the 2 x 2 weight scaling
     const double wk = ws * nd.wk;
     k0 += wk * f0; k1 += wk * f1; k2 += wk * f2;
-    if (n & 1) {  // Gauss nodes only (warp-uniform: all lanes walk the same n)
+    if ((n & 1) || P.rule == RP_RULE_SIMPSON) {  // G7: Gauss nodes only (warp-uniform n)
       const double wg = ws * nd.wg;
       g0 += wg * f0; g1 += wg * f1; g2 += wg * f2;
     }
@@ -604,10 +604,14 @@ __global__ void __launch_bounds__(32 * kWarps) k_integrate(
       const double m = __dmul_rn(0.5, __dadd_rn(a, b)), hw = __dmul_rn(0.5, __dsub_rn(b, a));
       // ---- node phase: lanes 0..14 build the r' nodes of the GK15 rule
       int cnt = 0;
-      if (lane < 15) {
+      const int nn = P.rule == RP_RULE_SIMPSON ? 5 : 15;  // r' nodes per segment
+      if (lane < nn) {
         const int i = lane < 7 ? lane : (lane == 7 ? 7 : 14 - lane);
         double r;
-        if (lane < 7) r = __dsub_rn(m, __dmul_rn(hw, c_xgk[i]));
+        if (P.rule == RP_RULE_SIMPSON) {  // r_0 = a, r_2 = m, r_4 = b, r_1, r_3 midpoints
+          r = lane == 0 ? a : lane == 2 ? m : lane == 4 ? b
+                                : __dmul_rn(0.5, __dadd_rn(lane == 1 ? a : m, lane == 1 ? m : b));
+        } else if (lane < 7) r = __dsub_rn(m, __dmul_rn(hw, c_xgk[i]));
         else if (lane == 7) r = m;
         else r = __dadd_rn(m, __dmul_rn(hw, c_xgk[i]));
         double cu, cv, w0, w1, w2;
@@ -616,8 +620,14 @@ __global__ void __launch_bounds__(32 * kWarps) k_integrate(
         int na = arcs<KIND>(it, P, cu, cv, r, th1, dth);
         NodeRec nr;
         nr.r = r; nr.cu = cu; nr.cv = cv; nr.w0 = w0; nr.w1 = w1; nr.w2 = w2;
-        nr.wk = hw * c_wgk[i];
-        nr.wg = (i & 1) ? hw * c_wg[i >> 1] : 0.0;  // Gauss nodes are the odd i (i = 7 centre)
+        if (P.rule == RP_RULE_SIMPSON) {  // Boole h/90 (7,32,12,32,7); Simpson h/12 (1,4,2,4,1)
+          const double h = __dsub_rn(b, a);
+          nr.wk = h / 90.0 * (lane == 2 ? 12.0 : (lane & 1) ? 32.0 : 7.0);
+          nr.wg = h / 12.0 * (lane == 2 ? 2.0 : (lane & 1) ? 4.0 : 1.0);
+        } else {
+          nr.wk = hw * c_wgk[i];
+          nr.wg = (i & 1) ? hw * c_wg[i >> 1] : 0.0;  // Gauss nodes are the odd i (i = 7 centre)
+        }
         S.node[lane] = nr;
         S.na[lane] = na;
         for (int q = 0; q < (na > 0 ? na : 0); ++q) {
@@ -651,11 +661,11 @@ __global__ void __launch_bounds__(32 * kWarps) k_integrate(
       const int rounds = emax >> 5, left = emax - 32 * rounds;
       for (int rr = 0; rr < rounds; ++rr) {
         const int r = (nseg & 1) ? rounds - 1 - rr : rr;
-        eval_nodes<KIND>(it, P, S, trig_full, 32 * r + lane, 0, 15, N, wfull, third, st, cix, ciy,
+        eval_nodes<KIND>(it, P, S, trig_full, 32 * r + lane, 0, nn, N, wfull, third, st, cix, ciy,
                          k0, k1, k2, g0, g1, g2);
       }
-      for (int u = lane; u < 15 * left; u += 32) {
-        const int e = 32 * rounds + u / 15, n = u - 15 * (u / 15);
+      for (int u = lane; u < nn * left; u += 32) {
+        const int e = 32 * rounds + u / nn, n = u - nn * (u / nn);
         eval_nodes<KIND, false>(it, P, S, trig_full, e, n, n + 1, N, wfull, third, st, cix, ciy,
                                 k0, k1, k2, g0, g1, g2);
       }
@@ -903,7 +913,7 @@ int rp_potentials_impl(rp_ctx* ctx, int kind, const double src[6], int32_t rank,
   Params P;
   P.nx = c.nx; P.ny = c.ny; P.PX = ctx->PX; P.npts = c.nx * c.ny; P.kmax = c.history_depth;
   P.kap = kappa_of(ctx); P.k = ctx->k; P.H = ctx->H; P.n_theta = c.n_theta;
-  P.max_depth = c.max_depth; P.n_root = c.n_root;
+  P.max_depth = c.max_depth; P.n_root = c.n_root; P.rule = c.outer_rule;
   P.hx = c.hx; P.hy = c.hy; P.inv_hx = 1.0 / c.hx; P.inv_hy = 1.0 / c.hy;
   P.cdt = c.c * c.dt; P.tau = c.tau; P.R = (double)P.kap * P.cdt;
   P.slot_doubles = ctx->slot_doubles; P.ring = ctx->ring; P.frames = ctx->frames_dev;
@@ -926,7 +936,7 @@ int rp_potentials_impl(rp_ctx* ctx, int kind, const double src[6], int32_t rank,
       info->items = (int64_t)h[C_ITEMS];
       info->evals = (int64_t)h[C_EVALS];
       info->segments = (int64_t)h[C_SEGS];
-      info->nodes = 15 * (int64_t)h[C_SEGS];
+      info->nodes = (c.outer_rule == RP_RULE_SIMPSON ? 5 : 15) * (int64_t)h[C_SEGS];
       info->leaves = (int64_t)h[C_LEAVES];
       info->capped = (int64_t)h[C_CAPPED];
       info->ties = (int64_t)h[C_TIES];

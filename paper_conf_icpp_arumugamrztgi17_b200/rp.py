@@ -18,6 +18,7 @@ LIB_PATH = os.path.join(_HERE, "librp.so")
 
 RP_SRC_GRID, RP_SRC_GAUSS, RP_SRC_DISK = 0, 1, 2
 RP_SCHED_INDEX, RP_SCHED_PERSISTENCE, RP_SCHED_KNN = 0, 1, 2
+RP_RULE_GK15, RP_RULE_SIMPSON = 0, 1
 
 
 class RpError(RuntimeError):
@@ -35,7 +36,7 @@ class rp_config(C.Structure):
     _fields_ = [("nx", C.c_int32), ("ny", C.c_int32), ("hx", C.c_double), ("hy", C.c_double),
                 ("history_depth", C.c_int32), ("c", C.c_double), ("dt", C.c_double),
                 ("tau", C.c_double), ("n_theta", C.c_int32), ("max_depth", C.c_int32),
-                ("n_root", C.c_int32), ("device", C.c_int32)]
+                ("n_root", C.c_int32), ("device", C.c_int32), ("outer_rule", C.c_int32)]
 
 
 class rp_deposit_info(C.Structure):
@@ -195,8 +196,9 @@ def rp_profile_read(ctx) -> rp_profile:
 
 
 def rp_create(nx, ny, hx, hy, history_depth, c, dt, tau, n_theta=64, max_depth=30, n_root=2,
-              device=0):
-    cfg = rp_config(nx, ny, hx, hy, history_depth, c, dt, tau, n_theta, max_depth, n_root, device)
+              device=0, outer_rule=0):
+    cfg = rp_config(nx, ny, hx, hy, history_depth, c, dt, tau, n_theta, max_depth, n_root, device,
+                    outer_rule)
     out = C.c_void_p()
     _check(_lib.rp_create(C.byref(cfg), C.byref(out)), None, "rp_create")
     return out

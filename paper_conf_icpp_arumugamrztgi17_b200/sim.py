@@ -37,7 +37,8 @@ class Simulation:
         self.device = torch.device("cuda", torch.cuda.current_device()) if device is None else torch.device(device)
         dev_index = self.device.index if self.device.type == "cuda" else 0
         self.ctx = ops.rp_create(cfg.nx, cfg.ny, cfg.hx, cfg.hy, cfg.kappa_max, cfg.c, cfg.dt,
-                                 cfg.tau, cfg.n_theta, cfg.max_depth, cfg.n_root, dev_index or 0)
+                                 cfg.tau, cfg.n_theta, cfg.max_depth, cfg.n_root, dev_index or 0,
+                                 cfg.rule)
         if self.device.type == "cuda":
             ops.rp_set_stream(self.ctx, torch.cuda.current_stream(self.device))
         ops.rp_history_init(self.ctx, cfg.n_pre, W.frames(cfg, range(-cfg.n_pre, 0)), None, True)

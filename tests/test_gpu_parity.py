@@ -180,11 +180,14 @@ def _bend_small(n=24, kap=60):
                     r0=c.r0, sigma_xp=c.sigma_xp, q_over_mc=c.q_over_mc)
 
 
-def test_potentials_bend_small_full_mesh_two_steps(torch):
+@pytest.mark.parametrize("rule", [0, 1])
+def test_potentials_bend_small_full_mesh_two_steps(torch, rule):
     """Moving frames, node-sampled history with a time-varying amplitude, two consecutive
-    steps (the second uses the first step's counts as the schedule forecast)."""
+    steps (the second uses the first step's counts as the schedule forecast); GK15 and the
+    paper's Simpson rule (R-22)."""
     from paper_conf_icpp_arumugamrztgi17_b200 import rp
     cfg = _bend_small()
+    cfg.rule = rule
     ctx = G.make_ctx(cfg)
     try:
         for k in (5, 6):
@@ -201,7 +204,8 @@ def test_potentials_bend_small_full_mesh_two_steps(torch):
         rp.rp_destroy(ctx)
 
 
-@pytest.mark.parametrize("variant", [dict(n_root=1), dict(max_depth=5), dict(n_theta=16)])
+@pytest.mark.parametrize("variant", [dict(n_root=1), dict(max_depth=5), dict(n_theta=16),
+                                     dict(rule=1), dict(rule=1, n_root=1)])
 def test_potentials_variants(torch, variant):
     from paper_conf_icpp_arumugamrztgi17_b200 import rp
     cfg = W.Config(number=0, name="v", nx=20, ny=13, n_particles=4000, steps=4, kappa_max=7,

@@ -34,10 +34,23 @@ def gauss_problem(kap=12, cdt=1.6, k=20, tau=1e-6 * SQ, amp=None, beta=(0.0, 0.0
 @pytest.mark.parametrize("s", [0.0, 0.5, 1.0, 2.0, 4.0, 6.5])
 def test_static_gaussian_closed_form(s):
     P = gauss_problem(beta=(0.3, -0.2))
+    _check_gauss(P, s, tight=True)
+
+
+@pytest.mark.parametrize("s", [0.0, 1.0, 4.0])
+def test_static_gaussian_closed_form_simpson_rule(s):
+    """The paper's own outer rule (R-22) meets tau on the closed form too."""
+    P = gauss_problem(beta=(0.3, -0.2))
+    P.params.rule = 1
+    _check_gauss(P, s, tight=False)
+
+
+def _check_gauss(P, s, tight):
     r = P.point_lab(s * math.cos(0.4), s * math.sin(0.4))
     exact = SQ * sp.i0e(s * s / 4)
     assert abs(r.phi - exact) < 1e-6 * SQ
-    assert abs(r.phi - exact) < 1e-13  # the tree is far inside tau on a smooth source
+    if tight:
+        assert abs(r.phi - exact) < 1e-13  # GK15 is far inside tau on a smooth source
     # A = beta * phi for a rigid current (same integrand times a constant)
     assert abs(r.ax - 0.3 * r.phi) < 1e-15 and abs(r.ay + 0.2 * r.phi) < 1e-15
     assert r.capped == 0 and r.ties == 0
@@ -123,9 +136,10 @@ def _brute_outer(P, cfg, ix, iy, pieces=16):
 
 
 @pytest.mark.slow
-@pytest.mark.parametrize("ix,iy", [(15, 0), (8, 8), (3, 12)])
-def test_grid_outer_vs_bruteforce(ix, iy):
+@pytest.mark.parametrize("ix,iy,rule", [(15, 0, 0), (8, 8, 0), (3, 12, 0), (8, 8, 1), (15, 0, 1)])
+def test_grid_outer_vs_bruteforce(ix, iy, rule):
     cfg, P = _small_grid_problem()
+    P.params.rule = rule
     r = P.potentials([iy * cfg.nx + ix])[0]
     brute = _brute_outer(P, cfg, ix, iy, pieces=8)
     got = np.array([r["phi"], r["ax"], r["ay"]])

@@ -84,7 +84,8 @@ def test_lagrange3_reproduces_quadratics():
     np.testing.assert_array_equal(oracle.lagrange3_weights(0.0), [0.0, 1.0, 0.0])
 
 
-def test_gk15_segment_on_exact_quadratic():
+@pytest.mark.parametrize("rule", [0, 1])
+def test_gk15_segment_on_exact_quadratic(rule):
     # disk of radius a=10 centred on p: inner(r') = 2*pi*sigma_s*amp(t_k - r'/c) for r' < a.
     # amp is quadratic in time -> Lagrange-3 exact -> inner is an exact quadratic in r'.
     kap, dt, k = 4, 1.0, 9
@@ -95,7 +96,8 @@ def test_gk15_segment_on_exact_quadratic():
         t = l * dt
         amp[l % H] = al + be * t + ga * t * t
     P = oracle.Problem(nx=8, ny=8, hx=1.0, hy=1.0, c=1.0, dt=dt, tau=1e-9, kappa_max=kap, k=k,
-                       n_pre=0, source=oracle.SRC_DISK, x0=0.0, y0=0.0, width=10.0, q=2.0, amp=amp)
+                       n_pre=0, source=oracle.SRC_DISK, x0=0.0, y0=0.0, width=10.0, q=2.0, amp=amp,
+                       rule=rule)
     for j, (a, b) in [(0, (0.1, 0.9)), (2, (2.0, 3.0)), (3, (3.25, 3.5))]:
         K, G, err = P.gk15(0.0, 0.0, j, a, b)
         tk = k * dt
@@ -104,3 +106,23 @@ def test_gk15_segment_on_exact_quadratic():
         assert abs(K[0] - exact) < 1e-13 * abs(exact)
         assert abs(G[0] - exact) < 1e-13 * abs(exact)
         assert err < 1e-13 * abs(exact)
+
+
+def test_simpson_boole_weights():
+    """Rule 1 (the paper's Simpson, with the standard Richardson value = Boole's rule,
+    R-22): Boole h/90 (7,32,12,32,7) is exact to degree 5 and not 6, Simpson h/12 (1,4,2,4,1)
+    to degree 3 and not 4, on [0, 1] with nodes 0, 1/4, 1/2, 3/4, 1."""
+    x = np.array([0.0, 0.25, 0.5, 0.75, 1.0])
+    wb = np.array([7, 32, 12, 32, 7]) / 90.0
+    ws = np.array([1, 4, 2, 4, 1]) / 12.0
+    for d in range(6):
+        assert abs(np.dot(wb, x ** d) - 1.0 / (d + 1)) < 1e-15
+    assert abs(np.dot(wb, x ** 6) - 1.0 / 7) > 1e-6
+    for d in range(4):
+        assert abs(np.dot(ws, x ** d) - 1.0 / (d + 1)) < 1e-15
+    assert abs(np.dot(ws, x ** 4) - 1.0 / 5) > 1e-5
+    # the oracle's rule-1 segment on a constant inner integral (disk seen from its centre)
+    P = oracle.Problem(nx=8, ny=8, hx=1.0, hy=1.0, c=1.0, dt=1.0, tau=1e-9, kappa_max=3, k=9,
+                       n_pre=0, source=oracle.SRC_DISK, x0=0.0, y0=0.0, width=10.0, q=1.5, rule=1)
+    K, G, err = P.gk15(0.0, 0.0, 1, 1.2, 1.9)
+    assert abs(K[0] - 2 * math.pi * 1.5 * 0.7) < 1e-13 and err < 1e-13

@@ -46,6 +46,7 @@ class Config:
     n_theta: int = 64
     max_depth: int = 30
     n_root: int = 2
+    rule: int = 0            # outer segment rule: 0 = GK15, 1 = Simpson/Boole (the paper's)
     tau_rel: float = 1e-6    # tau = tau_rel * (Q/sigma) sqrt(pi/2)
     seed: int = 0
 
