@@ -183,7 +183,8 @@ int rp_push_particles(rp_ctx* ctx, double* x, double* y, double* ux, double* uy,
  * host->device, runs deposit_step, compute_potentials, compute_fields (with the previous
  * step's A kept by the context), push, and copies the pushed particles and the six mesh
  * outputs back.  x_host .. uy_host are updated in place; mesh_host is [6][ny*nx]
- * (phi, ax, ay, ex, ey, bz).  Pinned host memory gives full-bandwidth copies.  Syncs. */
+ * (phi, ax, ay, ex, ey, bz).  Pinned host memory gives full-bandwidth copies.  info
+ * (nullable) receives the potentials' work counters.  Syncs. */
 int rp_step_host(rp_ctx* ctx, double* x_host, double* y_host, double* ux_host,
                  double* uy_host, int64_t n, double q, const rp_frame* frame_k,
                  double q_over_mc, double bz_ext, double* mesh_host, rp_potential_info* info);

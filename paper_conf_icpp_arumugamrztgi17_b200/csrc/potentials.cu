@@ -10,9 +10,10 @@
 //   k_integrate  persistent warps pull (p, j) items; each warp walks the canonical dyadic
 //                GK15 tree of its item depth-first without a stack (R-8..R-12).  Per
 //                segment lanes 0..14 build the 15 r' nodes (retarded frame, circle/support
-//                arcs, R-5/R-7), then all 32 lanes sweep the flattened (node, arc, theta)
-//                evaluations of f (27-point TSC x Lagrange-3 gather, R-6) and reduce with
-//                xor shuffles, so every accept/split decision is warp-uniform.
+//                arcs, R-5/R-7); then lane l evaluates f (27-point TSC x Lagrange-3 gather,
+//                R-6) at theta slot 32r+l for all 15 nodes from a register stencil cache that
+//                survives across radially adjacent segments, and the K15/G7 sums are reduced
+//                with xor shuffles, so every accept/split decision is warp-uniform.
 //   k_reduce     per point, sum the items in j order -> phi, A, err, nseg; counts.
 // FP64 throughout.  No tensor cores: the work is an irregular gather stencil,
 // not a dense contraction.
@@ -426,17 +427,12 @@ struct WarpSmem {
   int na[16], cnt[16];
 };
 
-#ifndef RP_CHUNK
-#define RP_CHUNK 5
-#endif
-constexpr int kChunk = RP_CHUNK, kNChunks = 15 / RP_CHUNK;  // 15 r' nodes = kNChunks chunks
-
 // 256-bit read-only load of one padded node record (rho, rho*bx, rho*by, 0): sm_100
 // LDG.E.ENL2.256, one instruction per stencil node.
 __device__ __forceinline__ void ldg_node(const double* p, double& a, double& b, double& c) {
   double d;
   asm("ld.global.nc.v4.f64 {%0,%1,%2,%3}, [%4];" : "=d"(a), "=d"(b), "=d"(c), "=d"(d) : "l"(p));
-}  // 15 r' nodes = 3 chunks of 5
+}
 
 // Theta slot e of the r' nodes n0 .. n1-1 of the current segment.  The 27-node x 3-component
 // stencil cache (st, cix, ciy) belongs to the caller, so it survives across calls: a lane that
@@ -646,9 +642,7 @@ __global__ void __launch_bounds__(32 * kWarps) k_integrate(
       if (lane < 16) S.cnt[lane] = lane < 15 ? cnt : 0;
       const int E = __shfl_sync(0xffffffffu, incl, 31);
       __syncwarp();
-      // ---- evaluation phase: lane <-> (theta slot e, chunk c of kChunk r' nodes).  In a
-      // deep segment the points X_{n,e} of one chunk fall in the same cell, so the 27-node x
-      // 3-component stencil is loaded once into registers and reused across the chunk.
+      // ---- evaluation phase
       int emax = cnt;
 #pragma unroll
       for (int o = 16; o > 0; o >>= 1) emax = max(emax, __shfl_xor_sync(0xffffffffu, emax, o));

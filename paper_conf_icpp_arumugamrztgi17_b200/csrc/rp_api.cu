@@ -321,7 +321,7 @@ int rp_step_host(rp_ctx* ctx, double* xh, double* yh, double* uxh, double* uyh, 
   int rc = rp_deposit_step(ctx, ctx->hx_d, ctx->hy_d, ctx->hux_d, ctx->huy_d, q, n, frame_k, nullptr);
   if (rc) return rc;
   rc = rp_potentials_impl(ctx, RP_SRC_GRID, nullptr, 0, 1, phi, ax, ay, nullptr, nullptr, nullptr,
-                          0, nullptr, nullptr);
+                          0, nullptr, info);
   if (rc) return rc;
   rc = rp_fields_impl(ctx, phi, ax, ay, ctx->have_prev_A ? axp : nullptr,
                       ctx->have_prev_A ? ayp : nullptr, ex, ey, bz);
@@ -338,7 +338,6 @@ int rp_step_host(rp_ctx* ctx, double* xh, double* yh, double* uxh, double* uyh, 
     RP_CUDA(cudaMemcpyAsync(uyh, ctx->huy_d, nb, cudaMemcpyDeviceToHost, st));
   }
   RP_CUDA(cudaStreamSynchronize(st));
-  (void)info;
   return RP_OK;
 }
 

@@ -293,12 +293,15 @@ def rp_push_particles(ctx, x, y, ux, uy, q_over_mc, bz_ext, ex, ey, bz) -> None:
            ctx, "rp_push_particles")
 
 
-def rp_step_host(ctx, x, y, ux, uy, q, frame_k, q_over_mc, bz_ext, mesh_out) -> None:
+def rp_step_host(ctx, x, y, ux, uy, q, frame_k, q_over_mc, bz_ext, mesh_out, info=False):
     """x..uy and mesh_out ([6, npts]) are host buffers (pinned torch CPU tensors or numpy)."""
     n = x.numel() if hasattr(x, "numel") else len(x)
+    inf = rp_potential_info() if info else None
     _check(_lib.rp_step_host(ctx, _host(x), _host(y), _host(ux), _host(uy), n, float(q),
                              C.byref(frame(frame_k)), float(q_over_mc), float(bz_ext),
-                             _host(mesh_out), None), ctx, "rp_step_host")
+                             _host(mesh_out), C.byref(inf) if inf is not None else None), ctx,
+           "rp_step_host")
+    return inf
 
 
 def rp_load_state(ctx, k, n_pre, frames, ring) -> None:
