@@ -358,7 +358,7 @@ def _oracle_state(cfg):
     t0 = time.perf_counter()
     M, _, _ = oracle.deposit(x, y, ux, uy, q, W.frame(cfg, 0), cfg.nx, cfg.ny, cfg.hx, cfg.hy)
     t_dep = time.perf_counter() - t0
-    ring = np.repeat(M[None], cfg.H, axis=0)
+    ring = oracle.rigid_ring(M, W.ring_frames(cfg, 0))
     P = oracle.Problem(nx=cfg.nx, ny=cfg.ny, hx=cfg.hx, hy=cfg.hy, c=cfg.c, dt=cfg.dt, tau=cfg.tau,
                        kappa_max=cfg.kappa_max, k=0, n_pre=cfg.n_pre, ring=ring,
                        frames=W.ring_frames(cfg, 0), n_theta=cfg.n_theta, max_depth=cfg.max_depth,

@@ -101,8 +101,11 @@ int rp_set_stream(rp_ctx* ctx, void* stream);
 /* Optional pre-history, allowed only before the first deposit (else ESTATE).
  * n_pre in 1..history_depth+1 levels l = -n_pre .. -1; frames_host[n_pre] oldest first.
  * rigid = 0: grids_dev holds [n_pre][ny][nx][4] FP64 moment grids (component 3 ignored).
- * rigid = 1: grids_dev must be NULL; every pre-history level receives a copy of the
- *            step-0 grid when the first deposit is appended (steady state).
+ * rigid = 1: grids_dev must be NULL; every pre-history level l receives the step-0 grid
+ *            when the first deposit is appended (steady state): rho copied,
+ *            the current rotated from frame 0 to frame l (J_l = R(psi_l - psi_0) J_0 with
+ *            cos/sin of the difference from the frames' (cos, sin), R-23), so that every
+ *            level holds the same comoving bunch.  Static frames: an exact copy.
  * Without pre-history, kappa(k) = min(kappa_max, k - 1) (R-3). */
 int rp_history_init(rp_ctx* ctx, int32_t n_pre, const rp_frame* frames_host,
                     const double* grids_dev, int32_t rigid);

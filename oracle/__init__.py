@@ -80,6 +80,7 @@ def lib():
             "orc_lagrange3_weights": (None, [d, pd]),
             "orc_bin_of": (i32, [d, d, P(Frame), d, d, i32, i32, pi32, pi32, pd, pd]),
             "orc_deposit": (d, [i64, pd, pd, pd, pd, d, P(Frame), i32, i32, d, d, pd, pi32]),
+            "orc_rigid_level": (None, [pd, P(Frame), P(Frame), i32, i32, pd]),
             "orc_arcs_rect": (i32, [d, d, d, d, d, d, d, pd]),
             "orc_arcs_disk": (i32, [d, d, d, d, d, d, pd]),
             "orc_kappa": (i32, [P(Params), P(Hist)]),
@@ -237,6 +238,28 @@ def deposit(x, y, ux, uy, q, fr, nx, ny, hx, hy):
     ql = lib().orc_deposit(len(x), _pd(x), _pd(y), _pd(ux), _pd(uy), q, C.byref(frame(fr)),
                            nx, ny, hx, hy, _pd(M), _pi(bins))
     return M, bins, ql
+
+
+def rigid_level(M0, f0, fl):
+    """Step-0 moments M0 [ny,nx,4] as the same comoving bunch in frame fl (R-23)."""
+    M0 = np.ascontiguousarray(M0, dtype=np.float64)
+    ny, nx = M0.shape[:2]
+    out = np.zeros_like(M0)
+    lib().orc_rigid_level(_pd(M0), C.byref(frame(f0)), C.byref(frame(fl)), nx, ny, _pd(out))
+    return out
+
+
+def rigid_ring(M0, ring_frames, k=0, n_pre=None):
+    """Ring [H,ny,nx,4] at step k = 0 of a rigid pre-history: slot(0) = M0, slot(l) for the
+    n_pre levels l = -n_pre..-1 = rigid_level(M0, frame 0, frame l).  ``ring_frames`` as
+    stored in the ring (slot(l) = l mod H)."""
+    H = len(ring_frames)
+    n_pre = H - 1 if n_pre is None else n_pre
+    ring = np.zeros((H,) + np.shape(M0))
+    ring[0] = M0
+    for l in range(-n_pre, 0):
+        ring[l % H] = rigid_level(M0, ring_frames[0], ring_frames[l % H])
+    return ring
 
 
 def arcs_rect(cu, cv, r, U0, U1, V0, V1):

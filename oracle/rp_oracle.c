@@ -180,6 +180,26 @@ double orc_deposit(int64_t n, const double* x, const double* y, const double* ux
   return q_lost;
 }
 
+/* Rigid steady-state pre-history level (SURVEY 8(d) steady state; DESIGN R-23): the same
+ * comoving bunch as step 0, viewed in frame Fl.  rho is copied; the lab current is rotated
+ * by the angle between the frames, psi_l - psi_0:
+ *   cos(psi_l - psi_0) = c_l c_0 + s_l s_0,  sin(psi_l - psi_0) = s_l c_0 - c_l s_0,
+ *   J_l = [[cos, -sin], [sin, cos]] J_0.
+ * M0, Ml: [ny][nx][4]. */
+void orc_rigid_level(const double* M0, const orc_frame* F0, const orc_frame* Fl, int32_t nx,
+                     int32_t ny, double* Ml) {
+  double cd = Fl->c * F0->c + Fl->s * F0->s;
+  double sd = Fl->s * F0->c - Fl->c * F0->s;
+  for (int64_t i = 0; i < (int64_t)nx * ny; ++i) {
+    const double* m = M0 + 4 * i;
+    double* o = Ml + 4 * i;
+    o[0] = m[0];
+    o[1] = cd * m[1] - sd * m[2];
+    o[2] = sd * m[1] + cd * m[2];
+    o[3] = m[3];
+  }
+}
+
 /* ------------------------------------------------------------------ */
 /* History access ("stored linearly"; ring of H slots)            */
 /* ------------------------------------------------------------------ */

@@ -10,6 +10,8 @@
 // number (quantum 2^-shift, shift from |q|/(hx hy) so 2^40 particles cannot overflow) and the
 // integer sums are order-independent, so D_k is bit-identical however the particles are split
 // over ranks, lanes or warps.  The one rounding to FP64 happens in k_append.
+#include <algorithm>
+
 #include <cub/device/device_radix_sort.cuh>
 
 #include "rp_internal.cuh"
@@ -143,6 +145,27 @@ __global__ void k_append(int nx, int ny, int PX, const unsigned char* __restrict
   dst[3] = 0.0;
 }
 
+// Rigid steady-state pre-history (R-23): level l gets the step-0 moments with the current
+// rotated from frame 0 to frame l, J_l = R(psi_l - psi_0) J_0, so that every level holds the
+// same comoving bunch (same local (J.t, J.n)).  cos/sin of the difference angle from the
+// frames' (cos, sin) pairs; explicit _rn operations (no FMA contraction) so the copy is a
+// fixed function of the inputs.  Static frames give cd = 1, sd = 0: an exact copy.
+__global__ void k_rigid_copy(const double* __restrict__ src, double* __restrict__ dst,
+                             size_t nodes, rp_frame f0, rp_frame fl) {
+  const double cd = __dadd_rn(__dmul_rn(fl.cos_psi, f0.cos_psi), __dmul_rn(fl.sin_psi, f0.sin_psi));
+  const double sd = __dsub_rn(__dmul_rn(fl.sin_psi, f0.cos_psi), __dmul_rn(fl.cos_psi, f0.sin_psi));
+  for (size_t i = blockIdx.x * (size_t)blockDim.x + threadIdx.x; i < nodes;
+       i += (size_t)gridDim.x * blockDim.x) {
+    const double4 m = reinterpret_cast<const double4*>(src)[i];
+    double4 o;
+    o.x = m.x;
+    o.y = __dsub_rn(__dmul_rn(cd, m.y), __dmul_rn(sd, m.z));
+    o.z = __dadd_rn(__dmul_rn(sd, m.y), __dmul_rn(cd, m.z));
+    o.w = m.w;
+    reinterpret_cast<double4*>(dst)[i] = o;
+  }
+}
+
 __global__ void k_set_header(long long* hdr, long long shift) {
   hdr[0] = shift;
   hdr[1] = 0;
@@ -261,9 +284,13 @@ int rp_append_impl(rp_ctx* ctx, const void* parts, int32_t n_parts, const rp_fra
   ctx->fh[s] = *fk;
   RP_CUDA(cudaMemcpyAsync(ctx->frames_dev + s, fk, sizeof(rp_frame), cudaMemcpyHostToDevice, st));
   if (knew == 0 && ctx->rigid_pending) {
+    const size_t nodes = ctx->slot_doubles / 4;
     for (int l = -ctx->n_pre; l < 0; ++l) {
-      double* d = ctx->ring + (size_t)slot_of(l, ctx->H) * ctx->slot_doubles;
-      RP_CUDA(cudaMemcpyAsync(d, slot, ctx->slot_doubles * sizeof(double), cudaMemcpyDeviceToDevice, st));
+      const int sl = slot_of(l, ctx->H);
+      double* d = ctx->ring + (size_t)sl * ctx->slot_doubles;
+      k_rigid_copy<<<(unsigned)std::min<size_t>((nodes + 255) / 256, 4 * 148), 256, 0, st>>>(
+          slot, d, nodes, *fk, ctx->fh[sl]);
+      RP_CHECK_LAUNCH();
     }
     ctx->rigid_pending = 0;
   }

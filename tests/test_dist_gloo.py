@@ -72,7 +72,7 @@ class OracleOps:
         ctx.frames[ctx.k % ctx.H] = fk
         if ctx.k == 0 and ctx.rigid:
             for l in range(-ctx.n_pre, 0):
-                ctx.ring[l % ctx.H] = tot
+                ctx.ring[l % ctx.H] = oracle.rigid_level(tot, fk, ctx.frames[l % ctx.H])
 
     def rp_deposit_step(self, ctx, x, y, ux, uy, q, fk, info=False):
         part = torch.zeros(self.rp_partial_bytes(ctx), dtype=torch.uint8)

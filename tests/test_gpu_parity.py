@@ -71,6 +71,32 @@ def test_deposit_bins_bit_exact_and_moments(torch, cfgno):
         rp.rp_destroy(ctx)
 
 
+def test_rigid_prehistory_rotates_the_current(torch):
+    """rp_history_init(rigid=1) on the bend (R-23): every pre-history level is the step-0
+    deposit as the same comoving bunch in that level's frame (oracle.rigid_ring)."""
+    from paper_conf_icpp_arumugamrztgi17_b200 import rp
+    cfg = W.config(2)
+    x, y, ux, uy = W.particles(cfg, n=20_000, seed=11)
+    q = 1.0 / len(x)
+    M, _, _ = oracle.deposit(x, y, ux, uy, q, W.frame(cfg, 0), cfg.nx, cfg.ny, cfg.hx, cfg.hy)
+    want = oracle.rigid_ring(M, W.ring_frames(cfg, 0))
+    ctx = G.make_ctx(cfg)
+    try:
+        rp.rp_history_init(ctx, cfg.n_pre, W.frames(cfg, range(-cfg.n_pre, 0)), None, True)
+        xd, yd, uxd, uyd = _dev_arrays(torch, x, y, ux, uy)
+        rp.rp_deposit_step(ctx, xd, yd, uxd, uyd, q, W.frame(cfg, 0))
+        ring = torch.zeros((cfg.H, cfg.ny, cfg.nx, 4), dtype=torch.float64, device="cuda")
+        rp.rp_save_state(ctx, ring)
+        got = ring.cpu().numpy()
+    finally:
+        rp.rp_destroy(ctx)
+    scale = np.abs(M).max()
+    assert np.abs(got - want).max() <= 1e-12 * scale
+    for l in range(-cfg.n_pre, 0):  # rho is a copy of slot 0 bit for bit
+        np.testing.assert_array_equal(got[l % cfg.H, ..., 0], got[0, ..., 0])
+    assert np.abs(got[1, ..., 2] - got[0, ..., 2]).max() > 0.05 * np.abs(got[0, ..., 1]).max()
+
+
 def test_deposit_exact_for_any_particle_split(torch):
     """Exact fixed-point partial sums: depositing the bunch in one piece or
     split into 3 unequal rank shards and appending the partials gives a bit-identical D_k."""
@@ -124,7 +150,7 @@ def _deposit_rigid_ring(cfg, n=None, seed=None):
     x, y, ux, uy = W.particles(cfg, n=n, seed=seed)
     q = 1.0 / len(x)
     M, _, _ = oracle.deposit(x, y, ux, uy, q, W.frame(cfg, 0), cfg.nx, cfg.ny, cfg.hx, cfg.hy)
-    return np.repeat(M[None], cfg.H, axis=0), (x, y, ux, uy, q)
+    return oracle.rigid_ring(M, W.ring_frames(cfg, 0)), (x, y, ux, uy, q)
 
 
 def test_potentials_static_cfg1_full_mesh(torch):

@@ -84,3 +84,44 @@ def test_bend_steady_state_stationarity():
     # sanity: the bend potential at the bunch centre is O(Q/sigma)
     scale = 1.0 / cfg.sigma * math.sqrt(math.pi / 2)
     assert 0.5 < out[0]["phi"][0] / scale < 10
+
+
+# ---------------------------------------------------------------- rigid pre-history (R-23)
+def test_rigid_level_static_frames_is_exact_copy():
+    cfg = _cfg_static()
+    rng = np.random.default_rng(5)
+    M = rng.standard_normal((cfg.ny, cfg.nx, 4))
+    out = oracle.rigid_level(M, W.frame(cfg, 0), W.frame(cfg, -3))
+    np.testing.assert_array_equal(out, M)
+
+
+def test_rigid_level_quarter_turn_is_exact():
+    # psi_0 = 0, psi_l = pi/2 given exactly as (cos, sin) = (0, 1): (jx, jy) -> (-jy, jx)
+    M = np.random.default_rng(6).standard_normal((5, 6, 4))
+    out = oracle.rigid_level(M, [0, 0, 1.0, 0.0], [0, 0, 0.0, 1.0])
+    np.testing.assert_array_equal(out[..., 0], M[..., 0])
+    np.testing.assert_array_equal(out[..., 1], -M[..., 2])
+    np.testing.assert_array_equal(out[..., 2], M[..., 1])
+
+
+def test_rigid_ring_carries_the_tangent_current_of_each_level():
+    """A bunch moving along the step-0 tangent becomes, at every pre-history level, a bunch
+    moving along THAT level's tangent (circular orbit; the closed form of the rotation), with
+    the same charge density and the same local (J.t, J.n) components."""
+    cfg = _bend_small()
+    fr = W.ring_frames(cfg, 0)
+    g = W.node_gaussian_ring(cfg, k=0)[0, :, :, 0]
+    b = cfg.beta0
+    M0 = np.zeros((cfg.ny, cfg.nx, 4))
+    M0[..., 0] = g
+    M0[..., 1] = g * b * fr[0, 2]
+    M0[..., 2] = g * b * fr[0, 3]
+    ring = oracle.rigid_ring(M0, fr)
+    for l in range(-cfg.n_pre, 0):
+        _, _, c, s = W.frame(cfg, l)
+        R = ring[l % cfg.H]
+        np.testing.assert_array_equal(R[..., 0], g)
+        np.testing.assert_allclose(R[..., 1], g * b * c, rtol=0, atol=1e-15 * g.max())
+        np.testing.assert_allclose(R[..., 2], g * b * s, rtol=0, atol=1e-15 * g.max())
+    # the oldest level (l = -61, psi = -0.12 rad) is rotated, not copied
+    assert np.abs(ring[1, ..., 2]).max() > 0.1 * b * g.max()

@@ -11,7 +11,7 @@ lays out the geometry the paper's workloads are quoted on:
 
 Recipe (DESIGN.md sec. 2 "Inputs"): numpy PCG64 with seed 17_000 + config
 number; Gaussian bunch in the comoving frame; frames on the reference orbit;
-rigid steady-state pre-history (n_pre = kappa_max + 1 copies of step 0).
+rigid steady-state pre-history (n_pre = kappa_max + 1 levels of the step-0 bunch, R-23).
 Units: lengths in metres for the bend (sigma = 50e-6), sigma = 1 for the
 static config; c = 1 (time in length units); bunch charge Q = 1.
 """
