@@ -49,7 +49,7 @@ constexpr int kMaxArcs = 8;
 constexpr int kWarps = 4;  // warps per CTA of k_integrate
 
 struct Params {
-  int nx, ny, PX, npts, kmax, kap, k, H, n_theta, max_depth, n_root, rule;
+  int nx, ny, PX, npts, kmax, kap, k, H, n_theta, max_depth, n_root, rule, variant;
   double hx, hy, inv_hx, inv_hy, cdt, tau, R;
   size_t slot_doubles;
   const double* ring;        // padded ring, slot 0 node (-PAD, -PAD)
@@ -314,22 +314,33 @@ __device__ __forceinline__ void integrand(const Item& it, const Params& P, doubl
 // sin/cos for |x| <= 8 pi: Cody-Waite reduction by pi/2 with a two-term constant (k <= 16 is
 // exact enough for ulp-level accuracy) and the classic fdlibm minimax kernels on
 // [-pi/4, pi/4].  No Payne-Hanek slow path, so it inlines small.
+// fdlibm __kernel_sin / __kernel_cos coefficients, in the constant bank so every DFMA takes
+// them as a c[] operand (no per-call uniform-register moves)
+__constant__ double c_sinp[6] = {1.58969099521155010221e-10, -2.50507602534068634195e-08,
+                                 2.75573137070700676789e-06, -1.98412698298579493134e-04,
+                                 8.33333333332248946124e-03, -1.66666666666666324348e-01};
+__constant__ double c_cosp[6] = {-1.13596475577881948265e-11, 2.08757232129817482790e-09,
+                                 -2.75573143513906633035e-07, 2.48015872894767294178e-05,
+                                 -1.38888888888741095749e-03, 4.16666666666666019037e-02};
+__constant__ double c_pio2[3] = {0.63661977236758134308, 1.5707963267948965580,
+                                 6.1232339957367658e-17};  // 2/pi, pi/2 = hi + lo
+
 __device__ __forceinline__ void sincos_b(double x, double* s, double* c) {
-  const double k = rint(x * 0.63661977236758134308);  // 2/pi
-  double r = fma(-k, 1.5707963267948965580, x);
-  r = fma(-k, 6.1232339957367658e-17, r);
+  const double k = rint(x * c_pio2[0]);
+  double r = fma(-k, c_pio2[1], x);
+  r = fma(-k, c_pio2[2], r);
   const double z = r * r;
-  double ps = fma(z, 1.58969099521155010221e-10, -2.50507602534068634195e-08);
-  ps = fma(z, ps, 2.75573137070700676789e-06);
-  ps = fma(z, ps, -1.98412698298579493134e-04);
-  ps = fma(z, ps, 8.33333333332248946124e-03);
-  ps = fma(z, ps, -1.66666666666666324348e-01);
+  double ps = fma(z, c_sinp[0], c_sinp[1]);
+  ps = fma(z, ps, c_sinp[2]);
+  ps = fma(z, ps, c_sinp[3]);
+  ps = fma(z, ps, c_sinp[4]);
+  ps = fma(z, ps, c_sinp[5]);
   const double sr = fma(r * z, ps, r);
-  double pc = fma(z, -1.13596475577881948265e-11, 2.08757232129817482790e-09);
-  pc = fma(z, pc, -2.75573143513906633035e-07);
-  pc = fma(z, pc, 2.48015872894767294178e-05);
-  pc = fma(z, pc, -1.38888888888741095749e-03);
-  pc = fma(z, pc, 4.16666666666666019037e-02);
+  double pc = fma(z, c_cosp[0], c_cosp[1]);
+  pc = fma(z, pc, c_cosp[2]);
+  pc = fma(z, pc, c_cosp[3]);
+  pc = fma(z, pc, c_cosp[4]);
+  pc = fma(z, pc, c_cosp[5]);
   const double cr = fma(z * z, pc, fma(-0.5, z, 1.0));
   const int q = (int)k & 3;
   const double ss = (q & 1) ? cr : sr, cc = (q & 1) ? sr : cr;
@@ -363,11 +374,12 @@ __device__ int arcs(const Item& it, const Params& P, double cu, double cv, doubl
   // node phase runs on 15 lanes once per segment, so code size matters more than ILP).
   double t[8];
   int n = 0;
-#pragma unroll 1
-  for (int e = 0; e < 4; ++e) {
+  const double rinv = 1.0 / r;
+#pragma unroll
+  for (int e = 0; e < 4; ++e) {  // the 4 edges are independent: unrolled for ILP
     const bool vert = e < 2;
     const double edge = e == 0 ? it.U0 : e == 1 ? it.U1 : e == 2 ? it.V0 : it.V1;
-    const double d = (edge - (vert ? cu : cv)) / r;
+    const double d = (edge - (vert ? cu : cv)) * rinv;
     if (!(fabs(d) < 1.0)) continue;
     const double h = r * sqrt(1.0 - d * d);  // r sin(acos d) = r cos(asin d)
     const double lo = vert ? it.V0 : it.U0, hi = vert ? it.V1 : it.U1;
@@ -419,6 +431,8 @@ __device__ int arcs(const Item& it, const Params& P, double cu, double cv, doubl
 struct __align__(16) NodeRec {
   double r, cu, cv, w0, w1, w2, wk, wg;  // r', frame-local centre, time weights, hw*w_GK, hw*w_G7
 };
+
+constexpr int kNoCell = -0x7fffffff;  // geometry record of a slot a node does not have
 
 struct WarpSmem {
   Item it;  // per-item geometry, kept in shared memory to free registers for the eval loop
@@ -553,19 +567,171 @@ __device__ __forceinline__ void eval_nodes(const Item& it, const Params& P, cons
   }
 }
 
+// ---- software-pipelined round (VAR 4): geometry of node n+1 and the contraction of node n
+// form one basic block, so the long sincos / floor chains of the next point fill the latency
+// gaps of the current contraction (2 warps per scheduler cannot hide them otherwise).
+struct Geo {
+  double dx, dy, w;
+  int cell;
+};
+
+// Branch-free geometry of theta slot e of r' node n (FULL: full circle, uniform per node).
+template <bool FULL, int ABL = 0>
+__device__ __forceinline__ Geo geom_point(const Params& P, const WarpSmem& S, double2 trf, int e,
+                                          int n, int N, double wfull, double third,
+                                          float inv_n1) {
+  const bool valid = e < S.cnt[n];
+  double cs, sn, w;
+  if (FULL) {
+    cs = trf.x;
+    sn = trf.y;
+    w = wfull;
+  } else {
+    const int ec = valid ? e : 0;
+    const int q = __float2int_rz(((float)ec + 0.5f) * inv_n1);  // arc index, exact for e < 2^20
+    const int mm = ec - q * (N + 1);
+    const double d = S.dth[n][q];
+    if (ABL == 2) { const double a = S.th1[n][q] + (double)mm * d; cs = 1.0 - 0.5 * a * a; sn = a; }
+    else sincos_b(S.th1[n][q] + (double)mm * d, &sn, &cs);
+    const double coef = (mm == 0 || mm == N) ? 1.0 : ((mm & 1) ? 4.0 : 2.0);
+    w = coef * d * third;
+  }
+  const NodeRec& nd = S.node[n];
+  const double u = nd.cu + nd.r * cs, v = nd.cv + nd.r * sn;
+  const double tx = u * P.inv_hx, ty = v * P.inv_hy;
+  const double fx = floor(tx + 0.5), fy = floor(ty + 0.5);
+  const int ix = min(max(__double2int_rz(fx), -2), P.nx + 1);
+  const int iy = min(max(__double2int_rz(fy), -2), P.ny + 1);
+  Geo g;
+  g.dx = valid ? tx - fx : 0.0;
+  g.dy = valid ? ty - fy : 0.0;
+  g.w = valid ? 0.25 * w : 0.0;  // 0.25 undoes the 2 x 2 scaling of the TSC weights
+  g.cell = valid ? (iy - 1) * P.PX + (ix - 1) : kNoCell;
+  return g;
+}
+
+__device__ __forceinline__ void refill(const Item& it, size_t rs, int cell,
+                                       double (&st)[3][9][3]) {
+  const size_t base = (size_t)4 * (ptrdiff_t)cell;
+  const double* g[3] = {it.g0 + base, it.g1 + base, it.g2 + base};
+#pragma unroll
+  for (int l = 0; l < 3; ++l)
+#pragma unroll
+    for (int b = 0; b < 3; ++b) {
+      const double* row = g[l] + b * rs;
+#pragma unroll
+      for (int a = 0; a < 3; ++a)
+        ldg_node(row + 4 * a, st[l][3 * b + a][0], st[l][3 * b + a][1], st[l][3 * b + a][2]);
+    }
+}
+
+// L1 prefetch of the stencil rows of `cell` when it differs from the cell in use (predicated,
+// branch-free: it sits inside the interleaved geometry/contraction block).  A row of 3 nodes
+// (96 B) spans at most two 128-B lines: prefetch its first and last byte.
+__device__ __forceinline__ void prefetch_cell(const Item& it, size_t rs, int cell, int cur) {
+  const int p = (cell != kNoCell && cell != cur) ? 1 : 0;
+  const size_t base = (size_t)4 * (ptrdiff_t)(p ? cell : 0);
+  const double* g[3] = {it.g0 + base, it.g1 + base, it.g2 + base};
+#pragma unroll
+  for (int l = 0; l < 3; ++l)
+#pragma unroll
+    for (int b = 0; b < 3; ++b) {
+      const double* row = g[l] + b * rs;
+      asm volatile(
+          "{\n\t.reg .pred q;\n\tsetp.ne.s32 q, %2, 0;\n\t"
+          "@q prefetch.global.L1 [%0];\n\t@q prefetch.global.L1 [%1];\n\t}" ::"l"(row),
+          "l"(row + 11), "r"(p));
+    }
+}
+
+// 27-node x 3-component contraction at one point -> (f0, f1, f2)
+__device__ __forceinline__ void contract_point(const Geo& g, const NodeRec& nd,
+                                               const double (&st)[3][9][3], double& f0,
+                                               double& f1, double& f2) {
+  const double dx = g.dx, dy = g.dy;
+  const double ax = 0.5 - dx, bx = 0.5 + dx, ay = 0.5 - dy, by = 0.5 + dy;
+  const double wx[3] = {ax * ax, fma(-2.0 * dx, dx, 1.5), bx * bx};
+  const double wy[3] = {ay * ay, fma(-2.0 * dy, dy, 1.5), by * by};
+  double s[3][3];
+  const double w00 = wx[0] * wy[0];
+#pragma unroll
+  for (int l = 0; l < 3; ++l)
+#pragma unroll
+    for (int c = 0; c < 3; ++c) s[l][c] = w00 * st[l][0][c];
+#pragma unroll
+  for (int i = 1; i < 9; ++i) {
+    const double ww = wx[i % 3] * wy[i / 3];
+#pragma unroll
+    for (int l = 0; l < 3; ++l)
+#pragma unroll
+      for (int c = 0; c < 3; ++c) s[l][c] = fma(ww, st[l][i][c], s[l][c]);
+  }
+  f0 = nd.w0 * s[0][0] + nd.w1 * s[1][0] + nd.w2 * s[2][0];
+  f1 = nd.w0 * s[0][1] + nd.w1 * s[1][1] + nd.w2 * s[2][1];
+  f2 = nd.w0 * s[0][2] + nd.w1 * s[1][2] + nd.w2 * s[2][2];
+}
+
+template <int ABL>
+__device__ __forceinline__ void pipelined_round(const Item& it, const Params& P,
+                                                const WarpSmem& S,
+                                                const double2* __restrict__ trig_full, int e,
+                                                int nn, int N, double wfull, double third,
+                                                double (&st)[3][9][3], int& ccell, double& k0,
+                                                double& k1, double& k2, double& g0, double& g1,
+                                                double& g2, unsigned fullmask) {
+  const size_t rs = (size_t)4 * P.PX;
+  const float inv_n1 = 1.0f / (float)(N + 1);
+  const double2 trf = __ldg(trig_full + (e < N ? e : 0));
+  Geo cur = (fullmask & 1) ? geom_point<true, ABL>(P, S, trf, e, 0, N, wfull, third, inv_n1)
+                        : geom_point<false, ABL>(P, S, trf, e, 0, N, wfull, third, inv_n1);
+#pragma unroll 1
+  for (int n = 0; n < nn; ++n) {
+    if (cur.cell != kNoCell && cur.cell != ccell) {
+      ccell = cur.cell;
+      if (ABL != 1) refill(it, rs, cur.cell, st);
+      else { st[0][0][0] += 1.0; }
+    }
+    const NodeRec& nd = S.node[n];
+    double f0, f1, f2;
+    Geo nxt;
+    if (n + 1 < nn && ((fullmask >> (n + 1)) & 1)) {
+      nxt = geom_point<true, ABL>(P, S, trf, e, n + 1, N, wfull, third, inv_n1);
+      contract_point(cur, nd, st, f0, f1, f2);
+    } else if (n + 1 < nn) {
+      nxt = geom_point<false, ABL>(P, S, trf, e, n + 1, N, wfull, third, inv_n1);
+      contract_point(cur, nd, st, f0, f1, f2);
+    } else {
+      nxt = cur;
+      contract_point(cur, nd, st, f0, f1, f2);
+    }
+    const double wk = cur.w * nd.wk;
+    k0 += wk * f0; k1 += wk * f1; k2 += wk * f2;
+    if ((n & 1) || P.rule == RP_RULE_SIMPSON) {  // G7: Gauss nodes only (warp-uniform n)
+      const double wg = cur.w * nd.wg;
+      g0 += wg * f0; g1 += wg * f1; g2 += wg * f2;
+    }
+    cur = nxt;
+  }
+}
+
 __device__ __forceinline__ double warp_sum(double v) {
 #pragma unroll
   for (int o = 16; o > 0; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);
   return v;
 }
 
-template <int KIND>
+__device__ unsigned long long g_phase[8];  // development: per-phase SM cycles (VAR 7)
+
+// VAR 0: one pass per round (eval_nodes); VAR 4: software-pipelined rounds; VAR 7: VAR 4 with
+// per-phase clock accounting (development)
+template <int KIND, int VAR>
 __global__ void __launch_bounds__(32 * kWarps) k_integrate(
     Params P, const int32_t* __restrict__ order, const double2* __restrict__ AB,
     const double2* __restrict__ trig_full, double4* __restrict__ item_val,
     int4* __restrict__ item_cnt, uint2* __restrict__ item_aux,
     unsigned long long* __restrict__ counters) {
-  __shared__ WarpSmem smem[kWarps];
+  extern __shared__ __align__(16) unsigned char smem_raw[];
+  WarpSmem* smem = reinterpret_cast<WarpSmem*>(smem_raw);
   const int lane = threadIdx.x & 31;
   WarpSmem& S = smem[threadIdx.x >> 5];
   const unsigned long long n_items = counters[C_ITEMS];
@@ -573,6 +739,9 @@ __global__ void __launch_bounds__(32 * kWarps) k_integrate(
   const double Nd = (double)N;
   const double wfull = kTwoPi / Nd;
   const double third = 1.0 / 3.0;
+  constexpr bool TM = VAR == 7;
+  unsigned long long ph[6] = {0, 0, 0, 0, 0, 0};
+  long long t0 = TM ? clock64() : 0;
   for (;;) {
     unsigned long long idx = 0;
     if (lane == 0) idx = atomicAdd(&counters[C_NEXT], 1ULL);
@@ -590,9 +759,17 @@ __global__ void __launch_bounds__(32 * kWarps) k_integrate(
     double s_phi = 0.0, s_ax = 0.0, s_ay = 0.0, s_err = 0.0;
     double st[3][9][3];                      // per-lane stencil cache (valid for this item's levels)
     int cix = -1000000, ciy = -1000000;
+    int ccell = kNoCell;  // cached cell of the two-pass rounds (empty cache reads as zeros)
+    if (KIND == RP_SRC_GRID && VAR >= 4) {
+#pragma unroll
+      for (int l = 0; l < 3; ++l)
+#pragma unroll
+        for (int i = 0; i < 9; ++i) st[l][i][0] = st[l][i][1] = st[l][i][2] = 0.0;
+    }
     int nseg = 0, nleaf = 0, capped = 0, ties = 0, maxlev = 0;
     unsigned evals = 0;
     int lev = P.n_root == 2 ? 1 : 0;
+    if (TM) { long long t = clock64(); ph[0] += t - t0; t0 = t; }
     long long ix = 0;
     for (;;) {
       const double fa = ldexp((double)ix, -lev), fb = ldexp((double)(ix + 1), -lev);
@@ -632,6 +809,7 @@ __global__ void __launch_bounds__(32 * kWarps) k_integrate(
         }
         cnt = na < 0 ? N : na * (N + 1);
       }
+      if (TM) { __syncwarp(); long long t = clock64(); ph[1] += t - t0; t0 = t; }
       // inclusive scan of counts over lanes -> exclusive node offsets
       int incl = cnt;
 #pragma unroll
@@ -641,6 +819,8 @@ __global__ void __launch_bounds__(32 * kWarps) k_integrate(
       }
       if (lane < 16) S.cnt[lane] = lane < 15 ? cnt : 0;
       const int E = __shfl_sync(0xffffffffu, incl, 31);
+      // r' nodes whose circle lies wholly inside the support (warp-uniform bit per node)
+      const unsigned fullmask = __ballot_sync(0xffffffffu, lane < nn && cnt == N);
       __syncwarp();
       // ---- evaluation phase
       int emax = cnt;
@@ -653,16 +833,28 @@ __global__ void __launch_bounds__(32 * kWarps) k_integrate(
       // the previous (radially adjacent) segment.  Leftover slots (65-node arcs) go last as
       // (slot, node) units.
       const int rounds = emax >> 5, left = emax - 32 * rounds;
-      for (int rr = 0; rr < rounds; ++rr) {
-        const int r = (nseg & 1) ? rounds - 1 - rr : rr;
-        eval_nodes<KIND>(it, P, S, trig_full, 32 * r + lane, 0, nn, N, wfull, third, st, cix, ciy,
-                         k0, k1, k2, g0, g1, g2);
+      if (TM) { long long t = clock64(); ph[2] += t - t0; t0 = t; }
+      if (KIND == RP_SRC_GRID && VAR >= 4) {
+        for (int rr = 0; rr < rounds; ++rr) {
+          const int r = (nseg & 1) ? rounds - 1 - rr : rr;
+          pipelined_round<VAR == 7 ? 0 : VAR - 4>(it, P, S, trig_full, 32 * r + lane, nn, N,
+                                                   wfull, third, st, ccell, k0, k1, k2, g0, g1,
+                                                   g2, fullmask);
+        }
+      } else {
+        for (int rr = 0; rr < rounds; ++rr) {
+          const int r = (nseg & 1) ? rounds - 1 - rr : rr;
+          eval_nodes<KIND>(it, P, S, trig_full, 32 * r + lane, 0, nn, N, wfull, third, st, cix,
+                           ciy, k0, k1, k2, g0, g1, g2);
+        }
       }
+      if (TM) { __syncwarp(); long long t = clock64(); ph[3] += t - t0; t0 = t; }
       for (int u = lane; u < nn * left; u += 32) {
         const int e = 32 * rounds + u / nn, n = u - nn * (u / nn);
         eval_nodes<KIND, false>(it, P, S, trig_full, e, n, n + 1, N, wfull, third, st, cix, ciy,
                                 k0, k1, k2, g0, g1, g2);
       }
+      if (TM) { __syncwarp(); long long t = clock64(); ph[4] += t - t0; t0 = t; }
       k0 = warp_sum(k0); k1 = warp_sum(k1); k2 = warp_sum(k2);
       g0 = warp_sum(g0); g1 = warp_sum(g1); g2 = warp_sum(g2);
       __syncwarp();
@@ -685,6 +877,7 @@ __global__ void __launch_bounds__(32 * kWarps) k_integrate(
         ++lev;
         ix <<= 1;
       }
+      if (TM) { long long t = clock64(); ph[5] += t - t0; t0 = t; }
     }
     if (lane == 0) {
       item_val[item] = make_double4(s_phi, s_ax, s_ay, s_err);
@@ -692,6 +885,8 @@ __global__ void __launch_bounds__(32 * kWarps) k_integrate(
       item_aux[item] = make_uint2((unsigned)maxlev, evals);
     }
   }
+  if (TM && lane == 0)
+    for (int i = 0; i < 6; ++i) atomicAdd(&g_phase[i], ph[i]);
 }
 
 // ------------------------------------------------------------- k_reduce
@@ -824,6 +1019,23 @@ int rp_alloc_potential_scratch(rp_ctx* ctx) {
   return RP_OK;
 }
 
+template <int KIND, int VAR>
+static int launch_integrate(rp_ctx* ctx, const Params& P) {
+  int occ = 0;
+  const size_t smem = sizeof(WarpSmem) * kWarps;
+  RP_CUDA(cudaFuncSetAttribute(k_integrate<KIND, VAR>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                               (int)smem));
+  RP_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_integrate<KIND, VAR>, 32 * kWarps,
+                                                        smem));
+  if (occ < 1) occ = 1;
+  ProfScope ps(ctx, PK_INTEGRATE);
+  k_integrate<KIND, VAR><<<ctx->sm_count * occ, 32 * kWarps, smem, ctx->stream>>>(
+      P, ctx->sched_order, ctx->clipAB, ctx->trig_full, ctx->item_val, ctx->item_cnt,
+      ctx->item_aux, ctx->counters);
+  RP_CHECK_LAUNCH();
+  return RP_OK;
+}
+
 template <int KIND>
 static int run_potentials(rp_ctx* ctx, const Params& P, int32_t rank, int32_t world,
                           double* phi, double* ax, double* ay, double* err, int32_t* nseg,
@@ -877,16 +1089,13 @@ static int run_potentials(rp_ctx* ctx, const Params& P, int32_t rank, int32_t wo
                                               ctx->sched_key_sorted, ctx->sched_idx,
                                               ctx->sched_order, (int)nd, 0, 16, st));
     }
-    int occ = 0;
-    RP_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_integrate<KIND>, 32 * kWarps, 0));
-    if (occ < 1) occ = 1;
-    {
-      ProfScope ps(ctx, PK_INTEGRATE);
-      k_integrate<KIND><<<ctx->sm_count * occ, 32 * kWarps, 0, st>>>(
-          P, ctx->sched_order, ctx->clipAB, ctx->trig_full, ctx->item_val, ctx->item_cnt,
-          ctx->item_aux, ctx->counters);
-      RP_CHECK_LAUNCH();
-    }
+    const int var = KIND == RP_SRC_GRID ? ctx->eval_variant : 0;
+    int rc2 = var == 4 ? launch_integrate<KIND, 4>(ctx, P)
+              : var == 5 ? launch_integrate<KIND, 5>(ctx, P)
+              : var == 6 ? launch_integrate<KIND, 6>(ctx, P)
+              : var == 7 ? launch_integrate<KIND, 7>(ctx, P)
+                         : launch_integrate<KIND, 0>(ctx, P);
+    if (rc2) return rc2;
   }
   ProfScope ps_red(ctx, PK_REDUCE);
   k_reduce<<<(P.npts + 255) / 256, 256, 0, st>>>(
@@ -908,6 +1117,7 @@ int rp_potentials_impl(rp_ctx* ctx, int kind, const double src[6], int32_t rank,
   P.nx = c.nx; P.ny = c.ny; P.PX = ctx->PX; P.npts = c.nx * c.ny; P.kmax = c.history_depth;
   P.kap = kappa_of(ctx); P.k = ctx->k; P.H = ctx->H; P.n_theta = c.n_theta;
   P.max_depth = c.max_depth; P.n_root = c.n_root; P.rule = c.outer_rule;
+  P.variant = ctx->eval_variant;
   P.hx = c.hx; P.hy = c.hy; P.inv_hx = 1.0 / c.hx; P.inv_hy = 1.0 / c.hy;
   P.cdt = c.c * c.dt; P.tau = c.tau; P.R = (double)P.kap * P.cdt;
   P.slot_doubles = ctx->slot_doubles; P.ring = ctx->ring; P.frames = ctx->frames_dev;
@@ -953,4 +1163,14 @@ int rp_scatter_impl(rp_ctx* ctx, const double* shards, int32_t world, int64_t ca
   RP_CHECK_LAUNCH();
   ctx->has_forecast = 1;
   return RP_OK;
+}
+
+// development only (not in rp.h): per-phase SM cycles accumulated by k_integrate VAR 7
+extern "C" int rp_dev_phase_cycles(unsigned long long* out, int reset) {
+  if (cudaMemcpyFromSymbol(out, g_phase, sizeof(unsigned long long) * 6) != cudaSuccess) return -3;
+  if (reset) {
+    unsigned long long z[8] = {0};
+    cudaMemcpyToSymbol(g_phase, z, sizeof(z));
+  }
+  return 0;
 }

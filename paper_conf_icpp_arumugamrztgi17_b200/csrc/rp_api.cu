@@ -1,3 +1,4 @@
+#include <stdlib.h>
 // rp_api.cu -- the C ABI of librp (include/rp.h): context, history ring, state access and
 // the argument checking around the kernels of deposit.cu, potentials.cu, fields_push.cu.
 #include <new>
@@ -151,6 +152,7 @@ int rp_create(const rp_config* cfg, rp_ctx** out) {
   };
   if (cudaSetDevice(cfg->device) != cudaSuccess) return fail(RP_ENODEV);
   cudaDeviceGetAttribute(&ctx->sm_count, cudaDevAttrMultiProcessorCount, cfg->device);
+  if (const char* ev = getenv("RP_EVAL")) ctx->eval_variant = atoi(ev);
   ctx->H = cfg->history_depth + 2;
   ctx->PX = cfg->nx + 2 * RP_PAD;
   ctx->PY = cfg->ny + 2 * RP_PAD;

@@ -61,6 +61,7 @@ struct rp_ctx {
   int has_forecast = 0;
   int sched_policy = 1;             // RP_SCHED_*
   int sched_k = 9;                  // kNN neighbours
+  int eval_variant = 4;             // integrator evaluation loop (development A/B: RP_EVAL)
 
   // sharding scratch
   int32_t* point_key = nullptr;     // per point predicted work key

@@ -1,0 +1,55 @@
+"""Development A/B of integrator evaluation loops (RP_EVAL=<v> selects one at rp_create).
+
+Runs `steps` steps of a config per variant in one process, checks that every variant's
+potentials / segment counts are bit-identical to the first one's, and prints the integrator's
+CUDA-event time per step.  usage: python tools/ab_eval.py [config] [steps] [variants...]
+"""
+import os
+import sys
+
+import numpy as np
+import torch
+
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+import workloads as W  # noqa: E402
+from paper_conf_icpp_arumugamrztgi17_b200 import rp  # noqa: E402
+from paper_conf_icpp_arumugamrztgi17_b200.sim import Simulation  # noqa: E402
+
+cfgn = int(sys.argv[1]) if len(sys.argv) > 1 else 2
+steps = int(sys.argv[2]) if len(sys.argv) > 2 else 4
+variants = [int(v) for v in sys.argv[3:]] or [0, 1]
+cfg = W.config(cfgn)
+ref = None
+for v in variants:
+    os.environ["RP_EVAL"] = str(v)
+    sim = Simulation(cfg)
+    rp.rp_profile_enable(sim.ctx, True)
+    outs, ms, ev, last = [], [], [], 0.0
+    for s in range(steps):
+        info = sim.step(info=True)
+        torch.cuda.synchronize()
+        prof = rp.rp_profile_read(sim.ctx)
+        ms.append(prof.integrate_ms - last)
+        last = prof.integrate_ms
+        ev.append(info.evals)
+        outs.append([t.cpu().numpy().copy() for t in (sim.phi, sim.ax, sim.ay, sim.nseg)])
+    if v == 7:
+        import ctypes
+        buf = (ctypes.c_ulonglong * 6)()
+        rp._lib.rp_dev_phase_cycles(buf, 1)
+        tot = sum(buf)
+        names = ["item", "nodes", "scan", "rounds", "leftover", "tail"]
+        print("phase cycles (all steps, warp-summed):",
+              {n: f"{100 * b / tot:.1f}%" for n, b in zip(names, buf)}, flush=True)
+    sim.close()
+    same = None
+    if ref is None:
+        ref = outs
+    else:
+        same = all(np.array_equal(a.view(np.uint8) if a.dtype != np.int32 else a,
+                                  b.view(np.uint8) if b.dtype != np.int32 else b)
+                   for oa, ob in zip(outs, ref) for a, b in zip(oa, ob))
+    print(f"variant {v}: integrate ms/step {[round(x, 2) for x in ms]} "
+          f"(steps 2+: {np.mean(ms[2:]) if len(ms) > 2 else np.mean(ms):.2f}); "
+          f"ps/eval {[round(1e9 * m / e, 2) for m, e in zip(ms, ev)]}; "
+          f"evals {info.evals}; bit-identical to first: {same}", flush=True)
