@@ -40,7 +40,10 @@ F_SEG = 60     # one GK15 segment: K15/G7 sums, error, decision
 
 
 def algorithmic_flops(info: dict) -> float:
-    return info["evals"] * F_EVAL + info["nodes"] * F_NODE + info["segments"] * F_SEG
+    # evaluations performed: the rules' integrand nodes minus the arc end nodes on the support
+    # boundary, where the integrand vanishes and the GPU path skips them (DESIGN R-24)
+    performed = info["evals"] - info.get("skipped", 0)
+    return performed * F_EVAL + info["nodes"] * F_NODE + info["segments"] * F_SEG
 
 
 def measured_peaks():
@@ -182,7 +185,7 @@ def run_ours(args):
     clocks.start()
     barrier()
     step_ms = []
-    totals = {"evals": 0, "nodes": 0, "segments": 0, "capped": 0, "items": 0}
+    totals = {"evals": 0, "skipped": 0, "nodes": 0, "segments": 0, "capped": 0, "items": 0}
     for _ in range(args.steps):
         flush.fill_(1.0)  # evict L2 between timed steps (outside the events)
         e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)

@@ -76,7 +76,7 @@ typedef struct {
 } rp_deposit_info;
 
 typedef struct {
-  int64_t evals;           /* integrand evaluations f(r', theta', t') (flop census)             */
+  int64_t evals;           /* integrand nodes f(r', theta', t') of the rules (as the oracle counts)*/
   int64_t nodes;           /* r' nodes (15 per GK15 segment)                                     */
   int64_t segments;        /* GK15 segments evaluated (sum of nseg)                              */
   int64_t leaves;          /* accepted segments                                                  */
@@ -85,6 +85,9 @@ typedef struct {
   int64_t items;           /* (point, subregion) pairs with support                              */
   int32_t max_level;       /* deepest tree level reached                                         */
   int32_t kappa;           /* subregions kappa(k) used at this step (R-3)                        */
+  int64_t skipped;         /* of `evals`, arc end nodes on the support boundary, where the zero-
+                              padded TSC integrand vanishes, not evaluated (DESIGN R-24); the
+                              evaluations performed are evals - skipped                         */
 } rp_potential_info;
 
 /* Create a context on cfg->device: allocates the HBM history ring of history_depth+2

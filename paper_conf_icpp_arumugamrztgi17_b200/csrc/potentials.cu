@@ -42,7 +42,7 @@ __constant__ double c_wg[4] = {
     0.381830050505118944950369775488975, 0.417959183673469387755102040816327};
 
 enum : int { C_ITEMS = 0, C_NEXT = 1, C_EVALS = 2, C_SEGS = 3, C_LEAVES = 4, C_CAPPED = 5,
-             C_TIES = 6, C_MAXLEV = 7, C_NODES = 8, C_NOUT = 9, C_COUNT = 16 };
+             C_TIES = 6, C_MAXLEV = 7, C_NODES = 8, C_NOUT = 9, C_SKIP = 10, C_COUNT = 16 };
 
 constexpr double kTwoPi = 6.283185307179586476925286766559;
 constexpr int kMaxArcs = 8;
@@ -576,7 +576,7 @@ struct Geo {
 };
 
 // Branch-free geometry of theta slot e of r' node n (FULL: full circle, uniform per node).
-template <bool FULL, int ABL = 0>
+template <bool FULL>
 __device__ __forceinline__ Geo geom_point(const Params& P, const WarpSmem& S, double2 trf, int e,
                                           int n, int N, double wfull, double third,
                                           float inv_n1) {
@@ -587,14 +587,14 @@ __device__ __forceinline__ Geo geom_point(const Params& P, const WarpSmem& S, do
     sn = trf.y;
     w = wfull;
   } else {
+    // slot e -> arc q, interior Simpson node mm = 1 .. N-1: the end nodes mm = 0, N of an arc
+    // lie on the support boundary, where the zero-padded TSC stencil vanishes (R-24)
     const int ec = valid ? e : 0;
     const int q = __float2int_rz(((float)ec + 0.5f) * inv_n1);  // arc index, exact for e < 2^20
-    const int mm = ec - q * (N + 1);
+    const int mm = ec - q * (N - 1) + 1;
     const double d = S.dth[n][q];
-    if (ABL == 2) { const double a = S.th1[n][q] + (double)mm * d; cs = 1.0 - 0.5 * a * a; sn = a; }
-    else sincos_b(S.th1[n][q] + (double)mm * d, &sn, &cs);
-    const double coef = (mm == 0 || mm == N) ? 1.0 : ((mm & 1) ? 4.0 : 2.0);
-    w = coef * d * third;
+    sincos_b(S.th1[n][q] + (double)mm * d, &sn, &cs);
+    w = ((mm & 1) ? 4.0 : 2.0) * d * third;
   }
   const NodeRec& nd = S.node[n];
   const double u = nd.cu + nd.r * cs, v = nd.cv + nd.r * sn;
@@ -625,25 +625,6 @@ __device__ __forceinline__ void refill(const Item& it, size_t rs, int cell,
     }
 }
 
-// L1 prefetch of the stencil rows of `cell` when it differs from the cell in use (predicated,
-// branch-free: it sits inside the interleaved geometry/contraction block).  A row of 3 nodes
-// (96 B) spans at most two 128-B lines: prefetch its first and last byte.
-__device__ __forceinline__ void prefetch_cell(const Item& it, size_t rs, int cell, int cur) {
-  const int p = (cell != kNoCell && cell != cur) ? 1 : 0;
-  const size_t base = (size_t)4 * (ptrdiff_t)(p ? cell : 0);
-  const double* g[3] = {it.g0 + base, it.g1 + base, it.g2 + base};
-#pragma unroll
-  for (int l = 0; l < 3; ++l)
-#pragma unroll
-    for (int b = 0; b < 3; ++b) {
-      const double* row = g[l] + b * rs;
-      asm volatile(
-          "{\n\t.reg .pred q;\n\tsetp.ne.s32 q, %2, 0;\n\t"
-          "@q prefetch.global.L1 [%0];\n\t@q prefetch.global.L1 [%1];\n\t}" ::"l"(row),
-          "l"(row + 11), "r"(p));
-    }
-}
-
 // 27-node x 3-component contraction at one point -> (f0, f1, f2)
 __device__ __forceinline__ void contract_point(const Geo& g, const NodeRec& nd,
                                                const double (&st)[3][9][3], double& f0,
@@ -671,7 +652,6 @@ __device__ __forceinline__ void contract_point(const Geo& g, const NodeRec& nd,
   f2 = nd.w0 * s[0][2] + nd.w1 * s[1][2] + nd.w2 * s[2][2];
 }
 
-template <int ABL>
 __device__ __forceinline__ void pipelined_round(const Item& it, const Params& P,
                                                 const WarpSmem& S,
                                                 const double2* __restrict__ trig_full, int e,
@@ -680,25 +660,24 @@ __device__ __forceinline__ void pipelined_round(const Item& it, const Params& P,
                                                 double& k1, double& k2, double& g0, double& g1,
                                                 double& g2, unsigned fullmask) {
   const size_t rs = (size_t)4 * P.PX;
-  const float inv_n1 = 1.0f / (float)(N + 1);
+  const float inv_n1 = 1.0f / (float)(N - 1);  // interior nodes per arc (R-24)
   const double2 trf = __ldg(trig_full + (e < N ? e : 0));
-  Geo cur = (fullmask & 1) ? geom_point<true, ABL>(P, S, trf, e, 0, N, wfull, third, inv_n1)
-                        : geom_point<false, ABL>(P, S, trf, e, 0, N, wfull, third, inv_n1);
+  Geo cur = (fullmask & 1) ? geom_point<true>(P, S, trf, e, 0, N, wfull, third, inv_n1)
+                        : geom_point<false>(P, S, trf, e, 0, N, wfull, third, inv_n1);
 #pragma unroll 1
   for (int n = 0; n < nn; ++n) {
     if (cur.cell != kNoCell && cur.cell != ccell) {
       ccell = cur.cell;
-      if (ABL != 1) refill(it, rs, cur.cell, st);
-      else { st[0][0][0] += 1.0; }
+      refill(it, rs, cur.cell, st);
     }
     const NodeRec& nd = S.node[n];
     double f0, f1, f2;
     Geo nxt;
     if (n + 1 < nn && ((fullmask >> (n + 1)) & 1)) {
-      nxt = geom_point<true, ABL>(P, S, trf, e, n + 1, N, wfull, third, inv_n1);
+      nxt = geom_point<true>(P, S, trf, e, n + 1, N, wfull, third, inv_n1);
       contract_point(cur, nd, st, f0, f1, f2);
     } else if (n + 1 < nn) {
-      nxt = geom_point<false, ABL>(P, S, trf, e, n + 1, N, wfull, third, inv_n1);
+      nxt = geom_point<false>(P, S, trf, e, n + 1, N, wfull, third, inv_n1);
       contract_point(cur, nd, st, f0, f1, f2);
     } else {
       nxt = cur;
@@ -767,7 +746,7 @@ __global__ void __launch_bounds__(32 * kWarps) k_integrate(
         for (int i = 0; i < 9; ++i) st[l][i][0] = st[l][i][1] = st[l][i][2] = 0.0;
     }
     int nseg = 0, nleaf = 0, capped = 0, ties = 0, maxlev = 0;
-    unsigned evals = 0;
+    unsigned evals = 0, nskip = 0;
     int lev = P.n_root == 2 ? 1 : 0;
     if (TM) { long long t = clock64(); ph[0] += t - t0; t0 = t; }
     long long ix = 0;
@@ -776,7 +755,8 @@ __global__ void __launch_bounds__(32 * kWarps) k_integrate(
       const double a = __dadd_rn(A, __dmul_rn(BA, fa)), b = __dadd_rn(A, __dmul_rn(BA, fb));
       const double m = __dmul_rn(0.5, __dadd_rn(a, b)), hw = __dmul_rn(0.5, __dsub_rn(b, a));
       // ---- node phase: lanes 0..14 build the r' nodes of the GK15 rule
-      int cnt = 0;
+      int cnt = 0, skip = 0;
+      bool full = false;
       const int nn = P.rule == RP_RULE_SIMPSON ? 5 : 15;  // r' nodes per segment
       if (lane < nn) {
         const int i = lane < 7 ? lane : (lane == 7 ? 7 : 14 - lane);
@@ -808,6 +788,11 @@ __global__ void __launch_bounds__(32 * kWarps) k_integrate(
           S.dth[lane][q] = dth[q];
         }
         cnt = na < 0 ? N : na * (N + 1);
+        full = na < 0;
+        if (KIND == RP_SRC_GRID && VAR >= 4 && na > 0) {  // interior arc nodes only (R-24)
+          skip = 2 * na;
+          cnt = na * (N - 1);
+        }
       }
       if (TM) { __syncwarp(); long long t = clock64(); ph[1] += t - t0; t0 = t; }
       // inclusive scan of counts over lanes -> exclusive node offsets
@@ -818,9 +803,12 @@ __global__ void __launch_bounds__(32 * kWarps) k_integrate(
         if (lane >= o) incl += y;
       }
       if (lane < 16) S.cnt[lane] = lane < 15 ? cnt : 0;
-      const int E = __shfl_sync(0xffffffffu, incl, 31);
+      int skipped = skip;  // arc end nodes known to vanish (not evaluated)
+#pragma unroll
+      for (int o = 16; o > 0; o >>= 1) skipped += __shfl_xor_sync(0xffffffffu, skipped, o);
+      const int E = __shfl_sync(0xffffffffu, incl, 31) + skipped;  // integrand nodes of the rule
       // r' nodes whose circle lies wholly inside the support (warp-uniform bit per node)
-      const unsigned fullmask = __ballot_sync(0xffffffffu, lane < nn && cnt == N);
+      const unsigned fullmask = __ballot_sync(0xffffffffu, lane < nn && full);
       __syncwarp();
       // ---- evaluation phase
       int emax = cnt;
@@ -832,12 +820,15 @@ __global__ void __launch_bounds__(32 * kWarps) k_integrate(
       // to segment, so the first round of a segment finds the cell left by the last round of
       // the previous (radially adjacent) segment.  Leftover slots (65-node arcs) go last as
       // (slot, node) units.
-      const int rounds = emax >> 5, left = emax - 32 * rounds;
+      // grid path: whole rounds (at most 2 idle slots per arc); otherwise leftover (slot, node)
+      // units after the full rounds
+      const int rounds = (KIND == RP_SRC_GRID && VAR >= 4) ? (emax + 31) >> 5 : emax >> 5;
+      const int left = (KIND == RP_SRC_GRID && VAR >= 4) ? 0 : emax - 32 * rounds;
       if (TM) { long long t = clock64(); ph[2] += t - t0; t0 = t; }
       if (KIND == RP_SRC_GRID && VAR >= 4) {
         for (int rr = 0; rr < rounds; ++rr) {
           const int r = (nseg & 1) ? rounds - 1 - rr : rr;
-          pipelined_round<VAR == 7 ? 0 : VAR - 4>(it, P, S, trig_full, 32 * r + lane, nn, N,
+          pipelined_round(it, P, S, trig_full, 32 * r + lane, nn, N,
                                                    wfull, third, st, ccell, k0, k1, k2, g0, g1,
                                                    g2, fullmask);
         }
@@ -859,6 +850,7 @@ __global__ void __launch_bounds__(32 * kWarps) k_integrate(
       g0 = warp_sum(g0); g1 = warp_sum(g1); g2 = warp_sum(g2);
       __syncwarp();
       evals += (unsigned)E;
+      nskip += (unsigned)skipped;
       ++nseg;
       if (lev > maxlev) maxlev = lev;
       double err = fabs(k0 - g0);
@@ -883,6 +875,7 @@ __global__ void __launch_bounds__(32 * kWarps) k_integrate(
       item_val[item] = make_double4(s_phi, s_ax, s_ay, s_err);
       item_cnt[item] = make_int4(nseg, nleaf, capped, ties);
       item_aux[item] = make_uint2((unsigned)maxlev, evals);
+      if (nskip) atomicAdd(&counters[C_SKIP], (unsigned long long)nskip);
     }
   }
   if (TM && lane == 0)
@@ -1091,8 +1084,6 @@ static int run_potentials(rp_ctx* ctx, const Params& P, int32_t rank, int32_t wo
     }
     const int var = KIND == RP_SRC_GRID ? ctx->eval_variant : 0;
     int rc2 = var == 4 ? launch_integrate<KIND, 4>(ctx, P)
-              : var == 5 ? launch_integrate<KIND, 5>(ctx, P)
-              : var == 6 ? launch_integrate<KIND, 6>(ctx, P)
               : var == 7 ? launch_integrate<KIND, 7>(ctx, P)
                          : launch_integrate<KIND, 0>(ctx, P);
     if (rc2) return rc2;
@@ -1146,6 +1137,7 @@ int rp_potentials_impl(rp_ctx* ctx, int kind, const double src[6], int32_t rank,
       info->ties = (int64_t)h[C_TIES];
       info->max_level = (int32_t)h[C_MAXLEV];
       info->kappa = P.kap;
+      info->skipped = (int64_t)h[C_SKIP];
     }
     if (n_out) *n_out = (int64_t)h[C_NOUT];
   }

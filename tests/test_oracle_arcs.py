@@ -141,3 +141,32 @@ def test_static_clip_closed_form():
             else:
                 assert clip is not None
                 assert abs(clip[0] - A) < 1e-13 and abs(clip[1] - B) < 1e-13
+
+
+def test_integrand_vanishes_at_arc_ends():
+    """R-24: the end nodes of every arc lie on the support rectangle [-1.5h, (N+0.5)h]^2,
+    where every node of the zero-padded 3x3 TSC stencil is outside the grid or has weight
+    0, so the integrand there is 0 up to the rounding of the crossing angle.  (The GPU path
+    skips these nodes; the oracle evaluates them.)"""
+    rng = np.random.default_rng(24)
+    nx, ny, hx, hy = 12, 9, 0.7, 0.45
+    kmax = 2
+    H = kmax + 2
+    ring = rng.uniform(0.5, 1.5, size=(H, ny, nx, 4))
+    ring[..., 3] = 0.0
+    P = oracle.Problem(nx=nx, ny=ny, hx=hx, hy=hy, c=1.0, dt=1.0, tau=1e-6, kappa_max=kmax,
+                       k=2, n_pre=0, ring=ring)
+    U0, U1, V0, V1 = -1.5 * hx, (nx + 0.5) * hx, -1.5 * hy, (ny + 0.5) * hy
+    scale = float(np.abs(ring).max())
+    n_ends = 0
+    for _ in range(400):
+        cu, cv = rng.uniform(-3, 11), rng.uniform(-3, 7)
+        r = rng.uniform(0.1, 9.0)
+        n, arcs = oracle.arcs_rect(cu, cv, r, U0, U1, V0, V1)
+        for t1, t2 in (arcs if n > 0 else []):
+            for t in (t1, t2):
+                u, v = cu + r * math.cos(t), cv + r * math.sin(t)
+                f = P.integrand(0, u, v, rng.uniform(0.0, 1.0))
+                assert np.all(np.abs(f) <= 1e-20 * scale), (cu, cv, r, t, f)
+                n_ends += 1
+    assert n_ends > 200
