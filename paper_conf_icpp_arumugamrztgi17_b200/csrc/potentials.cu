@@ -46,7 +46,8 @@ enum : int { C_ITEMS = 0, C_NEXT = 1, C_EVALS = 2, C_SEGS = 3, C_LEAVES = 4, C_C
 
 constexpr double kTwoPi = 6.283185307179586476925286766559;
 constexpr int kMaxArcs = 8;
-constexpr int kWarps = 4;  // warps per CTA of k_integrate
+constexpr int kWarps = 1;  // warps per CTA of k_integrate (1: the warp's shared block sits at
+                            // a constant address, no per-iteration warp-index arithmetic)
 
 struct Params {
   int nx, ny, PX, npts, kmax, kap, k, H, n_theta, max_depth, n_root, rule, variant;
@@ -712,7 +713,7 @@ __global__ void __launch_bounds__(32 * kWarps) k_integrate(
   extern __shared__ __align__(16) unsigned char smem_raw[];
   WarpSmem* smem = reinterpret_cast<WarpSmem*>(smem_raw);
   const int lane = threadIdx.x & 31;
-  WarpSmem& S = smem[threadIdx.x >> 5];
+  WarpSmem& S = smem[kWarps == 1 ? 0 : (threadIdx.x >> 5)];
   const unsigned long long n_items = counters[C_ITEMS];
   const int N = P.n_theta;
   const double Nd = (double)N;
@@ -795,33 +796,27 @@ __global__ void __launch_bounds__(32 * kWarps) k_integrate(
         }
       }
       if (TM) { __syncwarp(); long long t = clock64(); ph[1] += t - t0; t0 = t; }
-      // inclusive scan of counts over lanes -> exclusive node offsets
-      int incl = cnt;
-#pragma unroll
-      for (int o = 1; o < 32; o <<= 1) {
-        int y = __shfl_up_sync(0xffffffffu, incl, o);
-        if (lane >= o) incl += y;
-      }
+      // integrand nodes of the rules over the 15 r' nodes (E, including the skipped arc end
+      // nodes) and the largest per-node slot count (rounds): two independent butterflies
       if (lane < 16) S.cnt[lane] = lane < 15 ? cnt : 0;
-      int skipped = skip;  // arc end nodes known to vanish (not evaluated)
+      int E = cnt + skip, emax = cnt, skipped = skip;
 #pragma unroll
-      for (int o = 16; o > 0; o >>= 1) skipped += __shfl_xor_sync(0xffffffffu, skipped, o);
-      const int E = __shfl_sync(0xffffffffu, incl, 31) + skipped;  // integrand nodes of the rule
+      for (int o = 16; o > 0; o >>= 1) {
+        E += __shfl_xor_sync(0xffffffffu, E, o);
+        emax = max(emax, __shfl_xor_sync(0xffffffffu, emax, o));
+        skipped += __shfl_xor_sync(0xffffffffu, skipped, o);
+      }
       // r' nodes whose circle lies wholly inside the support (warp-uniform bit per node)
       const unsigned fullmask = __ballot_sync(0xffffffffu, lane < nn && full);
       __syncwarp();
       // ---- evaluation phase
-      int emax = cnt;
-#pragma unroll
-      for (int o = 16; o > 0; o >>= 1) emax = max(emax, __shfl_xor_sync(0xffffffffu, emax, o));
       double k0 = 0.0, k1 = 0.0, k2 = 0.0, g0 = 0.0, g1 = 0.0, g2 = 0.0;
-      // Lane <-> theta slot: full rounds of 32 slots, each lane running all 15 r' nodes of
-      // its slot with the register stencil cache.  The round order alternates from segment
-      // to segment, so the first round of a segment finds the cell left by the last round of
-      // the previous (radially adjacent) segment.  Leftover slots (65-node arcs) go last as
-      // (slot, node) units.
-      // grid path: whole rounds (at most 2 idle slots per arc); otherwise leftover (slot, node)
-      // units after the full rounds
+      // Lane <-> theta slot: rounds of 32 slots, each lane running all 15 r' nodes of its slot
+      // with the register stencil cache.  The round order alternates from segment to segment,
+      // so the first round of a segment finds the cell left by the last round of the previous
+      // (radially adjacent) segment.  Grid path: whole rounds (arc end nodes skipped, R-24: at
+      // most 2 idle slots per arc); analytic sources: full rounds, then the leftover slots of
+      // 65-node arcs as (slot, node) units.
       const int rounds = (KIND == RP_SRC_GRID && VAR >= 4) ? (emax + 31) >> 5 : emax >> 5;
       const int left = (KIND == RP_SRC_GRID && VAR >= 4) ? 0 : emax - 32 * rounds;
       if (TM) { long long t = clock64(); ph[2] += t - t0; t0 = t; }
