@@ -161,6 +161,7 @@ def run_ours(args):
         group = dist.group.WORLD
     cfg = W.config(args.config)
     cfg.rule = 1 if args.rule == "simpson" else 0
+    cfg.interp = 1 if args.interp == "lagrange3" else 0
     sim = Simulation(cfg, group=group)
     sched = args.schedule
     if sched == "index":
@@ -249,7 +250,8 @@ def run_ours(args):
                        "tau": cfg.tau, "n_theta": cfg.n_theta, "n_root": cfg.n_root,
                        "parallelism": f"mesh-point shards x{world}, history replicated",
                        "l2": "flushed between timed steps (512 MB write)",
-                       "schedule": args.schedule, "outer_rule": args.rule},
+                       "schedule": args.schedule, "outer_rule": args.rule,
+                       "interp": args.interp},
             "fp64_gflops": gflops,
             "work_per_step": {k2: v / args.steps for k2, v in totals.items()},
             "roofline": {"kernel": "k_integrate (GK15 tree integrator)", "bound": "alu",
@@ -324,7 +326,8 @@ def run_e2e(cfg, args, dev):
     npts = cfg.nx * cfg.ny
     mesh = torch.zeros((6, npts), dtype=torch.float64).pin_memory()
     ctx = rp.rp_create(cfg.nx, cfg.ny, cfg.hx, cfg.hy, cfg.kappa_max, cfg.c, cfg.dt, cfg.tau,
-                       cfg.n_theta, cfg.max_depth, cfg.n_root, dev.index or 0)
+                       cfg.n_theta, cfg.max_depth, cfg.n_root, dev.index or 0, cfg.rule,
+                       cfg.interp)
     try:
         stream = torch.cuda.current_stream()
         rp.rp_set_stream(ctx, stream)
@@ -442,6 +445,8 @@ def main():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--rule", default="gk15", choices=["gk15", "simpson"],
                     help="outer segment rule (simpson = the paper's RP-QUADRULE, a variant)")
+    ap.add_argument("--interp", default="tsc", choices=["tsc", "lagrange3"],
+                    help="spatial part of the 27-point stencil (lagrange3 = variant R-25)")
     ap.add_argument("--schedule", default="persistence",
                     help="work-order forecast: index | persistence | knn5 | knn9 | knn25")
     args = ap.parse_args()

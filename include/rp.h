@@ -65,10 +65,15 @@ typedef struct {
   int32_t device;          /* CUDA ordinal                                                       */
   int32_t outer_rule;      /* RP_RULE_GK15 (default, R-8) or RP_RULE_SIMPSON: the paper's own   */
                            /* rule (P:155 RP-QUADRULE), Boole value + |S2 - S1|/15 estimate (R-22) */
+  int32_t interp;          /* spatial part of the "27 neighbouring points": RP_INTERP_TSC */
+                           /* (default, R-6) or RP_INTERP_LAGRANGE3 (tri-quadratic Lagrange with  */
+                           /* the time interpolation, R-25; discontinuous across cells)          */
 } rp_config;
 
 #define RP_RULE_GK15 0
 #define RP_RULE_SIMPSON 1
+#define RP_INTERP_TSC 0
+#define RP_INTERP_LAGRANGE3 1
 
 typedef struct {
   int64_t n_lost;          /* particles whose 3x3 stencil leaves the grid (R-14)                 */

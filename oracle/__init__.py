@@ -43,7 +43,7 @@ class Params(C.Structure):
     _fields_ = [("nx", C.c_int32), ("ny", C.c_int32), ("hx", C.c_double), ("hy", C.c_double),
                 ("c", C.c_double), ("dt", C.c_double), ("tau", C.c_double),
                 ("n_theta", C.c_int32), ("max_depth", C.c_int32), ("n_root", C.c_int32),
-                ("kappa_max", C.c_int32), ("rule", C.c_int32)]
+                ("kappa_max", C.c_int32), ("rule", C.c_int32), ("interp", C.c_int32)]
 
 
 class Hist(C.Structure):
@@ -129,10 +129,10 @@ class Problem:
     def __init__(self, *, nx, ny, hx, hy, c, dt, tau, kappa_max, k, n_pre,
                  ring=None, frames=None, n_theta=64, max_depth=30, n_root=2,
                  source=SRC_GRID, x0=0.0, y0=0.0, width=1.0, q=1.0, bx=0.0, by=0.0, amp=None,
-                 rule=0):
+                 rule=0, interp=0):
         H = kappa_max + 2
         self.params = Params(nx, ny, hx, hy, c, dt, tau, n_theta, max_depth, n_root, kappa_max,
-                             rule)
+                             rule, interp)
         self.ring = None if ring is None else np.ascontiguousarray(ring, dtype=np.float64)
         if self.ring is not None:
             assert self.ring.shape == (H, ny, nx, 4), self.ring.shape

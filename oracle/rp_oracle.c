@@ -50,6 +50,7 @@ typedef struct {
   int32_t n_root;    /* 2: start from both halves of [A,B]; 1: from [A,B]   */
   int32_t kappa_max; /* history depth (R-4)                                  */
   int32_t rule;      /* outer segment rule: 0 = GK15 (R-8), 1 = Simpson/Boole (R-22) */
+  int32_t interp;    /* spatial weights: 0 = TSC (R-6), 1 = quadratic Lagrange (R-25)  */
 } orc_params;
 
 typedef struct {
@@ -417,8 +418,13 @@ static void integrand(const subctx* X, double u, double v, const double* wt, dou
     double tx = u / P->hx, ty = v / P->hy;
     double fx = floor(tx + 0.5), fy = floor(ty + 0.5);
     double wx[3], wy[3];
-    orc_tsc_weights(tx - fx, wx);
-    orc_tsc_weights(ty - fy, wy);
+    if (P->interp == 1) { /* R-25: the time interpolation's quadratic Lagrange in x and y */
+      orc_lagrange3_weights(tx - fx, wx);
+      orc_lagrange3_weights(ty - fy, wy);
+    } else {
+      orc_tsc_weights(tx - fx, wx);
+      orc_tsc_weights(ty - fy, wy);
+    }
     /* clamp far-out indices before the int conversion (values are 0 there) */
     if (fx < -4.0 || fx > P->nx + 4.0 || fy < -4.0 || fy > P->ny + 4.0) {
       f[0] = f[1] = f[2] = 0.0;

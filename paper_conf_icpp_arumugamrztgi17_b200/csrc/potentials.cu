@@ -50,7 +50,7 @@ constexpr int kWarps = 1;  // warps per CTA of k_integrate (1: the warp's shared
                             // a constant address, no per-iteration warp-index arithmetic)
 
 struct Params {
-  int nx, ny, PX, npts, kmax, kap, k, H, n_theta, max_depth, n_root, rule, variant;
+  int nx, ny, PX, npts, kmax, kap, k, H, n_theta, max_depth, n_root, rule, variant, interp;
   double hx, hy, inv_hx, inv_hy, cdt, tau, R;
   size_t slot_doubles;
   const double* ring;        // padded ring, slot 0 node (-PAD, -PAD)
@@ -577,7 +577,7 @@ struct Geo {
 };
 
 // Branch-free geometry of theta slot e of r' node n (FULL: full circle, uniform per node).
-template <bool FULL>
+template <bool FULL, bool LAG>
 __device__ __forceinline__ Geo geom_point(const Params& P, const WarpSmem& S, double2 trf, int e,
                                           int n, int N, double wfull, double third,
                                           float inv_n1) {
@@ -590,12 +590,14 @@ __device__ __forceinline__ Geo geom_point(const Params& P, const WarpSmem& S, do
   } else {
     // slot e -> arc q, interior Simpson node mm = 1 .. N-1: the end nodes mm = 0, N of an arc
     // lie on the support boundary, where the zero-padded TSC stencil vanishes (R-24)
+    // (Lagrange-3, R-25: the integrand does not vanish there, all N+1 nodes are evaluated)
     const int ec = valid ? e : 0;
     const int q = __float2int_rz(((float)ec + 0.5f) * inv_n1);  // arc index, exact for e < 2^20
-    const int mm = ec - q * (N - 1) + 1;
+    const int mm = LAG ? ec - q * (N + 1) : ec - q * (N - 1) + 1;
     const double d = S.dth[n][q];
     sincos_b(S.th1[n][q] + (double)mm * d, &sn, &cs);
-    w = ((mm & 1) ? 4.0 : 2.0) * d * third;
+    const double coef = (LAG && (mm == 0 || mm == N)) ? 1.0 : ((mm & 1) ? 4.0 : 2.0);
+    w = coef * d * third;
   }
   const NodeRec& nd = S.node[n];
   const double u = nd.cu + nd.r * cs, v = nd.cv + nd.r * sn;
@@ -606,7 +608,7 @@ __device__ __forceinline__ Geo geom_point(const Params& P, const WarpSmem& S, do
   Geo g;
   g.dx = valid ? tx - fx : 0.0;
   g.dy = valid ? ty - fy : 0.0;
-  g.w = valid ? 0.25 * w : 0.0;  // 0.25 undoes the 2 x 2 scaling of the TSC weights
+  g.w = valid ? (LAG ? w : 0.25 * w) : 0.0;  // 0.25 undoes the 2 x 2 scaling of the TSC weights
   g.cell = valid ? (iy - 1) * P.PX + (ix - 1) : kNoCell;
   return g;
 }
@@ -627,13 +629,21 @@ __device__ __forceinline__ void refill(const Item& it, size_t rs, int cell,
 }
 
 // 27-node x 3-component contraction at one point -> (f0, f1, f2)
+template <bool LAG>
 __device__ __forceinline__ void contract_point(const Geo& g, const NodeRec& nd,
                                                const double (&st)[3][9][3], double& f0,
                                                double& f1, double& f2) {
   const double dx = g.dx, dy = g.dy;
-  const double ax = 0.5 - dx, bx = 0.5 + dx, ay = 0.5 - dy, by = 0.5 + dy;
-  const double wx[3] = {ax * ax, fma(-2.0 * dx, dx, 1.5), bx * bx};
-  const double wy[3] = {ay * ay, fma(-2.0 * dy, dy, 1.5), by * by};
+  double wx[3], wy[3];
+  if (LAG) {  // quadratic Lagrange at nodes -1, 0, +1 (R-25)
+    const double hx = 0.5 * dx, hy = 0.5 * dy;
+    wx[0] = hx * (dx - 1.0); wx[1] = fma(-dx, dx, 1.0); wx[2] = hx * (dx + 1.0);
+    wy[0] = hy * (dy - 1.0); wy[1] = fma(-dy, dy, 1.0); wy[2] = hy * (dy + 1.0);
+  } else {  // 2 x TSC
+    const double ax = 0.5 - dx, bx = 0.5 + dx, ay = 0.5 - dy, by = 0.5 + dy;
+    wx[0] = ax * ax; wx[1] = fma(-2.0 * dx, dx, 1.5); wx[2] = bx * bx;
+    wy[0] = ay * ay; wy[1] = fma(-2.0 * dy, dy, 1.5); wy[2] = by * by;
+  }
   double s[3][3];
   const double w00 = wx[0] * wy[0];
 #pragma unroll
@@ -653,6 +663,7 @@ __device__ __forceinline__ void contract_point(const Geo& g, const NodeRec& nd,
   f2 = nd.w0 * s[0][2] + nd.w1 * s[1][2] + nd.w2 * s[2][2];
 }
 
+template <bool LAG>
 __device__ __forceinline__ void pipelined_round(const Item& it, const Params& P,
                                                 const WarpSmem& S,
                                                 const double2* __restrict__ trig_full, int e,
@@ -661,10 +672,10 @@ __device__ __forceinline__ void pipelined_round(const Item& it, const Params& P,
                                                 double& k1, double& k2, double& g0, double& g1,
                                                 double& g2, unsigned fullmask) {
   const size_t rs = (size_t)4 * P.PX;
-  const float inv_n1 = 1.0f / (float)(N - 1);  // interior nodes per arc (R-24)
+  const float inv_n1 = 1.0f / (float)(LAG ? N + 1 : N - 1);  // arc slots per arc (R-24)
   const double2 trf = __ldg(trig_full + (e < N ? e : 0));
-  Geo cur = (fullmask & 1) ? geom_point<true>(P, S, trf, e, 0, N, wfull, third, inv_n1)
-                        : geom_point<false>(P, S, trf, e, 0, N, wfull, third, inv_n1);
+  Geo cur = (fullmask & 1) ? geom_point<true, LAG>(P, S, trf, e, 0, N, wfull, third, inv_n1)
+                        : geom_point<false, LAG>(P, S, trf, e, 0, N, wfull, third, inv_n1);
 #pragma unroll 1
   for (int n = 0; n < nn; ++n) {
     if (cur.cell != kNoCell && cur.cell != ccell) {
@@ -675,14 +686,14 @@ __device__ __forceinline__ void pipelined_round(const Item& it, const Params& P,
     double f0, f1, f2;
     Geo nxt;
     if (n + 1 < nn && ((fullmask >> (n + 1)) & 1)) {
-      nxt = geom_point<true>(P, S, trf, e, n + 1, N, wfull, third, inv_n1);
-      contract_point(cur, nd, st, f0, f1, f2);
+      nxt = geom_point<true, LAG>(P, S, trf, e, n + 1, N, wfull, third, inv_n1);
+      contract_point<LAG>(cur, nd, st, f0, f1, f2);
     } else if (n + 1 < nn) {
-      nxt = geom_point<false>(P, S, trf, e, n + 1, N, wfull, third, inv_n1);
-      contract_point(cur, nd, st, f0, f1, f2);
+      nxt = geom_point<false, LAG>(P, S, trf, e, n + 1, N, wfull, third, inv_n1);
+      contract_point<LAG>(cur, nd, st, f0, f1, f2);
     } else {
       nxt = cur;
-      contract_point(cur, nd, st, f0, f1, f2);
+      contract_point<LAG>(cur, nd, st, f0, f1, f2);
     }
     const double wk = cur.w * nd.wk;
     k0 += wk * f0; k1 += wk * f1; k2 += wk * f2;
@@ -790,7 +801,7 @@ __global__ void __launch_bounds__(32 * kWarps) k_integrate(
         }
         cnt = na < 0 ? N : na * (N + 1);
         full = na < 0;
-        if (KIND == RP_SRC_GRID && VAR >= 4 && na > 0) {  // interior arc nodes only (R-24)
+        if (KIND == RP_SRC_GRID && VAR >= 4 && VAR != 6 && na > 0) {  // interior nodes (R-24)
           skip = 2 * na;
           cnt = na * (N - 1);
         }
@@ -823,7 +834,7 @@ __global__ void __launch_bounds__(32 * kWarps) k_integrate(
       if (KIND == RP_SRC_GRID && VAR >= 4) {
         for (int rr = 0; rr < rounds; ++rr) {
           const int r = (nseg & 1) ? rounds - 1 - rr : rr;
-          pipelined_round(it, P, S, trig_full, 32 * r + lane, nn, N,
+          pipelined_round<VAR == 6>(it, P, S, trig_full, 32 * r + lane, nn, N,
                                                    wfull, third, st, ccell, k0, k1, k2, g0, g1,
                                                    g2, fullmask);
         }
@@ -1077,8 +1088,9 @@ static int run_potentials(rp_ctx* ctx, const Params& P, int32_t rank, int32_t wo
                                               ctx->sched_key_sorted, ctx->sched_idx,
                                               ctx->sched_order, (int)nd, 0, 16, st));
     }
-    const int var = KIND == RP_SRC_GRID ? ctx->eval_variant : 0;
+    const int var = KIND != RP_SRC_GRID ? 0 : (P.interp == RP_INTERP_LAGRANGE3 ? 6 : ctx->eval_variant);
     int rc2 = var == 4 ? launch_integrate<KIND, 4>(ctx, P)
+              : var == 6 ? launch_integrate<KIND, 6>(ctx, P)
               : var == 7 ? launch_integrate<KIND, 7>(ctx, P)
                          : launch_integrate<KIND, 0>(ctx, P);
     if (rc2) return rc2;
@@ -1104,6 +1116,7 @@ int rp_potentials_impl(rp_ctx* ctx, int kind, const double src[6], int32_t rank,
   P.kap = kappa_of(ctx); P.k = ctx->k; P.H = ctx->H; P.n_theta = c.n_theta;
   P.max_depth = c.max_depth; P.n_root = c.n_root; P.rule = c.outer_rule;
   P.variant = ctx->eval_variant;
+  P.interp = c.interp;
   P.hx = c.hx; P.hy = c.hy; P.inv_hx = 1.0 / c.hx; P.inv_hy = 1.0 / c.hy;
   P.cdt = c.c * c.dt; P.tau = c.tau; P.R = (double)P.kap * P.cdt;
   P.slot_doubles = ctx->slot_doubles; P.ring = ctx->ring; P.frames = ctx->frames_dev;

@@ -36,7 +36,8 @@ class rp_config(C.Structure):
     _fields_ = [("nx", C.c_int32), ("ny", C.c_int32), ("hx", C.c_double), ("hy", C.c_double),
                 ("history_depth", C.c_int32), ("c", C.c_double), ("dt", C.c_double),
                 ("tau", C.c_double), ("n_theta", C.c_int32), ("max_depth", C.c_int32),
-                ("n_root", C.c_int32), ("device", C.c_int32), ("outer_rule", C.c_int32)]
+                ("n_root", C.c_int32), ("device", C.c_int32), ("outer_rule", C.c_int32),
+                ("interp", C.c_int32)]
 
 
 class rp_deposit_info(C.Structure):
@@ -197,9 +198,9 @@ def rp_profile_read(ctx) -> rp_profile:
 
 
 def rp_create(nx, ny, hx, hy, history_depth, c, dt, tau, n_theta=64, max_depth=30, n_root=2,
-              device=0, outer_rule=0):
+              device=0, outer_rule=0, interp=0):
     cfg = rp_config(nx, ny, hx, hy, history_depth, c, dt, tau, n_theta, max_depth, n_root, device,
-                    outer_rule)
+                    outer_rule, interp)
     out = C.c_void_p()
     _check(_lib.rp_create(C.byref(cfg), C.byref(out)), None, "rp_create")
     return out

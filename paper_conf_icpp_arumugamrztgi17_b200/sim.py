@@ -38,7 +38,7 @@ class Simulation:
         dev_index = self.device.index if self.device.type == "cuda" else 0
         self.ctx = ops.rp_create(cfg.nx, cfg.ny, cfg.hx, cfg.hy, cfg.kappa_max, cfg.c, cfg.dt,
                                  cfg.tau, cfg.n_theta, cfg.max_depth, cfg.n_root, dev_index or 0,
-                                 cfg.rule)
+                                 cfg.rule, cfg.interp)
         if self.device.type == "cuda":
             ops.rp_set_stream(self.ctx, torch.cuda.current_stream(self.device))
         ops.rp_history_init(self.ctx, cfg.n_pre, W.frames(cfg, range(-cfg.n_pre, 0)), None, True)

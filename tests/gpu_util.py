@@ -18,17 +18,19 @@ def torch_dev():
 
 def make_ctx(cfg: W.Config, **over):
     from paper_conf_icpp_arumugamrztgi17_b200 import rp
-    kw = dict(n_theta=cfg.n_theta, max_depth=cfg.max_depth, n_root=cfg.n_root, rule=cfg.rule)
+    kw = dict(n_theta=cfg.n_theta, max_depth=cfg.max_depth, n_root=cfg.n_root, rule=cfg.rule,
+              interp=cfg.interp)
     kw.update(over)
     return rp.rp_create(cfg.nx, cfg.ny, cfg.hx, cfg.hy, cfg.kappa_max, cfg.c, cfg.dt,
                         over.get("tau", cfg.tau), kw["n_theta"], kw["max_depth"], kw["n_root"], 0,
-                        kw["rule"])
+                        kw["rule"], kw["interp"])
 
 
 def oracle_problem(cfg: W.Config, ring, frames, k, n_pre, **over):
     kw = dict(nx=cfg.nx, ny=cfg.ny, hx=cfg.hx, hy=cfg.hy, c=cfg.c, dt=cfg.dt, tau=cfg.tau,
               kappa_max=cfg.kappa_max, k=k, n_pre=n_pre, ring=ring, frames=frames,
-              n_theta=cfg.n_theta, max_depth=cfg.max_depth, n_root=cfg.n_root, rule=cfg.rule)
+              n_theta=cfg.n_theta, max_depth=cfg.max_depth, n_root=cfg.n_root, rule=cfg.rule,
+              interp=cfg.interp)
     kw.update(over)
     return oracle.Problem(**kw)
 

@@ -34,9 +34,10 @@ class _Ctx:
 class OracleOps:
     """CPU stand-in for the librp binding with the C-ABI semantics of include/rp.h."""
 
-    def rp_create(self, nx, ny, hx, hy, kap, c, dt, tau, n_theta, max_depth, n_root, dev, rule=0):
+    def rp_create(self, nx, ny, hx, hy, kap, c, dt, tau, n_theta, max_depth, n_root, dev, rule=0,
+                  interp=0):
         x = _Ctx()
-        x.rule = rule
+        x.rule, x.interp = rule, interp
         x.nx, x.ny, x.hx, x.hy, x.kap, x.c, x.dt, x.tau = nx, ny, hx, hy, kap, c, dt, tau
         x.n_theta, x.max_depth, x.n_root = n_theta, max_depth, n_root
         x.H = kap + 2
@@ -83,7 +84,8 @@ class OracleOps:
         return oracle.Problem(nx=ctx.nx, ny=ctx.ny, hx=ctx.hx, hy=ctx.hy, c=ctx.c, dt=ctx.dt,
                               tau=ctx.tau, kappa_max=ctx.kap, k=ctx.k, n_pre=ctx.n_pre,
                               ring=ctx.ring, frames=ctx.frames, n_theta=ctx.n_theta,
-                              max_depth=ctx.max_depth, n_root=ctx.n_root, rule=ctx.rule)
+                              max_depth=ctx.max_depth, n_root=ctx.n_root, rule=ctx.rule,
+                              interp=ctx.interp)
 
     def rp_compute_potentials(self, ctx, phi, ax, ay, err=None, nseg=None, info=False):
         r = self._problem(ctx).potentials(np.arange(ctx.nx * ctx.ny))

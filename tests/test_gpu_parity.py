@@ -206,14 +206,15 @@ def _bend_small(n=24, kap=60):
                     r0=c.r0, sigma_xp=c.sigma_xp, q_over_mc=c.q_over_mc)
 
 
-@pytest.mark.parametrize("rule", [0, 1])
-def test_potentials_bend_small_full_mesh_two_steps(torch, rule):
+@pytest.mark.parametrize("rule,interp", [(0, 0), (1, 0), (0, 1)])
+def test_potentials_bend_small_full_mesh_two_steps(torch, rule, interp):
     """Moving frames, node-sampled history with a time-varying amplitude, two consecutive
-    steps (the second uses the first step's counts as the schedule forecast); GK15 and the
-    paper's Simpson rule (R-22)."""
+    steps (the second uses the first step's counts as the schedule forecast); GK15, the
+    paper's Simpson rule (R-22) and the Lagrange-3 spatial stencil (R-25)."""
     from paper_conf_icpp_arumugamrztgi17_b200 import rp
     cfg = _bend_small()
     cfg.rule = rule
+    cfg.interp = interp
     ctx = G.make_ctx(cfg)
     try:
         for k in (5, 6):
@@ -231,7 +232,8 @@ def test_potentials_bend_small_full_mesh_two_steps(torch, rule):
 
 
 @pytest.mark.parametrize("variant", [dict(n_root=1), dict(max_depth=5), dict(n_theta=16),
-                                     dict(rule=1), dict(rule=1, n_root=1)])
+                                     dict(rule=1), dict(rule=1, n_root=1), dict(interp=1),
+                                     dict(interp=1, n_theta=16)])
 def test_potentials_variants(torch, variant):
     from paper_conf_icpp_arumugamrztgi17_b200 import rp
     cfg = W.Config(number=0, name="v", nx=20, ny=13, n_particles=4000, steps=4, kappa_max=7,

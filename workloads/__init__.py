@@ -47,6 +47,7 @@ class Config:
     max_depth: int = 30
     n_root: int = 2
     rule: int = 0            # outer segment rule: 0 = GK15, 1 = Simpson/Boole (the paper's)
+    interp: int = 0          # spatial weights: 0 = TSC (R-6), 1 = quadratic Lagrange (R-25)
     tau_rel: float = 1e-6    # tau = tau_rel * (Q/sigma) sqrt(pi/2)
     seed: int = 0
 
