@@ -67,7 +67,8 @@ typedef struct {
                            /* rule (P:155 RP-QUADRULE), Boole value + |S2 - S1|/15 estimate (R-22) */
   int32_t interp;          /* spatial part of the "27 neighbouring points": RP_INTERP_TSC */
                            /* (default, R-6) or RP_INTERP_LAGRANGE3 (tri-quadratic Lagrange with  */
-                           /* the time interpolation, R-25; discontinuous across cells)          */
+                           /* the time interpolation, R-25; discontinuous across cells; arc end  */
+                           /* nodes on the support boundary take the outside limit 0, R-25b)     */
 } rp_config;
 
 #define RP_RULE_GK15 0
@@ -91,8 +92,9 @@ typedef struct {
   int32_t max_level;       /* deepest tree level reached                                         */
   int32_t kappa;           /* subregions kappa(k) used at this step (R-3)                        */
   int64_t skipped;         /* of `evals`, arc end nodes on the support boundary, where the zero-
-                              padded TSC integrand vanishes, not evaluated (DESIGN R-24); the
-                              evaluations performed are evals - skipped                         */
+                              padded TSC integrand vanishes (DESIGN R-24) or the Lagrange-3 one
+                              takes its outside limit 0 (R-25b), not evaluated; the evaluations
+                              performed are evals - skipped                                     */
 } rp_potential_info;
 
 /* Create a context on cfg->device: allocates the HBM history ring of history_depth+2

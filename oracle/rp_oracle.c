@@ -480,8 +480,12 @@ void orc_inner_ctx(subctx* X, double r, double* out) {
     for (int32_t m = 0; m <= N; ++m) {
       double th = t1 + (double)m * h;
       double w = (m == 0 || m == N) ? h / 3.0 : ((m & 1) ? 4.0 * h / 3.0 : 2.0 * h / 3.0);
-      integrand(X, cu + r * cos(th), cv + r * sin(th), wt, f);
       X->evals++;
+      /* R-25b: with the Lagrange-3 stencil the integrand jumps on the support boundary, where
+       * every arc ends; the end nodes take the limit from outside the support, 0 (under TSC
+       * the integrand is continuous there and already 0, R-24) */
+      if ((m == 0 || m == N) && X->S->kind == ORC_SRC_GRID && X->P->interp == 1) continue;
+      integrand(X, cu + r * cos(th), cv + r * sin(th), wt, f);
       for (int c = 0; c < 3; ++c) out[c] += w * f[c];
     }
   }

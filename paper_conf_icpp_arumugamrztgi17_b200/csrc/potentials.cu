@@ -589,14 +589,14 @@ __device__ __forceinline__ Geo geom_point(const Params& P, const WarpSmem& S, do
     w = wfull;
   } else {
     // slot e -> arc q, interior Simpson node mm = 1 .. N-1: the end nodes mm = 0, N of an arc
-    // lie on the support boundary, where the zero-padded TSC stencil vanishes (R-24)
-    // (Lagrange-3, R-25: the integrand does not vanish there, all N+1 nodes are evaluated)
+    // lie on the support boundary, where the zero-padded TSC stencil vanishes (R-24) and the
+    // Lagrange-3 integrand takes its limit from outside, 0 (R-25b)
     const int ec = valid ? e : 0;
     const int q = __float2int_rz(((float)ec + 0.5f) * inv_n1);  // arc index, exact for e < 2^20
-    const int mm = LAG ? ec - q * (N + 1) : ec - q * (N - 1) + 1;
+    const int mm = ec - q * (N - 1) + 1;
     const double d = S.dth[n][q];
     sincos_b(S.th1[n][q] + (double)mm * d, &sn, &cs);
-    const double coef = (LAG && (mm == 0 || mm == N)) ? 1.0 : ((mm & 1) ? 4.0 : 2.0);
+    const double coef = (mm & 1) ? 4.0 : 2.0;
     w = coef * d * third;
   }
   const NodeRec& nd = S.node[n];
@@ -672,7 +672,7 @@ __device__ __forceinline__ void pipelined_round(const Item& it, const Params& P,
                                                 double& k1, double& k2, double& g0, double& g1,
                                                 double& g2, unsigned fullmask) {
   const size_t rs = (size_t)4 * P.PX;
-  const float inv_n1 = 1.0f / (float)(LAG ? N + 1 : N - 1);  // arc slots per arc (R-24)
+  const float inv_n1 = 1.0f / (float)(N - 1);  // arc slots per arc (R-24, R-25b)
   const double2 trf = __ldg(trig_full + (e < N ? e : 0));
   Geo cur = (fullmask & 1) ? geom_point<true, LAG>(P, S, trf, e, 0, N, wfull, third, inv_n1)
                         : geom_point<false, LAG>(P, S, trf, e, 0, N, wfull, third, inv_n1);
@@ -801,7 +801,7 @@ __global__ void __launch_bounds__(32 * kWarps) k_integrate(
         }
         cnt = na < 0 ? N : na * (N + 1);
         full = na < 0;
-        if (KIND == RP_SRC_GRID && VAR >= 4 && VAR != 6 && na > 0) {  // interior nodes (R-24)
+        if (KIND == RP_SRC_GRID && VAR >= 4 && na > 0) {  // interior nodes (R-24, R-25b)
           skip = 2 * na;
           cnt = na * (N - 1);
         }

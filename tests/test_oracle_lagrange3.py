@@ -84,3 +84,29 @@ def test_lagrange3_inner_circle_closed_form():
         assert n == 64
         want = 2 * math.pi * (_p(co, px, py) + (d + f2) * r * r / 2)
         np.testing.assert_allclose(out, [want, 2 * want, -want], rtol=1e-13, atol=1e-13)
+
+
+def test_arc_end_nodes_take_the_outside_limit():
+    """R-25b: the Lagrange-3 integrand jumps on the support boundary (just inside, the node
+    row outside the grid has weight 0 but the first grid row has -1/8; just outside, every
+    node is outside the grid), and every arc ends on that boundary.  The end nodes take the
+    outside limit 0, so inner(r') no longer depends on which side the rounding of a crossing
+    angle puts them: it is continuous in r' (a 1e-13 relative change of r' moves it by
+    rounding only), which evaluating the end nodes fails by O(h g / 3)."""
+    P, coeffs = _problem(1)
+    hx = P.params.hx
+    # the jump: just inside / outside the left edge u = -1.5 h of the support rectangle
+    v = 7.3 * P.params.hy
+    inside = P.integrand(0, -1.5 * hx * (1 - 1e-12), v, 0.5)
+    outside = P.integrand(0, -1.5 * hx * (1 + 1e-12), v, 0.5)
+    assert np.all(outside == 0.0) and abs(inside[0]) > 1e-3
+    rng = np.random.default_rng(3)
+    worst = 0.0
+    for _ in range(150):
+        ix, iy = rng.integers(0, 40), rng.integers(0, 36)
+        r = rng.uniform(2.0, 25.0)
+        px, py = P.mesh_point(ix, iy)
+        a, _ = P.inner(px, py, 0, r)
+        b, _ = P.inner(px, py, 0, r * (1 + 1e-13))
+        worst = max(worst, float(np.max(np.abs(a - b))) / max(float(np.max(np.abs(a))), 1e-300))
+    assert worst < 1e-9, worst

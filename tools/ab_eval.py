@@ -1,4 +1,5 @@
-"""Development A/B of integrator evaluation loops (RP_EVAL=<v> selects one at rp_create).
+"""Development A/B of integrator evaluation loops (RP_EVAL=<v> selects one at rp_create; a
+variant may also be a comma list of environment settings read at rp_create, e.g. RP_COEF=0).
 
 Runs `steps` steps of a config per variant in one process, checks that every variant's
 potentials / segment counts are bit-identical to the first one's, and prints the integrator's
@@ -17,11 +18,18 @@ from paper_conf_icpp_arumugamrztgi17_b200.sim import Simulation  # noqa: E402
 
 cfgn = int(sys.argv[1]) if len(sys.argv) > 1 else 2
 steps = int(sys.argv[2]) if len(sys.argv) > 2 else 4
-variants = [int(v) for v in sys.argv[3:]] or [0, 1]
+variants = sys.argv[3:] or ["4", "RP_COEF=0"]
 cfg = W.config(cfgn)
 ref = None
 for v in variants:
-    os.environ["RP_EVAL"] = str(v)
+    for key in ("RP_EVAL", "RP_COEF"):
+        os.environ.pop(key, None)
+    if "=" in v:
+        for kv in v.split(","):
+            key, val = kv.split("=")
+            os.environ[key] = val
+    else:
+        os.environ["RP_EVAL"] = v
     sim = Simulation(cfg)
     rp.rp_profile_enable(sim.ctx, True)
     outs, ms, ev, last = [], [], [], 0.0
@@ -33,7 +41,7 @@ for v in variants:
         last = prof.integrate_ms
         ev.append(info.evals)
         outs.append([t.cpu().numpy().copy() for t in (sim.phi, sim.ax, sim.ay, sim.nseg)])
-    if v == 7:
+    if v == "7":
         import ctypes
         buf = (ctypes.c_ulonglong * 6)()
         rp._lib.rp_dev_phase_cycles(buf, 1)
@@ -49,6 +57,11 @@ for v in variants:
         same = all(np.array_equal(a.view(np.uint8) if a.dtype != np.int32 else a,
                                   b.view(np.uint8) if b.dtype != np.int32 else b)
                    for oa, ob in zip(outs, ref) for a, b in zip(oa, ob))
+        if not same:  # rounding-level differences: report the relative size and nseg equality
+            rel = max(float(np.max(np.abs(a - b))) / max(float(np.max(np.abs(b))), 1e-300)
+                      for oa, ob in zip(outs, ref) for a, b in zip(oa[:3], ob[:3]))
+            nseg_eq = all(np.array_equal(oa[3], ob[3]) for oa, ob in zip(outs, ref))
+            same = f"no (max rel diff {rel:.2e}, nseg equal {nseg_eq})"
     print(f"variant {v}: integrate ms/step {[round(x, 2) for x in ms]} "
           f"(steps 2+: {np.mean(ms[2:]) if len(ms) > 2 else np.mean(ms):.2f}); "
           f"ps/eval {[round(1e9 * m / e, 2) for m, e in zip(ms, ev)]}; "
