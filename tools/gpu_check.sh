@@ -1,6 +1,5 @@
-# quick GPU check: parity tests (per-test timeout, durations), integrator A/B, short bench
-timeout 1500 python -m pytest tests -m gpu -x -q --timeout=400 --durations=15 > gpurun_out/pytest_gpu.log 2>&1; tail -25 gpurun_out/pytest_gpu.log
-python tools/ab_eval.py 2 5 ${AB_VARIANTS:-4 RP_COEF=0} 2>&1 | tail -4
+# quick GPU check: parity tests (per-test timeout, durations), short bench
+timeout 1500 python -m pytest tests -m gpu -q --timeout=400 --durations=12 > gpurun_out/pytest_gpu.log 2>&1; tail -22 gpurun_out/pytest_gpu.log
 python bench.py --steps 3 --warmup 3 --no-cpu-baseline > gpurun_out/bench_quick.json 2> gpurun_out/bench_quick.err
 python -c "
 import json; d=json.load(open('gpurun_out/bench_quick.json')); print(d['ms_per_step'], d['roofline']['frac'], d['kernel_ms_per_step'])"
