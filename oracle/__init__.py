@@ -74,6 +74,7 @@ def lib():
         P = C.POINTER
         d, i32, i64 = C.c_double, C.c_int32, C.c_int64
         pd, pi32 = P(d), P(i32)
+        pu16, pi64 = P(C.c_uint16), P(i64)
         sig = {
             "orc_gk15_constants": (None, [pd, pd, pd]),
             "orc_tsc_weights": (None, [d, pd]),
@@ -87,6 +88,12 @@ def lib():
             "orc_mesh_point": (None, [P(Params), P(Frame), i32, i32, pd, pd]),
             "orc_point_lab": (None, [P(Params), P(Hist), P(Source), d, d, P(Result)]),
             "orc_potentials": (None, [P(Params), P(Hist), P(Source), pi32, i32, P(Result)]),
+            "orc_potentials_ex": (None, [P(Params), P(Hist), P(Source), pi32, i32, pu16, P(Result)]),
+            "orc_potentials_predictive": (i32, [P(Params), P(Hist), P(Source), pu16, i32, i32, i32,
+                                                pi32, i32, pi32, pu16, P(Result)]),
+            "orc_knn_pattern": (i32, [pu16, i32, i32, i32, i32, i32, i32]),
+            "orc_kmeans": (i32, [pu16, i32, i32, i32, i32, pi32]),
+            "orc_merge_partitions": (i64, [P(Params), pu16, pi32, i32, i32, pi64, pd]),
             "orc_clip_at": (i32, [P(Params), P(Hist), P(Source), d, d, i32, pd, pd]),
             "orc_dists_at": (None, [P(Params), P(Hist), P(Source), d, d, i32, d, pd, pd]),
             "orc_inner_at": (i64, [P(Params), P(Hist), P(Source), d, d, i32, d, pd]),
@@ -113,6 +120,25 @@ def _pd(a):
 def _pi(a):
     assert a.dtype == np.int32 and a.flags.c_contiguous
     return a.ctypes.data_as(C.POINTER(C.c_int32))
+
+
+def _pu16(a):
+    assert a.dtype == np.uint16 and a.flags["C_CONTIGUOUS"]
+    return a.ctypes.data_as(C.POINTER(C.c_uint16))
+
+
+def knn_pattern(prev, nx, ny, p, j, knn):
+    prev = np.ascontiguousarray(prev, dtype=np.uint16)
+    return lib().orc_knn_pattern(_pu16(prev), nx, ny, prev.shape[1], p, j, knn)
+
+
+def kmeans(pattern, m, max_iters=20):
+    """RP-CLUSTERING (P:134, P:159; R-26): (assignment, passes)."""
+    pattern = np.ascontiguousarray(pattern, dtype=np.uint16)
+    assign = np.zeros(pattern.shape[0], dtype=np.int32)
+    it = lib().orc_kmeans(_pu16(pattern), pattern.shape[0], pattern.shape[1], m, max_iters,
+                          _pi(assign))
+    return assign, it
 
 
 def frame(f) -> Frame:
@@ -172,6 +198,45 @@ class Problem:
         lib().orc_potentials(C.byref(self.params), C.byref(self.hist), C.byref(self.source),
                              _pi(pts), len(pts), out)
         return np.ctypeslib.as_array(out).copy() if len(pts) else np.zeros(0)
+
+    def potentials_items(self, pts):
+        """Potentials at flattened mesh points plus the observed access pattern: accepted
+        segments per (point, subregion), uint16 [len(pts), kappa_max]."""
+        pts = np.ascontiguousarray(pts, dtype=np.int32)
+        out = (Result * len(pts))()
+        leaves = np.zeros((len(pts), self.params.kappa_max), dtype=np.uint16)
+        lib().orc_potentials_ex(C.byref(self.params), C.byref(self.hist), C.byref(self.source),
+                                _pi(pts), len(pts), _pu16(leaves), out)
+        return np.ctypeslib.as_array(out).copy(), leaves
+
+    def potentials_predictive(self, prev, pts, knn=9, m=0, max_iters=20):
+        """Predictive-RP variant (Algorithm 1, reading R-26) at step k from the previous
+        step's pattern prev [nx*ny, kappa_max] (uint16).  Returns (results, clusters [nx*ny],
+        leaves [len(pts), kappa_max], k-means passes)."""
+        prev = np.ascontiguousarray(prev, dtype=np.uint16)
+        nall = self.params.nx * self.params.ny
+        assert prev.shape == (nall, self.params.kappa_max)
+        pts = np.ascontiguousarray(pts, dtype=np.int32)
+        out = (Result * max(len(pts), 1))()
+        clusters = np.zeros(nall, dtype=np.int32)
+        leaves = np.zeros((len(pts), self.params.kappa_max), dtype=np.uint16)
+        it = lib().orc_potentials_predictive(C.byref(self.params), C.byref(self.hist),
+                                             C.byref(self.source), _pu16(prev), knn, m, max_iters,
+                                             _pi(pts), len(pts), _pi(clusters), _pu16(leaves), out)
+        res = np.ctypeslib.as_array(out).copy()[:len(pts)]
+        return res, clusters, leaves, it
+
+    def merge_partitions(self, pattern, assign, m):
+        """Per-cluster merged uniform partitions of S_j (lines 4, 9-12): (off, breakpoints)."""
+        pattern = np.ascontiguousarray(pattern, dtype=np.uint16)
+        assign = np.ascontiguousarray(assign, dtype=np.int32)
+        off = np.zeros(m * self.params.kappa_max + 1, dtype=np.int64)
+        n = lib().orc_merge_partitions(C.byref(self.params), _pu16(pattern), _pi(assign),
+                                       len(assign), m, off.ctypes.data_as(C.POINTER(C.c_int64)), None)
+        bp = np.zeros(max(n, 1))
+        lib().orc_merge_partitions(C.byref(self.params), _pu16(pattern), _pi(assign), len(assign),
+                                   m, off.ctypes.data_as(C.POINTER(C.c_int64)), _pd(bp))
+        return off, bp[:n]
 
     def clip(self, px, py, j):
         A, B = C.c_double(), C.c_double()

@@ -619,8 +619,19 @@ void orc_mesh_point(const orc_params* P, const orc_frame* F, int32_t ix, int32_t
   *py = F->oy + u * F->s + v * F->c;
 }
 
-void orc_point_lab(const orc_params* P, const orc_hist* Hh, const orc_source* S, double px,
-                   double py, orc_result* res) {
+/* Root intervals of one (point, subregion) item under the Predictive-RP variant (R-26):
+ * the intervals of the item's cluster partition list (sorted breakpoints of S_j) cut to
+ * the item's support [A, B]; empty pieces dropped. */
+typedef struct {
+  const double* bp;      /* breakpoints, all lists back to back                         */
+  const int64_t* off;    /* [n_clusters * kappa_max + 1]: list (c, j) = bp[off[i], off[i+1]) */
+  int32_t cluster;       /* the point's cluster                                          */
+  int32_t kappa_max;
+} orc_roots;
+
+static void point_lab_ex(const orc_params* P, const orc_hist* Hh, const orc_source* S,
+                         double px, double py, const orc_roots* RT, uint16_t* leaves_row,
+                         orc_result* res) {
   memset(res, 0, sizeof(*res));
   res->min_margin = INFINITY;
   int32_t kap = orc_kappa(P, Hh);
@@ -632,27 +643,222 @@ void orc_point_lab(const orc_params* P, const orc_hist* Hh, const orc_source* S,
     setup_sub(&X, P, Hh, S, px, py, j);
     double A, B;
     if (!orc_clip(&X, j * cdt, (j + 1) * cdt, &A, &B)) continue;
-    if (P->n_root == 1) {
+    int32_t leaves0 = res->nleaf;
+    int64_t lo = 0, hi = 0;
+    if (RT) {
+      int64_t i = (int64_t)RT->cluster * RT->kappa_max + j;
+      lo = RT->off[i];
+      hi = RT->off[i + 1];
+    }
+    if (hi - lo >= 2) {
+      /* Algorithm 1 lines 13-16 (COMPUTE-RP-INTEGRAL over the cluster partition) and 18-24
+       * (adaptive quadrature on the intervals that fail): each cut interval is the root of
+       * a dyadic tree, its first evaluation being the partition-phase estimate */
+      for (int64_t t = lo; t + 1 < hi; ++t) {
+        double a = RT->bp[t] > A ? RT->bp[t] : A;
+        double b = RT->bp[t + 1] < B ? RT->bp[t + 1] : B;
+        if (a < b) tree(&X, a, b, R, 0, 0, res);
+      }
+    } else if (P->n_root == 1) {
       tree(&X, A, B, R, 0, 0, res);
     } else {
       tree(&X, A, B, R, 1, 0, res);
       tree(&X, A, B, R, 1, 1, res);
     }
+    if (leaves_row) {
+      int32_t nl = res->nleaf - leaves0;
+      leaves_row[j] = (uint16_t)(nl < 0xFFFF ? nl : 0xFFFF);
+    }
     res->evals += X.evals;
   }
 }
 
-/* Potentials at a list of mesh points (flattened iy*nx+ix) of frame k. */
-void orc_potentials(const orc_params* P, const orc_hist* Hh, const orc_source* S,
-                    const int32_t* pts, int32_t npts, orc_result* out) {
+void orc_point_lab(const orc_params* P, const orc_hist* Hh, const orc_source* S, double px,
+                   double py, orc_result* res) {
+  point_lab_ex(P, Hh, S, px, py, NULL, NULL, res);
+}
+
+/* Potentials at a list of mesh points (flattened iy*nx+ix) of frame k.  leaves (nullable):
+ * [npts][kappa_max] accepted segments per (point, subregion) -- the observed access
+ * pattern n_j(p) of P:83-95 that the Predictive-RP variant forecasts from. */
+void orc_potentials_ex(const orc_params* P, const orc_hist* Hh, const orc_source* S,
+                       const int32_t* pts, int32_t npts, uint16_t* leaves, orc_result* out) {
   const orc_frame* Fk = Hh->frames + slot_of(Hh->k, Hh->H);
 #pragma omp parallel for schedule(dynamic, 1)
   for (int32_t i = 0; i < npts; ++i) {
     int32_t p = pts[i];
     double px, py;
     orc_mesh_point(P, Fk, p % P->nx, p / P->nx, &px, &py);
-    orc_point_lab(P, Hh, S, px, py, out + i);
+    uint16_t* row = leaves ? leaves + (int64_t)i * P->kappa_max : NULL;
+    if (row) memset(row, 0, sizeof(uint16_t) * P->kappa_max);
+    point_lab_ex(P, Hh, S, px, py, NULL, row, out + i);
   }
+}
+
+void orc_potentials(const orc_params* P, const orc_hist* Hh, const orc_source* S,
+                    const int32_t* pts, int32_t npts, orc_result* out) {
+  orc_potentials_ex(P, Hh, S, pts, npts, NULL, out);
+}
+
+/* ------------------------------------------------------------------ */
+/* Predictive-RP: the paper's COMPUTE-POTENTIALS (Algorithm 1) as a variant    */
+/* (reading R-26).  Lines 1-6 and 9-12 are host work in the paper; here they are   */
+/* written out plainly, in the paper's order.                                              */
+/* ------------------------------------------------------------------ */
+/* Line 3, g = kNN regression over the mesh: the mean of the previous step's access
+ * pattern n_j over the k nearest mesh nodes in index space (k = 1: the node; 5: the node and
+ * its 4 edge neighbours; 9: the 3x3 block; 25: the 5x5 block; nodes off the mesh are not
+ * neighbours), rounded half up: (sum + cnt/2) / cnt in integers. */
+int32_t orc_knn_pattern(const uint16_t* prev, int32_t nx, int32_t ny, int32_t kmax, int32_t p,
+                        int32_t j, int32_t knn) {
+  int32_t ix = p % nx, iy = p / nx;
+  int32_t rad = knn >= 25 ? 2 : (knn >= 5 ? 1 : 0);
+  uint32_t sum = 0, cnt = 0;
+  for (int32_t dy = -rad; dy <= rad; ++dy)
+    for (int32_t dx = -rad; dx <= rad; ++dx) {
+      if (knn == 5 && dx != 0 && dy != 0) continue;
+      int32_t x = ix + dx, y = iy + dy;
+      if (x < 0 || x >= nx || y < 0 || y >= ny) continue;
+      sum += prev[((int64_t)y * nx + x) * kmax + j];
+      cnt++;
+    }
+  return (int32_t)((sum + cnt / 2) / cnt);
+}
+
+/* Line 6, RP-CLUSTERING: k-means of the access-pattern vectors
+ * a(p) = (n_0(p) .. n_{kmax-1}(p)) into m clusters.  Deterministic reading (R-26): initial
+ * centres a(p_c) with p_c = floor(c * npts / m); Lloyd iterations -- assign every point to
+ * the centre of least squared distance (sum over j ascending of (a_j - mu_j)^2, ties to the
+ * lower c), then every non-empty cluster's centre to the mean of its members (integer sums
+ * divided once) -- until no assignment changes or max_iters assignments were made.
+ * Returns the number of assignment passes. */
+int32_t orc_kmeans(const uint16_t* pat, int32_t npts, int32_t kmax, int32_t m, int32_t max_iters,
+                   int32_t* assign) {
+  double* mu = (double*)malloc(sizeof(double) * (size_t)m * kmax);
+  int64_t* sum = (int64_t*)malloc(sizeof(int64_t) * (size_t)m * kmax);
+  int64_t* cnt = (int64_t*)malloc(sizeof(int64_t) * (size_t)m);
+  for (int32_t c = 0; c < m; ++c) {
+    int64_t pc = (int64_t)c * npts / m;
+    for (int32_t j = 0; j < kmax; ++j) mu[(int64_t)c * kmax + j] = (double)pat[pc * kmax + j];
+  }
+  for (int32_t p = 0; p < npts; ++p) assign[p] = -1;
+  int32_t it = 0;
+  for (;;) {
+    int32_t changed = 0;
+    ++it;
+    for (int32_t p = 0; p < npts; ++p) {
+      int32_t best = 0;
+      double bd = INFINITY;
+      for (int32_t c = 0; c < m; ++c) {
+        double d = 0.0;
+        for (int32_t j = 0; j < kmax; ++j) {
+          double e = (double)pat[(int64_t)p * kmax + j] - mu[(int64_t)c * kmax + j];
+          d += e * e;
+        }
+        if (d < bd) { bd = d; best = c; }
+      }
+      if (assign[p] != best) { assign[p] = best; changed = 1; }
+    }
+    if (!changed || it >= max_iters) break;
+    memset(sum, 0, sizeof(int64_t) * (size_t)m * kmax);
+    memset(cnt, 0, sizeof(int64_t) * (size_t)m);
+    for (int32_t p = 0; p < npts; ++p) {
+      cnt[assign[p]]++;
+      for (int32_t j = 0; j < kmax; ++j) sum[(int64_t)assign[p] * kmax + j] += pat[(int64_t)p * kmax + j];
+    }
+    for (int32_t c = 0; c < m; ++c)
+      if (cnt[c] > 0)
+        for (int32_t j = 0; j < kmax; ++j)
+          mu[(int64_t)c * kmax + j] = (double)sum[(int64_t)c * kmax + j] / (double)cnt[c];
+  }
+  free(mu); free(sum); free(cnt);
+  return it;
+}
+
+
+/* Lines 4 and 9-12: COMPUTE-PARTITION by uniform partitioning (n_j(p) equal pieces of
+ * S_j = [j c dt, (j+1) c dt], breakpoints a_j + (b_j - a_j) * (t / n)), then MERGE-LISTS over
+ * the members of each cluster (sorted, duplicate values removed).  off has
+ * m * kmax + 1 entries; bp (nullable: count only) receives the lists.  A point with
+ * n_j(p) = 0 contributes nothing; an empty list means "no forecast" (canonical roots). */
+int64_t orc_merge_partitions(const orc_params* P, const uint16_t* pat, const int32_t* assign,
+                             int32_t npts, int32_t m, int64_t* off, double* bp) {
+  const int32_t kmax = P->kappa_max;
+  const double cdt = P->c * P->dt;
+  int64_t total = 0;
+  uint8_t* seen = (uint8_t*)calloc(65536, 1);
+  double* buf = NULL;
+  int64_t cap = 0;
+  for (int32_t c = 0; c < m; ++c)
+    for (int32_t j = 0; j < kmax; ++j) {
+      off[(int64_t)c * kmax + j] = total;
+      memset(seen, 0, 65536);
+      int64_t n_all = 0;
+      for (int32_t p = 0; p < npts; ++p) {
+        int32_t n = pat[(int64_t)p * kmax + j];
+        if (assign[p] != c || n == 0 || seen[n]) continue;
+        seen[n] = 1;
+        n_all += n + 1;
+      }
+      if (n_all > cap) {
+        cap = n_all;
+        buf = (double*)realloc(buf, sizeof(double) * (size_t)cap);
+      }
+      double a = j * cdt, b = (j + 1) * cdt;
+      int64_t q = 0;
+      for (int32_t n = 1; n < 65536; ++n) {
+        if (!seen[n]) continue;
+        for (int32_t t = 0; t <= n; ++t) buf[q++] = a + (b - a) * ((double)t / (double)n);
+      }
+      if (q) qsort(buf, (size_t)q, sizeof(double), cmp_double);
+      int64_t u = 0;
+      for (int64_t i = 0; i < q; ++i)
+        if (u == 0 || buf[i] != buf[u - 1]) buf[u++] = buf[i];
+      if (bp) memcpy(bp + total, buf, sizeof(double) * (size_t)u);
+      total += u;
+    }
+  off[(int64_t)m * kmax] = total;
+  free(seen);
+  free(buf);
+  return total;
+}
+
+/* The whole variant for step k (Algorithm 1 lines 1-24): prev = the previous step's observed
+ * pattern [nx*ny][kmax] (e.g. from orc_potentials_ex); m = number of clusters (0: max(nx,
+ * ny)).  Writes the clusters (nullable) and the results at pts; leaves (nullable) as
+ * in orc_potentials_ex.  Returns the number of k-means assignment passes. */
+int32_t orc_potentials_predictive(const orc_params* P, const orc_hist* Hh, const orc_source* S,
+                                  const uint16_t* prev, int32_t knn, int32_t m,
+                                  int32_t max_iters, const int32_t* pts, int32_t npts,
+                                  int32_t* cluster_out, uint16_t* leaves, orc_result* out) {
+  const int32_t nx = P->nx, ny = P->ny, kmax = P->kappa_max, nall = nx * ny;
+  const int32_t kap = orc_kappa(P, Hh);
+  if (m <= 0) m = nx > ny ? nx : ny;
+  if (m > nall) m = nall;
+  uint16_t* pat = (uint16_t*)calloc((size_t)nall * kmax, sizeof(uint16_t));
+  for (int32_t p = 0; p < nall; ++p)
+    for (int32_t j = 0; j < kap; ++j)
+      pat[(int64_t)p * kmax + j] = (uint16_t)orc_knn_pattern(prev, nx, ny, kmax, p, j, knn);
+  int32_t* assign = (int32_t*)malloc(sizeof(int32_t) * nall);
+  int32_t iters = orc_kmeans(pat, nall, kmax, m, max_iters, assign);
+  int64_t* off = (int64_t*)malloc(sizeof(int64_t) * ((size_t)m * kmax + 1));
+  int64_t nbp = orc_merge_partitions(P, pat, assign, nall, m, off, NULL);
+  double* bp = (double*)malloc(sizeof(double) * (size_t)(nbp > 0 ? nbp : 1));
+  orc_merge_partitions(P, pat, assign, nall, m, off, bp);
+  const orc_frame* Fk = Hh->frames + slot_of(Hh->k, Hh->H);
+#pragma omp parallel for schedule(dynamic, 1)
+  for (int32_t i = 0; i < npts; ++i) {
+    int32_t p = pts[i];
+    double px, py;
+    orc_mesh_point(P, Fk, p % nx, p / nx, &px, &py);
+    orc_roots RT = {bp, off, assign[p], kmax};
+    uint16_t* row = leaves ? leaves + (int64_t)i * kmax : NULL;
+    if (row) memset(row, 0, sizeof(uint16_t) * kmax);
+    point_lab_ex(P, Hh, S, px, py, &RT, row, out + i);
+  }
+  if (cluster_out) memcpy(cluster_out, assign, sizeof(int32_t) * nall);
+  free(pat); free(assign); free(off); free(bp);
+  return iters;
 }
 
 /* Test hooks: the clip, inner integral and a single tree for (point, j). */
