@@ -238,6 +238,38 @@ int rp_debug_potentials_analytic(rp_ctx* ctx, int32_t kind, double x0, double y0
 #define RP_SCHED_KNN 2
 int rp_set_schedule(rp_ctx* ctx, int32_t policy, int32_t k);
 
+/* Predictive-RP variant: the paper's own COMPUTE-POTENTIALS (Algorithm 1; DESIGN
+ * reading R-26) instead of the canonical dyadic tree.  At every step that has the previous
+ * step's observed access pattern n_j(p) (accepted segments per point and subregion, recorded
+ * by every rp_compute_potentials call), the forecast partition is built on the host (the
+ * paper's lines 1-12 run on the CPU too): line 3 kNN forecast of n_j(p) over the
+ * k nearest mesh nodes (k in {1, 5, 9, 25}, as rp_set_schedule); line 4 uniform
+ * partitioning of each subregion S_j into n_j(p) pieces; line 6 k-means of the
+ * pattern vectors into n_clusters clusters (0: max(nx, ny); deterministic centres
+ * and Lloyd passes, at most max_iters); lines 9-12 MERGE-LISTS of the partitions of each
+ * cluster.  The kernel then integrates each (point, subregion) item over its cluster's
+ * merged intervals cut to the item's support (lines 13-16), each interval being the root
+ * of an adaptive dyadic tree that refines it where the estimate misses the tolerance
+ * (lines 18-24).  Results differ from the canonical tree within tau and depend on the
+ * forecast.  A step without a previous pattern uses the canonical tree.
+ * Single-call path only: rp_compute_potentials_shard returns RP_EINVAL while enabled.
+ * enable = 0 restores the canonical tree.  Returns RP_EINVAL on a bad k or n_clusters < 0. */
+int rp_set_predictive(rp_ctx* ctx, int32_t enable, int32_t knn, int32_t n_clusters,
+                      int32_t max_iters);
+
+typedef struct {
+  int32_t active;          /* 1 if the last rp_compute_potentials used a forecast partition    */
+  int32_t clusters;        /* k-means clusters m                                               */
+  int32_t kmeans_passes;   /* assignment passes made                                           */
+  int32_t pad;
+  int64_t breakpoints;     /* total length of the merged partition lists                      */
+  double host_ms;          /* host time of lines 1-12 (download of n_j, forecast, clustering,  */
+                           /* merge, upload), included in the call                             */
+} rp_predictive_info;
+/* Statistics of the last rp_compute_potentials (host struct, no sync).  clusters_host
+ * (nullable): the k-means cluster of every mesh point [nx * ny] (parity with the oracle). */
+int rp_predictive_info_read(rp_ctx* ctx, rp_predictive_info* out, int32_t* clusters_host);
+
 /* Per-kernel device time, measured with CUDA events recorded on the context's stream around
  * each launch while profiling is enabled (bench.py's live roofline numbers). */
 typedef struct {

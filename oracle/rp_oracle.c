@@ -777,7 +777,8 @@ int32_t orc_kmeans(const uint16_t* pat, int32_t npts, int32_t kmax, int32_t m, i
 
 
 /* Lines 4 and 9-12: COMPUTE-PARTITION by uniform partitioning (n_j(p) equal pieces of
- * S_j = [j c dt, (j+1) c dt], breakpoints a_j + (b_j - a_j) * (t / n)), then MERGE-LISTS over
+ * S_j = [j c dt, (j+1) c dt], breakpoints a_j + (b_j - a_j) * (t / n), the last one b_j
+ * itself so the list covers S_j exactly), then MERGE-LISTS over
  * the members of each cluster (sorted, duplicate values removed).  off has
  * m * kmax + 1 entries; bp (nullable: count only) receives the lists.  A point with
  * n_j(p) = 0 contributes nothing; an empty list means "no forecast" (canonical roots). */
@@ -808,7 +809,7 @@ int64_t orc_merge_partitions(const orc_params* P, const uint16_t* pat, const int
       int64_t q = 0;
       for (int32_t n = 1; n < 65536; ++n) {
         if (!seen[n]) continue;
-        for (int32_t t = 0; t <= n; ++t) buf[q++] = a + (b - a) * ((double)t / (double)n);
+        for (int32_t t = 0; t <= n; ++t) buf[q++] = t == n ? b : a + (b - a) * ((double)t / (double)n);
       }
       if (q) qsort(buf, (size_t)q, sizeof(double), cmp_double);
       int64_t u = 0;

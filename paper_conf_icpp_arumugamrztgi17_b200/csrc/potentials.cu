@@ -56,6 +56,11 @@ struct Params {
   const double* ring;        // padded ring, slot 0 node (-PAD, -PAD)
   const rp_frame* frames;    // [H]
   const double* amp;         // [H] analytic amplitudes
+  // Predictive-RP (R-26): merged partition lists per (cluster, j) and the point clusters;
+  // bp_off == nullptr selects the canonical roots
+  const double* bp;
+  const int64_t* bp_off;
+  const int32_t* cluster;
   // analytic source
   double sx0, sy0, swidth, sq, sbx, sby;
 };
@@ -741,7 +746,33 @@ __global__ void __launch_bounds__(32 * kWarps) k_integrate(
     const int item = order[idx];
     const int p = item / P.kmax, j = item % P.kmax;
     const double2 ab = AB[item];
-    const double A = ab.x, BA = __dsub_rn(ab.y, ab.x);
+    // roots of the item's trees: the n_root halves of its support [A, B] (canonical), or the
+    // intervals of its cluster's merged partition of S_j cut to [A, B] (Predictive-RP,
+    // Algorithm 1 lines 13-24, R-26); all lanes walk the list in step (uniform loads)
+    long long rt = 0, rt_end = 0;  // next interval [bp[rt], bp[rt + 1]], rt < rt_end
+    if (KIND == RP_SRC_GRID && P.bp_off) {
+      const long long li = (long long)P.cluster[p] * P.kmax + j;
+      rt = P.bp_off[li];
+      rt_end = P.bp_off[li + 1] - 1;
+      if (rt_end - rt < 1) {
+        rt = rt_end = 0;
+      } else {  // first interval that ends beyond A
+        long long lo = rt, hi = rt_end - 1;
+        while (lo < hi) {
+          const long long mid = (lo + hi) >> 1;
+          if (P.bp[mid + 1] > ab.x) hi = mid; else lo = mid + 1;
+        }
+        rt = lo;
+      }
+    }
+    const bool pred = rt < rt_end;
+    double A = ab.x, BA = __dsub_rn(ab.y, ab.x);
+    if (pred) {  // first non-empty cut interval (one exists: the list covers S_j, [A, B] in S_j)
+      for (; rt < rt_end; ++rt) {
+        const double a = fmax(P.bp[rt], ab.x), b = fmin(P.bp[rt + 1], ab.y);
+        if (a < b) { A = a; BA = __dsub_rn(b, a); ++rt; break; }
+      }
+    }
     __syncwarp();
     if (lane == 0) setup_item<KIND>(S.it, P, p, j);
     __syncwarp();
@@ -759,7 +790,7 @@ __global__ void __launch_bounds__(32 * kWarps) k_integrate(
     }
     int nseg = 0, nleaf = 0, capped = 0, ties = 0, maxlev = 0;
     unsigned evals = 0, nskip = 0;
-    int lev = P.n_root == 2 ? 1 : 0;
+    int lev = (P.n_root == 2 && !pred) ? 1 : 0;
     if (TM) { long long t = clock64(); ph[0] += t - t0; t0 = t; }
     long long ix = 0;
     for (;;) {
@@ -869,7 +900,18 @@ __global__ void __launch_bounds__(32 * kWarps) k_integrate(
         ++nleaf;
         s_phi += k0; s_ax += k1; s_ay += k2; s_err += err;
         while ((ix & 1) && lev > 0) { ix >>= 1; --lev; }
-        if (lev == 0) break;
+        if (lev == 0) {
+          if (!pred) break;
+          // next root interval of the merged partition, if any reaches into [A, B]
+          bool more = false;
+          for (; rt < rt_end && P.bp[rt] < ab.y; ++rt) {
+            const double a = fmax(P.bp[rt], ab.x), b = fmin(P.bp[rt + 1], ab.y);
+            if (a < b) { A = a; BA = __dsub_rn(b, a); ++rt; more = true; break; }
+          }
+          if (!more) break;
+          ix = 0;
+          continue;
+        }
         ++ix;
       } else {
         ++lev;
@@ -897,6 +939,7 @@ __global__ void k_reduce(int npts, int kmax, int kap, const uint16_t* __restrict
                          double* __restrict__ ay, double* __restrict__ err,
                          int32_t* __restrict__ nseg, double* __restrict__ shard,
                          uint16_t* __restrict__ cost, int32_t* __restrict__ nseg_pt,
+                         uint16_t* __restrict__ leaves,
                          unsigned long long* __restrict__ counters) {
   int p = blockIdx.x * blockDim.x + threadIdx.x;
   if (p >= npts) return;
@@ -908,6 +951,7 @@ __global__ void k_reduce(int npts, int kmax, int kap, const uint16_t* __restrict
     size_t id = (size_t)p * kmax + j;
     if (j >= kap || key[id] == 0xFFFF) {
       cost[id] = 0;
+      leaves[id] = 0;
       continue;
     }
     double4 v = val[id];
@@ -918,6 +962,7 @@ __global__ void k_reduce(int npts, int kmax, int kap, const uint16_t* __restrict
     ev += x.y;
     if ((int)x.x > ml) ml = (int)x.x;
     cost[id] = (uint16_t)(q.x < 0xFFFE ? q.x : 0xFFFE);
+    leaves[id] = (uint16_t)(q.y < 0xFFFF ? q.y : 0xFFFF);  // observed access pattern n_j(p)
   }
   if (shard) {
     double* r = shard + 6 * (size_t)row_of[p];
@@ -992,6 +1037,9 @@ int rp_alloc_potential_scratch(rp_ctx* ctx) {
   RP_CUDA(cudaMalloc(&ctx->sched_idx, nd * sizeof(int32_t)));
   RP_CUDA(cudaMalloc(&ctx->sched_order, nd * sizeof(int32_t)));
   RP_CUDA(cudaMalloc(&ctx->cost_prev, nd * sizeof(uint16_t)));
+  RP_CUDA(cudaMalloc(&ctx->leaves_prev, nd * sizeof(uint16_t)));
+  RP_CUDA(cudaMemset(ctx->leaves_prev, 0, nd * sizeof(uint16_t)));
+  RP_CUDA(cudaMalloc(&ctx->cluster_dev, npts * sizeof(int32_t)));
   RP_CUDA(cudaMemset(ctx->cost_prev, 0, nd * sizeof(uint16_t)));
   RP_CUDA(cudaMalloc(&ctx->item_val, nd * sizeof(double4)));
   RP_CUDA(cudaMalloc(&ctx->item_cnt, nd * sizeof(int4)));
@@ -1036,7 +1084,7 @@ static int launch_integrate(rp_ctx* ctx, const Params& P) {
 }
 
 template <int KIND>
-static int run_potentials(rp_ctx* ctx, const Params& P, int32_t rank, int32_t world,
+static int run_potentials(rp_ctx* ctx, Params P, int32_t rank, int32_t world,
                           double* phi, double* ax, double* ay, double* err, int32_t* nseg,
                           double* shard_out, int64_t cap) {
   cudaStream_t st = ctx->stream;
@@ -1089,6 +1137,15 @@ static int run_potentials(rp_ctx* ctx, const Params& P, int32_t rank, int32_t wo
                                               ctx->sched_order, (int)nd, 0, 16, st));
     }
     const int var = KIND != RP_SRC_GRID ? 0 : (P.interp == RP_INTERP_LAGRANGE3 ? 6 : ctx->eval_variant);
+    ctx->pred_info.active = 0;
+    if (KIND == RP_SRC_GRID && ctx->pred_on && ctx->have_leaves && !shard_out && var != 0) {
+      // Predictive-RP lines 1-12 on the host (R-26): forecast, partition, cluster, merge
+      int rc = rp_predictive_setup(ctx, P.kap);
+      if (rc) return rc;
+      P.bp = ctx->bp_dev;
+      P.bp_off = ctx->bp_off_dev;
+      P.cluster = ctx->cluster_dev;
+    }
     int rc2 = var == 4 ? launch_integrate<KIND, 4>(ctx, P)
               : var == 6 ? launch_integrate<KIND, 6>(ctx, P)
               : var == 7 ? launch_integrate<KIND, 7>(ctx, P)
@@ -1099,9 +1156,10 @@ static int run_potentials(rp_ctx* ctx, const Params& P, int32_t rank, int32_t wo
   k_reduce<<<(P.npts + 255) / 256, 256, 0, st>>>(
       P.npts, P.kmax, P.kap, ctx->sched_key, ctx->item_val, ctx->item_cnt, ctx->item_aux, owner,
       rank, row, world, phi, ax, ay, err, nseg, shard_out, ctx->cost_prev, ctx->nseg_prev_pt,
-      ctx->counters);
+      ctx->leaves_prev, ctx->counters);
   RP_CHECK_LAUNCH();
   ctx->has_forecast = 1;
+  ctx->have_leaves = shard_out ? 0 : 1;
   return RP_OK;
 }
 
@@ -1121,6 +1179,7 @@ int rp_potentials_impl(rp_ctx* ctx, int kind, const double src[6], int32_t rank,
   P.cdt = c.c * c.dt; P.tau = c.tau; P.R = (double)P.kap * P.cdt;
   P.slot_doubles = ctx->slot_doubles; P.ring = ctx->ring; P.frames = ctx->frames_dev;
   P.amp = ctx->amp_dev;
+  P.bp = nullptr; P.bp_off = nullptr; P.cluster = nullptr;
   P.sx0 = src ? src[0] : 0; P.sy0 = src ? src[1] : 0; P.swidth = src ? src[2] : 0;
   P.sq = src ? src[3] : 0; P.sbx = src ? src[4] : 0; P.sby = src ? src[5] : 0;
   int rc;

@@ -54,7 +54,7 @@ void free_all(rp_ctx* c) {
                   c->item_val, c->item_cnt, c->item_aux, c->counters, c->amp_dev, c->trig_full,
                   c->point_key, c->point_key_sorted, c->point_idx, c->point_order,
                   c->point_owner, c->nseg_prev_pt, c->hx_d, c->hy_d, c->hux_d, c->huy_d,
-                  c->mesh_d};
+                  c->mesh_d, c->leaves_prev, c->cluster_dev, c->bp_off_dev, c->bp_dev};
   for (void* p : ptrs)
     if (p) cudaFree(p);
   for (auto& r : c->prof) {
@@ -94,6 +94,29 @@ int rp_set_schedule(rp_ctx* ctx, int32_t policy, int32_t k) {
     return rp_fail(ctx, RP_EINVAL, "set_schedule: k must be 1, 5, 9 or 25");
   ctx->sched_policy = policy;
   ctx->sched_k = policy == RP_SCHED_KNN ? k : 1;
+  return RP_OK;
+}
+
+int rp_set_predictive(rp_ctx* ctx, int32_t enable, int32_t knn, int32_t n_clusters,
+                      int32_t max_iters) {
+  if (!ctx) return RP_EINVAL;
+  if (knn != 1 && knn != 5 && knn != 9 && knn != 25)
+    return rp_fail(ctx, RP_EINVAL, "set_predictive: k must be 1, 5, 9 or 25");
+  if (n_clusters < 0 || max_iters < 1) return rp_fail(ctx, RP_EINVAL, "set_predictive: bad args");
+  ctx->pred_on = enable ? 1 : 0;
+  ctx->pred_knn = knn;
+  ctx->pred_m = n_clusters;
+  ctx->pred_iters = max_iters;
+  return RP_OK;
+}
+
+int rp_predictive_info_read(rp_ctx* ctx, rp_predictive_info* out, int32_t* clusters_host) {
+  if (!ctx || !out) return RP_EINVAL;
+  *out = ctx->pred_info;
+  if (clusters_host) {
+    if (!ctx->pred_info.active) return rp_fail(ctx, RP_ESTATE, "predictive_info: no forecast partition yet");
+    memcpy(clusters_host, ctx->cluster_host.data(), ctx->cluster_host.size() * sizeof(int32_t));
+  }
   return RP_OK;
 }
 
@@ -266,6 +289,7 @@ int rp_compute_potentials_shard(rp_ctx* ctx, int32_t rank, int32_t world, double
   if (!ctx) return RP_EINVAL;
   if (world < 1 || rank < 0 || rank >= world || !shard_out || cap < rp_shard_capacity(ctx, world))
     return rp_fail(ctx, RP_EINVAL, "potentials_shard: bad rank/world/cap");
+  if (ctx->pred_on) return rp_fail(ctx, RP_EINVAL, "potentials_shard: Predictive-RP is single-call only");
   return rp_potentials_impl(ctx, RP_SRC_GRID, nullptr, rank, world, nullptr, nullptr, nullptr,
                             nullptr, nullptr, shard_out, cap, n_out, info);
 }

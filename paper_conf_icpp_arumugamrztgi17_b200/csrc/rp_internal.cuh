@@ -63,6 +63,17 @@ struct rp_ctx {
   int sched_k = 9;                  // kNN neighbours
   int eval_variant = 4;             // integrator evaluation loop (development A/B: RP_EVAL)
 
+  // Predictive-RP variant (rp_set_predictive, DESIGN R-26)
+  int pred_on = 0, pred_knn = 9, pred_m = 0, pred_iters = 20;
+  uint16_t* leaves_prev = nullptr;  // [npts * kappa_max] accepted segments of the last call
+  int have_leaves = 0;
+  int32_t* cluster_dev = nullptr;   // [npts] k-means cluster of every point
+  int64_t* bp_off_dev = nullptr;    // [m * kappa_max + 1] merged-list offsets
+  double* bp_dev = nullptr;         // merged breakpoints
+  int64_t bp_cap = 0, off_cap = 0;
+  std::vector<int32_t> cluster_host;
+  rp_predictive_info pred_info{};
+
   // sharding scratch
   int32_t* point_key = nullptr;     // per point predicted work key
   int32_t* point_key_sorted = nullptr;
@@ -176,3 +187,4 @@ int rp_push_impl(rp_ctx* ctx, double* x, double* y, double* ux, double* uy, int6
 int rp_scatter_impl(rp_ctx* ctx, const double* shards, int32_t world, int64_t cap,
                     double* phi, double* ax, double* ay, double* err, int32_t* nseg);
 int rp_alloc_potential_scratch(rp_ctx* ctx);
+int rp_predictive_setup(rp_ctx* ctx, int kap);

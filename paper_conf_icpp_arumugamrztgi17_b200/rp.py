@@ -64,6 +64,14 @@ class rp_potential_info(C.Structure):
         return {k: getattr(self, k) for k, _ in self._fields_}
 
 
+class rp_predictive_info(C.Structure):
+    _fields_ = [("active", C.c_int32), ("clusters", C.c_int32), ("kmeans_passes", C.c_int32),
+                ("pad", C.c_int32), ("breakpoints", C.c_int64), ("host_ms", C.c_double)]
+
+    def as_dict(self) -> dict:
+        return {k: getattr(self, k) for k, _ in self._fields_ if k != "pad"}
+
+
 if not os.path.exists(LIB_PATH):
     raise ImportError(f"librp.so not built at {LIB_PATH}: run "
                       "`python -m paper_conf_icpp_arumugamrztgi17_b200.build` (no CPU fallback)")
@@ -78,6 +86,8 @@ _SIG = {
     "rp_launch_count": (_i64, [_vp]),
     "rp_profile_enable": (C.c_int, [_vp, _i32]),
     "rp_set_schedule": (C.c_int, [_vp, _i32, _i32]),
+    "rp_set_predictive": (C.c_int, [_vp, _i32, _i32, _i32, _i32]),
+    "rp_predictive_info_read": (C.c_int, [_vp, _P(rp_predictive_info), _vp]),
     "rp_profile_read": (C.c_int, [_vp, _P(rp_profile)]),
     "rp_create": (C.c_int, [_P(rp_config), _P(_vp)]),
     "rp_destroy": (None, [_vp]),
@@ -185,6 +195,23 @@ def rp_launch_count(ctx) -> int:
 
 def rp_set_schedule(ctx, policy, k=9) -> None:
     _check(_lib.rp_set_schedule(ctx, int(policy), int(k)), ctx, "rp_set_schedule")
+
+
+def rp_set_predictive(ctx, enable=True, knn=9, n_clusters=0, max_iters=20) -> None:
+    _check(_lib.rp_set_predictive(ctx, int(bool(enable)), int(knn), int(n_clusters),
+                                  int(max_iters)), ctx, "rp_set_predictive")
+
+
+def rp_predictive_info_read(ctx, npts=None):
+    """Returns rp_predictive_info; with npts = nx * ny also the int32 [npts] point clusters."""
+    info = rp_predictive_info()
+    if npts is None:
+        _check(_lib.rp_predictive_info_read(ctx, C.byref(info), None), ctx, "rp_predictive_info_read")
+        return info
+    out = np.zeros(int(npts), dtype=np.int32)
+    _check(_lib.rp_predictive_info_read(ctx, C.byref(info), out.ctypes.data_as(_vp)), ctx,
+           "rp_predictive_info_read")
+    return info, out
 
 
 def rp_profile_enable(ctx, enable=True) -> None:

@@ -1,0 +1,93 @@
+"""GPU parity of the Predictive-RP variant (the paper's Algorithm 1 COMPUTE-POTENTIALS,
+P:110-166; DESIGN reading R-26) through the C ABI: the previous step runs the canonical
+tree on both sides (each side records its own observed access pattern n_j(p)); the next step
+forecasts, clusters, merges and integrates over the merged partitions on both sides.
+
+Bars: k-means clusters identical; potentials within 1e-11 * max(|phi|, |A|) per point with
+equal segment counts; the results stay within tau of the canonical tree's.
+"""
+import numpy as np
+import pytest
+
+import workloads as W
+from tests import gpu_util as G
+from tests.test_gpu_parity import _bend_small, _deposit_rigid_ring
+
+pytestmark = pytest.mark.gpu
+
+
+def _two_steps(cfg, rings, n_pre, knn, m, pts=None):
+    from paper_conf_icpp_arumugamrztgi17_b200 import rp
+    (k0, ring0, fr0), (k1, ring1, fr1) = rings
+    npts = cfg.nx * cfg.ny
+    allp = np.arange(npts)
+    pts = allp if pts is None else pts
+    o0 = G.oracle_problem(cfg, ring0, fr0, k0, n_pre)
+    canon0, leaves0 = o0.potentials_items(allp)
+    o1 = G.oracle_problem(cfg, ring1, fr1, k1, n_pre)
+    pred1, clusters1, _, passes = o1.potentials_predictive(leaves0, pts, knn=knn, m=m)
+    canon1 = o1.potentials(pts)
+    ctx = G.make_ctx(cfg)
+    try:
+        rp.rp_set_predictive(ctx, True, knn, m, 20)
+        G.load_state(ctx, cfg, k0, n_pre, ring0, fr0)
+        gpu0, _ = G.gpu_potentials(ctx, npts)  # no previous pattern yet: canonical tree
+        assert rp.rp_predictive_info_read(ctx).active == 0
+        fail, worst, _ = G.compare_potentials(gpu0, canon0, allp)
+        assert not fail.any(), worst
+        G.load_state(ctx, cfg, k1, n_pre, ring1, fr1)
+        gpu1, info = G.gpu_potentials(ctx, npts)
+        pinfo, clusters = rp.rp_predictive_info_read(ctx, npts)
+    finally:
+        rp.rp_destroy(ctx)
+    assert pinfo.active == 1 and pinfo.kmeans_passes == passes
+    np.testing.assert_array_equal(clusters, clusters1)
+    fail, worst, nties = G.compare_potentials(gpu1, pred1, pts)
+    assert not fail.any(), (np.nonzero(fail)[0][:10], worst)
+    assert info.segments == int(pred1["nseg"].sum()) or len(pts) < npts
+    # forecast-dependent, but within the tolerance of the canonical result
+    scale = np.abs(canon1["phi"]).max()
+    assert np.abs(pred1["phi"] - canon1["phi"]).max() <= 2 * cfg.tau
+    assert np.abs(gpu1["phi"][pts] - canon1["phi"]).max() <= 2 * cfg.tau
+    assert (pred1["nseg"] != canon1["nseg"]).any()
+    return pinfo, scale
+
+
+def test_predictive_static_cfg1_full_mesh():
+    """Config 1 (32x32, static frame, rigid history): two consecutive steps."""
+    cfg = W.config(1)
+    ring, _ = _deposit_rigid_ring(cfg)
+    fr = W.ring_frames(cfg, 0)
+    fr1 = W.ring_frames(cfg, 1)
+    _two_steps(cfg, [(0, ring, fr), (1, ring, fr1)], cfg.n_pre, knn=9, m=0)
+
+
+@pytest.mark.parametrize("knn,m", [(9, 0), (1, 12), (25, 40)])
+def test_predictive_bend_small_full_mesh(knn, m):
+    """Moving frames (bend), node-sampled history with a time-varying amplitude."""
+    cfg = _bend_small(16, 24)
+    rings = []
+    for k in (5, 6):
+        ring = W.node_gaussian_ring(cfg, k=k, beta=(cfg.beta0, 0.01),
+                                    amp_of_level=lambda l: 1.0 + 0.01 * l)
+        rings.append((k, ring, W.ring_frames(cfg, k)))
+    _two_steps(cfg, rings, cfg.n_pre, knn=knn, m=m)
+
+
+def test_predictive_refuses_the_shard_path():
+    from paper_conf_icpp_arumugamrztgi17_b200 import rp
+    cfg = W.config(1)
+    ctx = G.make_ctx(cfg)
+    try:
+        rp.rp_set_predictive(ctx, True)
+        with pytest.raises(rp.RpError):
+            rp.rp_set_predictive(ctx, True, knn=4)
+        import torch
+        ring, _ = _deposit_rigid_ring(cfg)
+        G.load_state(ctx, cfg, 0, cfg.n_pre, ring, W.ring_frames(cfg, 0))
+        sh = torch.zeros((rp.rp_shard_capacity(ctx, 2), 6), dtype=torch.float64, device="cuda")
+        with pytest.raises(rp.RpError) as e:
+            rp.rp_compute_potentials_shard(ctx, 0, 2, sh)
+        assert e.value.code == -1
+    finally:
+        rp.rp_destroy(ctx)
