@@ -530,6 +530,57 @@ def test_potentials_bend_cfg3_full_size_sampled(torch):
         rp.rp_destroy(ctx)
 
 
+@pytest.mark.slow
+def test_potentials_bend_cfg4_full_size_sampled(torch):
+    """Config 4 (256x256, 1e8 particles, full history kappa = 1000: BASELINE.json configs[3])
+    through the product path on one GPU; the oracle computes 16 stratified points from its own
+    deposit of the same 1e8 particles (2.1 GB ring on the host)."""
+    from paper_conf_icpp_arumugamrztgi17_b200 import rp
+    cfg = W.config(4)
+    ring, (x, y, ux, uy, q) = _deposit_rigid_ring(cfg)
+    pts = W.sample_points(cfg.nx, cfg.ny, 16, seed=13)
+    orc = G.oracle_problem(cfg, ring, W.ring_frames(cfg, 0), 0, cfg.n_pre).potentials(pts)
+    del ring
+    ctx = G.make_ctx(cfg)
+    try:
+        rp.rp_history_init(ctx, cfg.n_pre, W.frames(cfg, range(-cfg.n_pre, 0)), None, True)
+        xd, yd, uxd, uyd = _dev_arrays(torch, x, y, ux, uy)
+        del x, y, ux, uy
+        rp.rp_deposit_step(ctx, xd, yd, uxd, uyd, q, W.frame(cfg, 0))
+        del xd, yd, uxd, uyd
+        gpu, info = G.gpu_potentials(ctx, cfg.nx * cfg.ny)
+        fail, worst, _ = G.compare_potentials(gpu, orc, pts)
+        assert not fail.any(), (pts[fail][:10], worst)
+        assert info.kappa == cfg.kappa_max
+    finally:
+        rp.rp_destroy(ctx)
+
+
+@pytest.mark.slow
+def test_potentials_bend_cfg5_full_size_sampled(torch):
+    """Config 5 (512x512, 1e8 particles, kappa = 2000: BASELINE.json configs[4]) on one GPU
+    (76 GB of HBM), the oracle on 12 stratified points with a 16.8 GB host ring."""
+    from paper_conf_icpp_arumugamrztgi17_b200 import rp
+    cfg = W.config(5)
+    ring, (x, y, ux, uy, q) = _deposit_rigid_ring(cfg)
+    pts = W.sample_points(cfg.nx, cfg.ny, 12, seed=17)
+    orc = G.oracle_problem(cfg, ring, W.ring_frames(cfg, 0), 0, cfg.n_pre).potentials(pts)
+    del ring
+    ctx = G.make_ctx(cfg)
+    try:
+        rp.rp_history_init(ctx, cfg.n_pre, W.frames(cfg, range(-cfg.n_pre, 0)), None, True)
+        xd, yd, uxd, uyd = _dev_arrays(torch, x, y, ux, uy)
+        del x, y, ux, uy
+        rp.rp_deposit_step(ctx, xd, yd, uxd, uyd, q, W.frame(cfg, 0))
+        del xd, yd, uxd, uyd
+        gpu, info = G.gpu_potentials(ctx, cfg.nx * cfg.ny)
+        fail, worst, _ = G.compare_potentials(gpu, orc, pts)
+        assert not fail.any(), (pts[fail][:10], worst)
+        assert info.kappa == cfg.kappa_max
+    finally:
+        rp.rp_destroy(ctx)
+
+
 @pytest.mark.parametrize("policy,k", [(0, 1), (2, 9), (2, 25), (2, 5)])
 def test_schedule_policies_bit_identical(torch, policy, k):
     """The forecast (paper's predictor g) only orders the work: every policy gives
