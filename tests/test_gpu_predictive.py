@@ -62,10 +62,12 @@ def test_predictive_static_cfg1_full_mesh():
     _two_steps(cfg, [(0, ring, fr), (1, ring, fr1)], cfg.n_pre, knn=9, m=0)
 
 
-@pytest.mark.parametrize("knn,m", [(9, 0), (1, 12), (25, 40)])
-def test_predictive_bend_small_full_mesh(knn, m):
-    """Moving frames (bend), node-sampled history with a time-varying amplitude."""
+@pytest.mark.parametrize("knn,m,rule", [(9, 0, 0), (1, 12, 0), (25, 40, 0), (9, 0, 1)])
+def test_predictive_bend_small_full_mesh(knn, m, rule):
+    """Moving frames (bend), node-sampled history with a time-varying amplitude; GK15 and the
+    paper's own Simpson rule (R-22), which Algorithm 1's RP-QUADRULE names."""
     cfg = _bend_small(16, 24)
+    cfg.rule = rule
     rings = []
     for k in (5, 6):
         ring = W.node_gaussian_ring(cfg, k=k, beta=(cfg.beta0, 0.01),
