@@ -216,6 +216,15 @@ int rp_save_state(rp_ctx* ctx, int32_t* k_out, double* ring_dev, rp_frame* frame
 /* Bin index of every particle of the last rp_deposit (-1 = lost), [n]. */
 int rp_debug_bins(rp_ctx* ctx, int32_t* bins_dev, int64_t n);
 
+/* The support clip of the last rp_compute_potentials call (step a5, R-5: per (point p,
+ * subregion j) the r'-interval [A, B] of S_j where the circle about p meets the support
+ * rectangle at the retarded time, by 64-step bisection on squared distances): copies
+ * npts * kappa_max pairs (A, B), p-major, into ab_dev (DEVICE, caller-owned, 2 * n doubles
+ * with n = nx * ny * history_depth); (0, 0) for items without support or with j >= kappa.
+ * The arithmetic mirrors the oracle's operation order with IEEE round-to-nearest intrinsics,
+ * so the limits are bit-identical to it.  RP_ESTATE before the first potentials call. */
+int rp_debug_clip(rp_ctx* ctx, double* ab_dev, int64_t n);
+
 /* Test hook: potentials with an analytic source in place of the grid:
  * kind = RP_SRC_GAUSS (centre (x0,y0) frame-local, width = sigma, q = Q) or RP_SRC_DISK
  * (width = radius, q = surface density); (bx, by) = beta; amp_host[H] per-slot amplitudes

@@ -421,6 +421,16 @@ int rp_debug_bins(rp_ctx* ctx, int32_t* bins_dev, int64_t n) {
   return RP_OK;
 }
 
+int rp_debug_clip(rp_ctx* ctx, double* ab_dev, int64_t n) {
+  if (!ctx) return RP_EINVAL;
+  const int64_t want = (int64_t)ctx->cfg.nx * ctx->cfg.ny * ctx->cfg.history_depth;
+  if (!ab_dev || n != want) return rp_fail(ctx, RP_EINVAL, "debug_clip: n must be nx*ny*history_depth");
+  if (!ctx->has_forecast) return rp_fail(ctx, RP_ESTATE, "debug_clip: no potentials call yet");
+  RP_CUDA(cudaMemcpyAsync(ab_dev, ctx->clipAB, (size_t)n * sizeof(double2), cudaMemcpyDeviceToDevice,
+                          ctx->stream));
+  return RP_OK;
+}
+
 int rp_debug_potentials_analytic(rp_ctx* ctx, int32_t kind, double x0, double y0, double width,
                                  double q, double bx, double by, const double* amp_host,
                                  double* phi, double* ax, double* ay, double* err, int32_t* nseg,

@@ -111,6 +111,7 @@ _SIG = {
     "rp_load_state": (C.c_int, [_vp, _i32, _i32, _P(rp_frame), _vp]),
     "rp_save_state": (C.c_int, [_vp, _P(_i32), _vp, _P(rp_frame)]),
     "rp_debug_bins": (C.c_int, [_vp, _vp, _i64]),
+    "rp_debug_clip": (C.c_int, [_vp, _vp, _i64]),
     "rp_debug_potentials_analytic": (C.c_int, [_vp, _i32, _d, _d, _d, _d, _d, _d, _vp, _vp, _vp,
                                                _vp, _vp, _vp, _P(rp_potential_info)]),
 }
@@ -346,6 +347,11 @@ def rp_save_state(ctx, ring=None, H=None):
     if fa is not None:
         frames = np.array([[f.ox, f.oy, f.cos_psi, f.sin_psi] for f in fa])
     return k.value, frames
+
+
+def rp_debug_clip(ctx, ab) -> None:
+    """ab: float64 CUDA tensor of nx*ny*history_depth*2 elements ((A, B) per item)."""
+    _check(_lib.rp_debug_clip(ctx, _f64(ab, "ab"), ab.numel() // 2), ctx, "rp_debug_clip")
 
 
 def rp_debug_bins(ctx, bins) -> None:

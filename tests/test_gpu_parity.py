@@ -235,6 +235,48 @@ def test_potentials_bend_small_full_mesh_two_steps(torch, rule, interp):
         rp.rp_destroy(ctx)
 
 
+@pytest.mark.parametrize("which", ["bend_small", "cfg2_sampled"])
+def test_support_clip_bit_exact(torch, which):
+    """Step a5 (R-5): the GPU's per-(point, subregion) support [A, B] equals the oracle's clip
+    bit for bit (both follow the same operation order in IEEE round-to-nearest), including
+    which items are empty."""
+    from paper_conf_icpp_arumugamrztgi17_b200 import rp
+    if which == "bend_small":
+        cfg = _bend_small()
+        k = 5
+        ring = W.node_gaussian_ring(cfg, k=k, beta=(cfg.beta0, 0.01),
+                                    amp_of_level=lambda l: 1.0 + 0.01 * l)
+        frames = W.ring_frames(cfg, k)
+    else:
+        cfg = W.config(2)
+        k = 0
+        ring, _ = _deposit_rigid_ring(cfg, n=20_000, seed=3)
+        frames = W.ring_frames(cfg, 0)
+    ctx = G.make_ctx(cfg)
+    try:
+        G.load_state(ctx, cfg, k, cfg.n_pre, ring, frames)
+        gpu, info = G.gpu_potentials(ctx, cfg.nx * cfg.ny)
+        ab = torch.zeros(cfg.nx * cfg.ny * cfg.kappa_max * 2, dtype=torch.float64, device="cuda")
+        rp.rp_debug_clip(ctx, ab)
+        ab = ab.cpu().numpy().reshape(cfg.nx * cfg.ny, cfg.kappa_max, 2)
+    finally:
+        rp.rp_destroy(ctx)
+    P = G.oracle_problem(cfg, ring, frames, k, cfg.n_pre)
+    kap = P.kappa()
+    assert kap == info.kappa and kap > 0
+    rng = np.random.default_rng(1)
+    items = [(p, j) for p in range(cfg.nx * cfg.ny) for j in range(kap)]
+    if len(items) > 30_000:
+        items = [items[i] for i in rng.choice(len(items), 30_000, replace=False)]
+    nonempty = 0
+    for p, j in items:
+        c = P.clip(*P.mesh_point(p % cfg.nx, p // cfg.nx), j)
+        want = (0.0, 0.0) if c is None else c
+        assert ab[p, j, 0] == want[0] and ab[p, j, 1] == want[1], (p, j, ab[p, j], c)
+        nonempty += c is not None
+    assert nonempty > 100
+
+
 @pytest.mark.parametrize("variant", [dict(n_root=1), dict(max_depth=5), dict(n_theta=16),
                                      dict(rule=1), dict(rule=1, n_root=1),
                                      dict(interp=1, max_depth=12),
