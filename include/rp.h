@@ -286,11 +286,12 @@ typedef struct {
   double append_ms;        /* rank-order sum into the ring                                      */
   double clip_ms;          /* support clip + schedule keys                                      */
   double sort_ms;          /* schedule sort (CUB)                                               */
-  double integrate_ms;     /* the GK15 integrator (dominant kernel)                             */
+  double integrate_ms;     /* the GK15 integrator (dominant kernel): items + subtree units + merge */
   double reduce_ms;        /* per-point reduction                                               */
   double fields_ms;
   double push_ms;
-  int64_t integrate_launches;
+  int64_t integrate_launches;  /* integrator calls (each: the item launch, then the units')  */
+  double units_ms;         /* of integrate_ms: the subtree-unit launch, its sort and merge      */
 } rp_profile;
 
 /* enable != 0 starts (and resets) event timing; 0 stops it.  Adds two event records per

@@ -42,7 +42,9 @@ __constant__ double c_wg[4] = {
     0.381830050505118944950369775488975, 0.417959183673469387755102040816327};
 
 enum : int { C_ITEMS = 0, C_NEXT = 1, C_EVALS = 2, C_SEGS = 3, C_LEAVES = 4, C_CAPPED = 5,
-             C_TIES = 6, C_MAXLEV = 7, C_NODES = 8, C_NOUT = 9, C_SKIP = 10, C_COUNT = 16 };
+             C_TIES = 6, C_MAXLEV = 7, C_NODES = 8, C_NOUT = 9, C_SKIP = 10, C_UNITS = 11,
+             C_NEXT_U = 12, C_UOVF = 13, C_COUNT = 16 };
+constexpr int kUnitShift = 20;  // unit key = item << 20 | index of the subtree root at its level
 
 constexpr double kTwoPi = 6.283185307179586476925286766559;
 constexpr int kMaxArcs = 8;
@@ -61,6 +63,13 @@ struct Params {
   const double* bp;
   const int64_t* bp_off;
   const int32_t* cluster;
+  // subtree work units (deep trees split at a fixed level, see k_integrate)
+  int split_level;                  // 0: off
+  long long unit_cap;
+  unsigned long long* unit_key;     // [unit_cap] item << kUnitShift | ix
+  double4* unit_val;
+  int4* unit_cnt;
+  uint2* unit_aux;
   // analytic source
   double sx0, sy0, swidth, sq, sbx, sby;
 };
@@ -720,7 +729,15 @@ __device__ unsigned long long g_phase[8];  // development: per-phase SM cycles (
 
 // VAR 0: one pass per round (eval_nodes); VAR 4: software-pipelined rounds; VAR 7: VAR 4 with
 // per-phase clock accounting (development)
-template <int KIND, int VAR>
+// UNIT = false: the (point, subregion) items in forecast order.  With P.split_level = L > 0
+// a segment at level L - 1 that splits does not descend: its two children become subtree work
+// units (appended to P.unit_key) and the walk goes on as if the segment were finished.  The
+// tree is the canonical one -- only nodes it reaches are deferred -- but the deep near-field
+// trees (thousands of segments, fanning out below level ~8) no longer bound the kernel (and an
+// N-GPU shard) by one warp's walk.  UNIT = true: the units, each walked from its root at
+// level L until the walk climbs back to L; per-unit results are merged into their items in
+// (item, subtree) order (k_merge_units), so results are deterministic for any N.
+template <int KIND, int VAR, bool UNIT = false>
 __global__ void __launch_bounds__(32 * kWarps) k_integrate(
     Params P, const int32_t* __restrict__ order, const double2* __restrict__ AB,
     const double2* __restrict__ trig_full, double4* __restrict__ item_val,
@@ -730,7 +747,7 @@ __global__ void __launch_bounds__(32 * kWarps) k_integrate(
   WarpSmem* smem = reinterpret_cast<WarpSmem*>(smem_raw);
   const int lane = threadIdx.x & 31;
   WarpSmem& S = smem[kWarps == 1 ? 0 : (threadIdx.x >> 5)];
-  const unsigned long long n_items = counters[C_ITEMS];
+  const unsigned long long n_items = counters[UNIT ? C_UNITS : C_ITEMS];
   const int N = P.n_theta;
   const double Nd = (double)N;
   const double wfull = kTwoPi / Nd;
@@ -740,17 +757,18 @@ __global__ void __launch_bounds__(32 * kWarps) k_integrate(
   long long t0 = TM ? clock64() : 0;
   for (;;) {
     unsigned long long idx = 0;
-    if (lane == 0) idx = atomicAdd(&counters[C_NEXT], 1ULL);
+    if (lane == 0) idx = atomicAdd(&counters[UNIT ? C_NEXT_U : C_NEXT], 1ULL);
     idx = __shfl_sync(0xffffffffu, idx, 0);
     if (idx >= n_items) break;
-    const int item = order[idx];
+    const unsigned long long ukey = UNIT ? P.unit_key[idx] : 0ULL;
+    const int item = UNIT ? (int)(ukey >> kUnitShift) : order[idx];
     const int p = item / P.kmax, j = item % P.kmax;
     const double2 ab = AB[item];
     // roots of the item's trees: the n_root halves of its support [A, B] (canonical), or the
     // intervals of its cluster's merged partition of S_j cut to [A, B] (Predictive-RP,
     // Algorithm 1 lines 13-24, R-26); all lanes walk the list in step (uniform loads)
     long long rt = 0, rt_end = 0;  // next interval [bp[rt], bp[rt + 1]], rt < rt_end
-    if (KIND == RP_SRC_GRID && P.bp_off) {
+    if (KIND == RP_SRC_GRID && P.bp_off && !UNIT) {
       const long long li = (long long)P.cluster[p] * P.kmax + j;
       rt = P.bp_off[li];
       rt_end = P.bp_off[li + 1] - 1;
@@ -790,9 +808,10 @@ __global__ void __launch_bounds__(32 * kWarps) k_integrate(
     }
     int nseg = 0, nleaf = 0, capped = 0, ties = 0, maxlev = 0;
     unsigned evals = 0, nskip = 0;
-    int lev = (P.n_root == 2 && !pred) ? 1 : 0;
+    int lev = UNIT ? P.split_level : ((P.n_root == 2 && !pred) ? 1 : 0);
+    const int rlev = UNIT ? P.split_level : 0;  // the walk ends when it climbs back here
     if (TM) { long long t = clock64(); ph[0] += t - t0; t0 = t; }
-    long long ix = 0;
+    long long ix = UNIT ? (long long)(ukey & ((1ULL << kUnitShift) - 1)) : 0;
     for (;;) {
       const double fa = ldexp((double)ix, -lev), fb = ldexp((double)(ix + 1), -lev);
       const double a = __dadd_rn(A, __dmul_rn(BA, fa)), b = __dadd_rn(A, __dmul_rn(BA, fb));
@@ -895,13 +914,33 @@ __global__ void __launch_bounds__(32 * kWarps) k_integrate(
       err = fmax(err, fabs(k2 - g2));
       const double tol = __ddiv_rn(__dmul_rn(P.tau, ldexp(BA, -lev)), P.R);
       if (fabs(err - tol) / tol < 1e-9) ++ties;
+      bool finished = false;
       if (err <= tol || lev >= P.max_depth) {
         if (!(err <= tol)) ++capped;
         ++nleaf;
         s_phi += k0; s_ax += k1; s_ay += k2; s_err += err;
-        while ((ix & 1) && lev > 0) { ix >>= 1; --lev; }
-        if (lev == 0) {
-          if (!pred) break;
+        finished = true;
+      } else if (!UNIT && P.split_level > 0 && lev + 1 == P.split_level) {
+        // defer both children as subtree units (falls back to descending if the unit list is
+        // full, flagged in counters[C_UOVF])
+        unsigned long long u = 0;
+        if (lane == 0) u = atomicAdd(&counters[C_UNITS], 2ULL);
+        u = __shfl_sync(0xffffffffu, u, 0);
+        if ((long long)u + 1 < P.unit_cap) {
+          if (lane == 0) {
+            const unsigned long long base = (unsigned long long)item << kUnitShift;
+            P.unit_key[u] = base | (unsigned long long)(2 * ix);
+            P.unit_key[u + 1] = base | (unsigned long long)(2 * ix + 1);
+          }
+          finished = true;
+        } else if (lane == 0) {
+          atomicExch(&counters[C_UOVF], 1ULL);
+        }
+      }
+      if (finished) {
+        while ((ix & 1) && lev > rlev) { ix >>= 1; --lev; }
+        if (lev == rlev) {
+          if (UNIT || !pred) break;
           // next root interval of the merged partition, if any reaches into [A, B]
           bool more = false;
           for (; rt < rt_end && P.bp[rt] < ab.y; ++rt) {
@@ -920,14 +959,50 @@ __global__ void __launch_bounds__(32 * kWarps) k_integrate(
       if (TM) { long long t = clock64(); ph[5] += t - t0; t0 = t; }
     }
     if (lane == 0) {
-      item_val[item] = make_double4(s_phi, s_ax, s_ay, s_err);
-      item_cnt[item] = make_int4(nseg, nleaf, capped, ties);
-      item_aux[item] = make_uint2((unsigned)maxlev, evals);
+      const size_t o = UNIT ? (size_t)idx : (size_t)item;
+      (UNIT ? P.unit_val : item_val)[o] = make_double4(s_phi, s_ax, s_ay, s_err);
+      (UNIT ? P.unit_cnt : item_cnt)[o] = make_int4(nseg, nleaf, capped, ties);
+      (UNIT ? P.unit_aux : item_aux)[o] = make_uint2((unsigned)maxlev, evals);
       if (nskip) atomicAdd(&counters[C_SKIP], (unsigned long long)nskip);
     }
   }
   if (TM && lane == 0)
     for (int i = 0; i < 6; ++i) atomicAdd(&g_phase[i], ph[i]);
+}
+
+// ------------------------------------------------------------- subtree units
+__global__ void k_iota(int32_t* a, long long n) {
+  const long long i = blockIdx.x * (long long)blockDim.x + threadIdx.x;
+  if (i < n) a[i] = (int32_t)i;
+}
+
+// Add every item's units to its own partial result, in (item, subtree index) order: one
+// thread per item (the first sorted position of its run), so the sums are deterministic.
+__global__ void k_merge_units(long long n, const unsigned long long* __restrict__ skey,
+                              const int32_t* __restrict__ perm, const double4* __restrict__ uv,
+                              const int4* __restrict__ uc, const uint2* __restrict__ ua,
+                              double4* __restrict__ item_val, int4* __restrict__ item_cnt,
+                              uint2* __restrict__ item_aux) {
+  const long long i = blockIdx.x * (long long)blockDim.x + threadIdx.x;
+  if (i >= n) return;
+  const unsigned long long it = skey[i] >> kUnitShift;
+  if (i > 0 && (skey[i - 1] >> kUnitShift) == it) return;
+  double4 v = item_val[it];
+  int4 c = item_cnt[it];
+  uint2 a = item_aux[it];
+  for (long long k = i; k < n && (skey[k] >> kUnitShift) == it; ++k) {
+    const int u = perm[k];
+    const double4 w = uv[u];
+    const int4 d = uc[u];
+    const uint2 b = ua[u];
+    v.x += w.x; v.y += w.y; v.z += w.z; v.w += w.w;
+    c.x += d.x; c.y += d.y; c.z += d.z; c.w += d.w;
+    a.x = max(a.x, b.x);
+    a.y += b.y;
+  }
+  item_val[it] = v;
+  item_cnt[it] = c;
+  item_aux[it] = a;
 }
 
 // ------------------------------------------------------------- k_reduce
@@ -1040,6 +1115,19 @@ int rp_alloc_potential_scratch(rp_ctx* ctx) {
   RP_CUDA(cudaMalloc(&ctx->leaves_prev, nd * sizeof(uint16_t)));
   RP_CUDA(cudaMemset(ctx->leaves_prev, 0, nd * sizeof(uint16_t)));
   RP_CUDA(cudaMalloc(&ctx->cluster_dev, npts * sizeof(int32_t)));
+  if (ctx->split_level > 0) {
+    const long long cap = std::max<long long>(1LL << 22, 64LL * (long long)npts) & ~1LL;
+    ctx->unit_cap = cap;
+    RP_CUDA(cudaMalloc(&ctx->unit_key, cap * sizeof(unsigned long long)));
+    RP_CUDA(cudaMalloc(&ctx->unit_key_sorted, cap * sizeof(unsigned long long)));
+    RP_CUDA(cudaMalloc(&ctx->unit_iota, cap * sizeof(int32_t)));
+    RP_CUDA(cudaMalloc(&ctx->unit_perm, cap * sizeof(int32_t)));
+    RP_CUDA(cudaMalloc(&ctx->unit_val, cap * sizeof(double4)));
+    RP_CUDA(cudaMalloc(&ctx->unit_cnt, cap * sizeof(int4)));
+    RP_CUDA(cudaMalloc(&ctx->unit_aux, cap * sizeof(uint2)));
+    k_iota<<<(unsigned)((cap + 255) / 256), 256>>>(ctx->unit_iota, cap);
+    RP_CUDA(cudaGetLastError());
+  }
   RP_CUDA(cudaMemset(ctx->cost_prev, 0, nd * sizeof(uint16_t)));
   RP_CUDA(cudaMalloc(&ctx->item_val, nd * sizeof(double4)));
   RP_CUDA(cudaMalloc(&ctx->item_cnt, nd * sizeof(int4)));
@@ -1066,19 +1154,58 @@ int rp_alloc_potential_scratch(rp_ctx* ctx) {
   return RP_OK;
 }
 
-template <int KIND, int VAR>
-static int launch_integrate(rp_ctx* ctx, const Params& P) {
+template <int KIND, int VAR, bool UNIT = false>
+static int launch_integrate_one(rp_ctx* ctx, const Params& P) {
   int occ = 0;
   const size_t smem = sizeof(WarpSmem) * kWarps;
-  RP_CUDA(cudaFuncSetAttribute(k_integrate<KIND, VAR>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                               (int)smem));
-  RP_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_integrate<KIND, VAR>, 32 * kWarps,
-                                                        smem));
+  RP_CUDA(cudaFuncSetAttribute(k_integrate<KIND, VAR, UNIT>,
+                               cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+  RP_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_integrate<KIND, VAR, UNIT>,
+                                                        32 * kWarps, smem));
   if (occ < 1) occ = 1;
-  ProfScope ps(ctx, PK_INTEGRATE);
-  k_integrate<KIND, VAR><<<ctx->sm_count * occ, 32 * kWarps, smem, ctx->stream>>>(
+  k_integrate<KIND, VAR, UNIT><<<ctx->sm_count * occ, 32 * kWarps, smem, ctx->stream>>>(
       P, ctx->sched_order, ctx->clipAB, ctx->trig_full, ctx->item_val, ctx->item_cnt,
       ctx->item_aux, ctx->counters);
+  RP_CHECK_LAUNCH();
+  return RP_OK;
+}
+
+// The integrator: the items, then (split_level > 0) the deferred subtree units and their
+// merge into the items.  One profiling record covers the whole integration.
+template <int KIND, int VAR>
+static int launch_integrate(rp_ctx* ctx, const Params& P) {
+  ProfScope ps(ctx, PK_INTEGRATE);
+  int rc = launch_integrate_one<KIND, VAR, false>(ctx, P);
+  if (rc) return rc;
+  ctx->last_units = 0;
+  if (KIND != RP_SRC_GRID || VAR < 4 || P.split_level <= 0) return RP_OK;
+  cudaStream_t st = ctx->stream;
+  unsigned long long nu = 0;
+  RP_CUDA(cudaMemcpyAsync(&nu, ctx->counters + C_UNITS, sizeof(nu), cudaMemcpyDeviceToHost, st));
+  RP_CUDA(cudaStreamSynchronize(st));
+  if (nu == 0) return RP_OK;
+  if ((long long)nu > P.unit_cap) {  // overflowed pushes descended instead (see k_integrate)
+    nu = (unsigned long long)P.unit_cap;
+    RP_CUDA(cudaMemcpyAsync(ctx->counters + C_UNITS, &nu, sizeof(nu), cudaMemcpyHostToDevice, st));
+    RP_CUDA(cudaStreamSynchronize(st));
+  }
+  ctx->last_units = (int64_t)nu;
+  ProfScope pu(ctx, PK_UNITS);
+  rc = launch_integrate_one<KIND, VAR, true>(ctx, P);
+  if (rc) return rc;
+  size_t tmp = 0;
+  RP_CUDA(cub::DeviceRadixSort::SortPairs(nullptr, tmp, ctx->unit_key, ctx->unit_key_sorted,
+                                          ctx->unit_iota, ctx->unit_perm, (int)nu, 0,
+                                          32 + kUnitShift, st));
+  rc = rp_ensure_cub_tmp(ctx, tmp);
+  if (rc) return rc;
+  tmp = ctx->cub_tmp_bytes;
+  RP_CUDA(cub::DeviceRadixSort::SortPairs(ctx->cub_tmp, tmp, ctx->unit_key, ctx->unit_key_sorted,
+                                          ctx->unit_iota, ctx->unit_perm, (int)nu, 0,
+                                          32 + kUnitShift, st));
+  k_merge_units<<<(unsigned)((nu + 255) / 256), 256, 0, st>>>(
+      (long long)nu, ctx->unit_key_sorted, ctx->unit_perm, ctx->unit_val, ctx->unit_cnt,
+      ctx->unit_aux, ctx->item_val, ctx->item_cnt, ctx->item_aux);
   RP_CHECK_LAUNCH();
   return RP_OK;
 }
@@ -1146,6 +1273,13 @@ static int run_potentials(rp_ctx* ctx, Params P, int32_t rank, int32_t world,
       P.bp_off = ctx->bp_off_dev;
       P.cluster = ctx->cluster_dev;
     }
+    P.split_level = (KIND == RP_SRC_GRID && var >= 4 && P.bp_off == nullptr && ctx->unit_key)
+                        ? ctx->split_level : 0;
+    P.unit_cap = ctx->unit_cap;
+    P.unit_key = ctx->unit_key;
+    P.unit_val = ctx->unit_val;
+    P.unit_cnt = ctx->unit_cnt;
+    P.unit_aux = ctx->unit_aux;
     int rc2 = var == 4 ? launch_integrate<KIND, 4>(ctx, P)
               : var == 6 ? launch_integrate<KIND, 6>(ctx, P)
               : var == 7 ? launch_integrate<KIND, 7>(ctx, P)
@@ -1180,6 +1314,8 @@ int rp_potentials_impl(rp_ctx* ctx, int kind, const double src[6], int32_t rank,
   P.slot_doubles = ctx->slot_doubles; P.ring = ctx->ring; P.frames = ctx->frames_dev;
   P.amp = ctx->amp_dev;
   P.bp = nullptr; P.bp_off = nullptr; P.cluster = nullptr;
+  P.split_level = 0; P.unit_cap = 0; P.unit_key = nullptr; P.unit_val = nullptr;
+  P.unit_cnt = nullptr; P.unit_aux = nullptr;
   P.sx0 = src ? src[0] : 0; P.sy0 = src ? src[1] : 0; P.swidth = src ? src[2] : 0;
   P.sq = src ? src[3] : 0; P.sbx = src ? src[4] : 0; P.sby = src ? src[5] : 0;
   int rc;

@@ -54,7 +54,9 @@ void free_all(rp_ctx* c) {
                   c->item_val, c->item_cnt, c->item_aux, c->counters, c->amp_dev, c->trig_full,
                   c->point_key, c->point_key_sorted, c->point_idx, c->point_order,
                   c->point_owner, c->nseg_prev_pt, c->hx_d, c->hy_d, c->hux_d, c->huy_d,
-                  c->mesh_d, c->leaves_prev, c->cluster_dev, c->bp_off_dev, c->bp_dev};
+                  c->mesh_d, c->leaves_prev, c->cluster_dev, c->bp_off_dev, c->bp_dev,
+                  c->unit_key, c->unit_key_sorted, c->unit_iota, c->unit_perm, c->unit_val,
+                  c->unit_cnt, c->unit_aux};
   for (void* p : ptrs)
     if (p) cudaFree(p);
   for (auto& r : c->prof) {
@@ -154,6 +156,7 @@ int rp_profile_read(rp_ctx* ctx, rp_profile* out) {
   out->fields_ms = ctx->prof_acc[PK_FIELDS];
   out->push_ms = ctx->prof_acc[PK_PUSH];
   out->integrate_launches = ctx->prof_integrate_launches;
+  out->units_ms = ctx->prof_acc[PK_UNITS];
   return RP_OK;
 }
 
@@ -177,6 +180,7 @@ int rp_create(const rp_config* cfg, rp_ctx** out) {
   if (cudaSetDevice(cfg->device) != cudaSuccess) return fail(RP_ENODEV);
   cudaDeviceGetAttribute(&ctx->sm_count, cudaDevAttrMultiProcessorCount, cfg->device);
   if (const char* ev = getenv("RP_EVAL")) ctx->eval_variant = atoi(ev);
+  if (const char* sp = getenv("RP_SPLIT")) ctx->split_level = atoi(sp);
   ctx->H = cfg->history_depth + 2;
   ctx->PX = cfg->nx + 2 * RP_PAD;
   ctx->PY = cfg->ny + 2 * RP_PAD;

@@ -74,6 +74,18 @@ struct rp_ctx {
   std::vector<int32_t> cluster_host;
   rp_predictive_info pred_info{};
 
+  // subtree work units of the deep trees (k_integrate split_level)
+  int split_level = 12;             // RP_SPLIT overrides; 0 = off
+  long long unit_cap = 0;           // even
+  unsigned long long* unit_key = nullptr;
+  unsigned long long* unit_key_sorted = nullptr;
+  int32_t* unit_iota = nullptr;
+  int32_t* unit_perm = nullptr;
+  double4* unit_val = nullptr;
+  int4* unit_cnt = nullptr;
+  uint2* unit_aux = nullptr;
+  int64_t last_units = 0;           // units of the last call (diagnostics)
+
   // sharding scratch
   int32_t* point_key = nullptr;     // per point predicted work key
   int32_t* point_key_sorted = nullptr;
@@ -96,11 +108,12 @@ struct rp_ctx {
   int prof_on = 0;
   std::vector<ProfRec> prof;
   std::vector<cudaEvent_t> ev_pool;
-  double prof_acc[8] = {0, 0, 0, 0, 0, 0, 0, 0};
+  double prof_acc[9] = {0, 0, 0, 0, 0, 0, 0, 0, 0};
   int64_t prof_integrate_launches = 0;
 };
 
-enum { PK_DEPOSIT = 0, PK_APPEND, PK_CLIP, PK_SORT, PK_INTEGRATE, PK_REDUCE, PK_FIELDS, PK_PUSH };
+enum { PK_DEPOSIT = 0, PK_APPEND, PK_CLIP, PK_SORT, PK_INTEGRATE, PK_REDUCE, PK_FIELDS, PK_PUSH,
+       PK_UNITS };
 
 static inline cudaEvent_t prof_event(rp_ctx* ctx) {
   if (!ctx->ev_pool.empty()) {

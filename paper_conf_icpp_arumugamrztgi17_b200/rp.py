@@ -48,7 +48,7 @@ class rp_profile(C.Structure):
     _fields_ = [("deposit_ms", C.c_double), ("append_ms", C.c_double), ("clip_ms", C.c_double),
                 ("sort_ms", C.c_double), ("integrate_ms", C.c_double), ("reduce_ms", C.c_double),
                 ("fields_ms", C.c_double), ("push_ms", C.c_double),
-                ("integrate_launches", C.c_int64)]
+                ("integrate_launches", C.c_int64), ("units_ms", C.c_double)]
 
     def as_dict(self) -> dict:
         return {k: getattr(self, k) for k, _ in self._fields_}

@@ -38,17 +38,20 @@ per_n, scattered = {}, {}
 for world in (1, 2, 4, 8):
     cap = rp.rp_shard_capacity(sim.ctx, world)
     shards = torch.zeros((world, cap, 6), **f64)
-    times, evals = [], []
+    times, evals, units = [], [], []
     for r in range(world):
         rp.rp_profile_enable(sim.ctx, True)
         n, inf = rp.rp_compute_potentials_shard(sim.ctx, r, world, shards[r], info=True)
-        times.append(rp.rp_profile_read(sim.ctx).integrate_ms)
+        pr = rp.rp_profile_read(sim.ctx)
+        times.append(pr.integrate_ms)
+        units.append(round(pr.units_ms, 3))
         evals.append(inf.evals)
     res = {k: torch.zeros(npts, **f64) for k in ("phi", "ax", "ay", "err")}
     ns = torch.zeros(npts, dtype=torch.int32, device="cuda")
     rp.rp_shard_scatter(sim.ctx, shards, world, res["phi"], res["ax"], res["ay"], res["err"], ns)
     scattered[world] = (res, ns)
-    per_n[world] = {"shard_ms": [round(t, 3) for t in times], "max_ms": max(times),
+    per_n[world] = {"shard_ms": [round(t, 3) for t in times], "units_ms": units,
+                    "max_ms": max(times),
                     "evals_imbalance": max(evals) / (sum(evals) / world)}
 full = {k: torch.zeros(npts, **f64) for k in ("phi", "ax", "ay", "err")}
 nseg = torch.zeros(npts, dtype=torch.int32, device="cuda")
