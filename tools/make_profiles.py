@@ -44,27 +44,20 @@ for k, (n, ms) in sorted(agg.items(), key=lambda x: -x[1][1]):
 open(os.path.join(PROF, f"{tag}_launches.md"), "w").write("\n".join(lines) + "\n")
 
 # ---------------------------------------------------------------- full capture of k_integrate
+# one integrator call = the item launch + the subtree-unit launch (UNIT = true); the capture
+# holds both launches of one step
 rep = os.path.join(OUT, "prof_integrate.ncu-rep")
 raw = subprocess.run(["ncu", "-i", rep, "--page", "raw", "--csv"], capture_output=True, text=True).stdout
 rows = list(csv.reader(io.StringIO(raw)))
-d = {k: (u, v) for k, u, v in zip(rows[0], rows[1], rows[2])}
+launches = [{k: (u, v) for k, u, v in zip(rows[0], rows[1], r)} for r in rows[2:] if len(r) == len(rows[0])]
 
 
-def num(k):
+def num(d, k):
     u, v = d[k]
     return float(v.replace(",", "")) * BYTES.get(u, 1)
 
 
-stalls = []
-for k, (u, v) in d.items():
-    if "smsp__average_warps_issue_stalled" in k and k.endswith("_per_issue_active.ratio"):
-        try:
-            stalls.append((float(v), k.replace("smsp__average_warps_issue_stalled_", "").replace(
-                "_per_issue_active.ratio", "")))
-        except ValueError:
-            pass
-stalls.sort(reverse=True)
-dram = num("dram__bytes_read.sum") + num("dram__bytes_write.sum")
+
 keys = [("duration (ms, under ncu)", "gpu__time_duration.sum"),
         ("registers / thread", "launch__registers_per_thread"),
         ("achieved warps / SM (% of 64)", "sm__warps_active.avg.pct_of_peak_sustained_active"),
@@ -78,17 +71,35 @@ keys = [("duration (ms, under ncu)", "gpu__time_duration.sum"),
         ("L1 hit rate %", "l1tex__t_sector_hit_rate.pct"),
         ("L2 hit rate %", "lts__t_sector_hit_rate.pct"),
         ("DRAM read", "dram__bytes_read.sum"), ("DRAM write", "dram__bytes_write.sum")]
-lines = [f"# {tag}: ncu --set full of `k_integrate` (one launch, cfg2 64x64 bend, after warm-up)", "",
-         "| metric | value |", "|---|---|"]
+names = [d["Kernel Name"][1].split("(")[0].replace("void ", "").replace("<unnamed>::", "")[:60]
+         for d in launches]
+lines = [f"# {tag}: ncu --set full of the integrator (cfg2 64x64 bend, one step after warm-up)", "",
+         "One integrator call = the item launch (`k_integrate<..., false>`) + the subtree-unit launch",
+         "(`k_integrate<..., true>`, deep trees split at level 12).", "",
+         "| metric | " + " | ".join(f"`{n}`" for n in names) + " |",
+         "|---|" + "---|" * len(launches)]
 for label, k in keys:
-    if k in d:
-        lines.append(f"| {label} (`{k}`) | {d[k][1]} {d[k][0]} |")
-lines += ["", "Warp stall reasons (cycles per issued instruction):", ""]
-lines += [f"- {name}: {v:.3f}" for v, name in stalls[:10]]
-lines += ["", f"DRAM traffic per launch (read + write): {dram:.0f} bytes"]
+    if all(k in d for d in launches):
+        lines.append(f"| {label} (`{k}`) | " + " | ".join(f"{d[k][1]} {d[k][0]}" for d in launches) + " |")
+for i, d in enumerate(launches):
+    stalls = []
+    for k, (u, v) in d.items():
+        if "smsp__average_warps_issue_stalled" in k and k.endswith("_per_issue_active.ratio"):
+            try:
+                stalls.append((float(v), k.replace("smsp__average_warps_issue_stalled_", "").replace(
+                    "_per_issue_active.ratio", "")))
+            except ValueError:
+                pass
+    stalls.sort(reverse=True)
+    lines += ["", f"Warp stall reasons of `{names[i]}` (cycles per issued instruction):", ""]
+    lines += [f"- {name}: {v:.3f}" for v, name in stalls[:8]]
+dram = sum(num(d, "dram__bytes_read.sum") + num(d, "dram__bytes_write.sum") for d in launches)
+dur = sum(num(d, "gpu__time_duration.sum") for d in launches)
+lines += ["", f"DRAM traffic per integrator call (all {len(launches)} launches, read + write): {dram:.0f} bytes"]
 open(os.path.join(PROF, f"{tag}_ncu_integrate.md"), "w").write("\n".join(lines) + "\n")
-json.dump({"round": tag, "kernel": "k_integrate", "dram_bytes_per_launch": dram,
-           "duration_ms_under_ncu": num("gpu__time_duration.sum")},
+json.dump({"round": tag, "kernel": "k_integrate (items + units)", "launches": len(launches),
+           "dram_bytes_per_launch": dram, "dram_bytes_per_call": dram,
+           "duration_ms_under_ncu": dur},
           open(os.path.join(PROF, "ncu_integrate.json"), "w"), indent=1)
 print(open(os.path.join(PROF, f"{tag}_launches.md")).read())
 print("\n".join(lines))
