@@ -186,7 +186,8 @@ def run_ours(args):
     clocks.start()
     barrier()
     step_ms = []
-    totals = {"evals": 0, "skipped": 0, "nodes": 0, "segments": 0, "capped": 0, "items": 0}
+    totals = {"evals": 0, "skipped": 0, "nodes": 0, "segments": 0, "capped": 0, "items": 0,
+              "units": 0, "unit_overflow": 0}
     for _ in range(args.steps):
         flush.fill_(1.0)  # evict L2 between timed steps (outside the events)
         e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)

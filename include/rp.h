@@ -95,6 +95,11 @@ typedef struct {
                               padded TSC integrand vanishes (DESIGN R-24) or the Lagrange-3 one
                               takes its outside limit 0 (R-25b), not evaluated; the evaluations
                               performed are evals - skipped                                     */
+  int64_t units;           /* subtree work units walked separately (deep trees split at level 12,
+                              DESIGN sec. 6); 0 when the split is off                           */
+  int32_t unit_overflow;   /* 1 if the unit list was full and some subtrees were walked in place
+                              (same tree and values; only the summation grouping differs)       */
+  int32_t pad;
 } rp_potential_info;
 
 /* Create a context on cfg->device: allocates the HBM history ring of history_depth+2

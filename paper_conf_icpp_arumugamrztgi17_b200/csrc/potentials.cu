@@ -65,6 +65,8 @@ struct Params {
   const int32_t* cluster;
   // subtree work units (deep trees split at a fixed level, see k_integrate)
   int split_level;                  // 0: off
+  int split_j;                      // only subregions j < split_j are split (the near field)
+  int unit_budget;                  // at most this many units per item (the first in DFS order)
   long long unit_cap;
   unsigned long long* unit_key;     // [unit_cap] item << kUnitShift | ix
   double4* unit_val;
@@ -806,7 +808,7 @@ __global__ void __launch_bounds__(32 * kWarps) k_integrate(
 #pragma unroll
         for (int i = 0; i < 9; ++i) st[l][i][0] = st[l][i][1] = st[l][i][2] = 0.0;
     }
-    int nseg = 0, nleaf = 0, capped = 0, ties = 0, maxlev = 0;
+    int nseg = 0, nleaf = 0, capped = 0, ties = 0, maxlev = 0, ndef = 0;
     unsigned evals = 0, nskip = 0;
     int lev = UNIT ? P.split_level : ((P.n_root == 2 && !pred) ? 1 : 0);
     const int rlev = UNIT ? P.split_level : 0;  // the walk ends when it climbs back here
@@ -920,7 +922,9 @@ __global__ void __launch_bounds__(32 * kWarps) k_integrate(
         ++nleaf;
         s_phi += k0; s_ax += k1; s_ay += k2; s_err += err;
         finished = true;
-      } else if (!UNIT && P.split_level > 0 && lev + 1 == P.split_level) {
+      } else if (!UNIT && P.split_level > 0 && lev + 1 == P.split_level && j < P.split_j &&
+                 ndef < P.unit_budget) {
+        ndef += 2;  // per-item budget, counted in DFS order: deterministic
         // defer both children as subtree units (falls back to descending if the unit list is
         // full, flagged in counters[C_UOVF])
         unsigned long long u = 0;
@@ -1116,7 +1120,14 @@ int rp_alloc_potential_scratch(rp_ctx* ctx) {
   RP_CUDA(cudaMemset(ctx->leaves_prev, 0, nd * sizeof(uint16_t)));
   RP_CUDA(cudaMalloc(&ctx->cluster_dev, npts * sizeof(int32_t)));
   if (ctx->split_level > 0) {
-    const long long cap = std::max<long long>(1LL << 22, 64LL * (long long)npts) & ~1LL;
+    // a unit list of up to 512 units per mesh point (config 4 needs ~130-300; 80 bytes each),
+    // at most 5 % of the device memory; a full list is exact (subtrees walked in place) and
+    // reported in rp_potential_info.unit_overflow
+    size_t fr = 0, tot = 0;
+    cudaMemGetInfo(&fr, &tot);
+    const long long budget = (long long)(0.05 * (double)tot / 80.0);
+    const long long cap =
+        std::max<long long>(1LL << 22, std::min<long long>(512LL * (long long)npts, budget)) & ~1LL;
     ctx->unit_cap = cap;
     RP_CUDA(cudaMalloc(&ctx->unit_key, cap * sizeof(unsigned long long)));
     RP_CUDA(cudaMalloc(&ctx->unit_key_sorted, cap * sizeof(unsigned long long)));
@@ -1275,6 +1286,8 @@ static int run_potentials(rp_ctx* ctx, Params P, int32_t rank, int32_t world,
     }
     P.split_level = (KIND == RP_SRC_GRID && var >= 4 && P.bp_off == nullptr && ctx->unit_key)
                         ? ctx->split_level : 0;
+    P.split_j = ctx->split_j;
+    P.unit_budget = 64;
     P.unit_cap = ctx->unit_cap;
     P.unit_key = ctx->unit_key;
     P.unit_val = ctx->unit_val;
@@ -1314,7 +1327,7 @@ int rp_potentials_impl(rp_ctx* ctx, int kind, const double src[6], int32_t rank,
   P.slot_doubles = ctx->slot_doubles; P.ring = ctx->ring; P.frames = ctx->frames_dev;
   P.amp = ctx->amp_dev;
   P.bp = nullptr; P.bp_off = nullptr; P.cluster = nullptr;
-  P.split_level = 0; P.unit_cap = 0; P.unit_key = nullptr; P.unit_val = nullptr;
+  P.split_level = 0; P.split_j = 0; P.unit_budget = 0; P.unit_cap = 0; P.unit_key = nullptr; P.unit_val = nullptr;
   P.unit_cnt = nullptr; P.unit_aux = nullptr;
   P.sx0 = src ? src[0] : 0; P.sy0 = src ? src[1] : 0; P.swidth = src ? src[2] : 0;
   P.sq = src ? src[3] : 0; P.sbx = src ? src[4] : 0; P.sby = src ? src[5] : 0;
@@ -1341,6 +1354,9 @@ int rp_potentials_impl(rp_ctx* ctx, int kind, const double src[6], int32_t rank,
       info->max_level = (int32_t)h[C_MAXLEV];
       info->kappa = P.kap;
       info->skipped = (int64_t)h[C_SKIP];
+      info->units = ctx->last_units;
+      info->unit_overflow = h[C_UOVF] ? 1 : 0;
+      info->pad = 0;
     }
     if (n_out) *n_out = (int64_t)h[C_NOUT];
   }

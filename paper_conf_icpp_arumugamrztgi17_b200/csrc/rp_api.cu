@@ -181,6 +181,7 @@ int rp_create(const rp_config* cfg, rp_ctx** out) {
   cudaDeviceGetAttribute(&ctx->sm_count, cudaDevAttrMultiProcessorCount, cfg->device);
   if (const char* ev = getenv("RP_EVAL")) ctx->eval_variant = atoi(ev);
   if (const char* sp = getenv("RP_SPLIT")) ctx->split_level = atoi(sp);
+  if (const char* sj = getenv("RP_SPLITJ")) ctx->split_j = atoi(sj);
   ctx->H = cfg->history_depth + 2;
   ctx->PX = cfg->nx + 2 * RP_PAD;
   ctx->PY = cfg->ny + 2 * RP_PAD;

@@ -76,6 +76,7 @@ struct rp_ctx {
 
   // subtree work units of the deep trees (k_integrate split_level)
   int split_level = 12;             // RP_SPLIT overrides; 0 = off
+  int split_j = 1;                  // RP_SPLITJ: split the trees of subregions j < split_j
   long long unit_cap = 0;           // even
   unsigned long long* unit_key = nullptr;
   unsigned long long* unit_key_sorted = nullptr;

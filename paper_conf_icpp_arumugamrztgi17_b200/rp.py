@@ -58,7 +58,8 @@ class rp_potential_info(C.Structure):
     _fields_ = [("evals", C.c_int64), ("nodes", C.c_int64), ("segments", C.c_int64),
                 ("leaves", C.c_int64), ("capped", C.c_int64), ("ties", C.c_int64),
                 ("items", C.c_int64), ("max_level", C.c_int32), ("kappa", C.c_int32),
-                ("skipped", C.c_int64)]
+                ("skipped", C.c_int64), ("units", C.c_int64), ("unit_overflow", C.c_int32),
+                ("pad", C.c_int32)]
 
     def as_dict(self) -> dict:
         return {k: getattr(self, k) for k, _ in self._fields_}

@@ -235,6 +235,32 @@ def test_potentials_bend_small_full_mesh_two_steps(torch, rule, interp):
         rp.rp_destroy(ctx)
 
 
+def test_subtree_units_match_the_unsplit_walk(torch, monkeypatch):
+    """Deep trees split into subtree work units walk the same canonical tree:
+    equal segment counts per point and values equal to the single-warp walk up to the
+    summation grouping (config 2 at full size, the bench workload)."""
+    from paper_conf_icpp_arumugamrztgi17_b200 import rp
+    cfg = W.config(2)
+    ring, _ = _deposit_rigid_ring(cfg)
+    frames = W.ring_frames(cfg, 0)
+    out = {}
+    for split in ("12", "0"):
+        monkeypatch.setenv("RP_SPLIT", split)
+        ctx = G.make_ctx(cfg)
+        try:
+            G.load_state(ctx, cfg, 0, cfg.n_pre, ring, frames)
+            out[split] = G.gpu_potentials(ctx, cfg.nx * cfg.ny)
+        finally:
+            rp.rp_destroy(ctx)
+    (a, ia), (b, ib) = out["12"], out["0"]
+    assert ia.units > 1000 and ia.unit_overflow == 0 and ib.units == 0
+    np.testing.assert_array_equal(a["nseg"], b["nseg"])
+    assert ia.evals == ib.evals and ia.leaves == ib.leaves and ia.capped == ib.capped
+    scale = max(np.abs(b["phi"]).max(), np.abs(b["ax"]).max(), np.abs(b["ay"]).max())
+    for k in ("phi", "ax", "ay"):
+        assert np.abs(a[k] - b[k]).max() <= 1e-13 * scale
+
+
 @pytest.mark.parametrize("which", ["bend_small", "cfg2_sampled"])
 def test_support_clip_bit_exact(torch, which):
     """Step a5 (R-5): the GPU's per-(point, subregion) support [A, B] equals the oracle's clip
@@ -568,6 +594,7 @@ def test_potentials_bend_cfg3_full_size_sampled(torch):
         fail, worst, _ = G.compare_potentials(gpu, orc, pts)
         assert not fail.any(), (pts[fail][:10], worst)
         assert info.kappa == cfg.kappa_max
+        assert info.units > 0 and info.unit_overflow == 0
     finally:
         rp.rp_destroy(ctx)
 
@@ -594,6 +621,7 @@ def test_potentials_bend_cfg4_full_size_sampled(torch):
         fail, worst, _ = G.compare_potentials(gpu, orc, pts)
         assert not fail.any(), (pts[fail][:10], worst)
         assert info.kappa == cfg.kappa_max
+        assert info.units > 0 and info.unit_overflow == 0
     finally:
         rp.rp_destroy(ctx)
 
@@ -619,6 +647,7 @@ def test_potentials_bend_cfg5_full_size_sampled(torch):
         fail, worst, _ = G.compare_potentials(gpu, orc, pts)
         assert not fail.any(), (pts[fail][:10], worst)
         assert info.kappa == cfg.kappa_max
+        assert info.units > 0 and info.unit_overflow == 0
     finally:
         rp.rp_destroy(ctx)
 
