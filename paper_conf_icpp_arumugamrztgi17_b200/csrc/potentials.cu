@@ -69,6 +69,7 @@ struct Params {
   int unit_budget;                  // at most this many units per item (the first in DFS order)
   long long unit_cap;
   unsigned long long* unit_key;     // [unit_cap] item << kUnitShift | ix
+  const int32_t* unit_order;        // unit launch: the units, longest-predicted-first
   double4* unit_val;
   int4* unit_cnt;
   uint2* unit_aux;
@@ -762,7 +763,8 @@ __global__ void __launch_bounds__(32 * kWarps) k_integrate(
     if (lane == 0) idx = atomicAdd(&counters[UNIT ? C_NEXT_U : C_NEXT], 1ULL);
     idx = __shfl_sync(0xffffffffu, idx, 0);
     if (idx >= n_items) break;
-    const unsigned long long ukey = UNIT ? P.unit_key[idx] : 0ULL;
+    const int uidx = UNIT ? P.unit_order[idx] : 0;
+    const unsigned long long ukey = UNIT ? P.unit_key[uidx] : 0ULL;
     const int item = UNIT ? (int)(ukey >> kUnitShift) : order[idx];
     const int p = item / P.kmax, j = item % P.kmax;
     const double2 ab = AB[item];
@@ -963,7 +965,7 @@ __global__ void __launch_bounds__(32 * kWarps) k_integrate(
       if (TM) { long long t = clock64(); ph[5] += t - t0; t0 = t; }
     }
     if (lane == 0) {
-      const size_t o = UNIT ? (size_t)idx : (size_t)item;
+      const size_t o = UNIT ? (size_t)uidx : (size_t)item;
       (UNIT ? P.unit_val : item_val)[o] = make_double4(s_phi, s_ax, s_ay, s_err);
       (UNIT ? P.unit_cnt : item_cnt)[o] = make_int4(nseg, nleaf, capped, ties);
       (UNIT ? P.unit_aux : item_aux)[o] = make_uint2((unsigned)maxlev, evals);
@@ -978,6 +980,17 @@ __global__ void __launch_bounds__(32 * kWarps) k_integrate(
 __global__ void k_iota(int32_t* a, long long n) {
   const long long i = blockIdx.x * (long long)blockDim.x + threadIdx.x;
   if (i < n) a[i] = (int32_t)i;
+}
+
+// Launch order of the units: their item's segment count of the previous step (the forecast),
+// largest first (ties by unit index), so the longest units do not start last.
+__global__ void k_unit_order_keys(long long n, const unsigned long long* __restrict__ key,
+                                  const uint16_t* __restrict__ cost,
+                                  unsigned long long* __restrict__ okey) {
+  const long long u = blockIdx.x * (long long)blockDim.x + threadIdx.x;
+  if (u >= n) return;
+  const unsigned long long item = key[u] >> kUnitShift;
+  okey[u] = ((unsigned long long)(0xFFFFu - cost[item]) << 32) | (unsigned long long)u;
 }
 
 // Add every item's units to its own partial result, in (item, subtree index) order: one
@@ -1125,12 +1138,13 @@ int rp_alloc_potential_scratch(rp_ctx* ctx) {
     // reported in rp_potential_info.unit_overflow
     size_t fr = 0, tot = 0;
     cudaMemGetInfo(&fr, &tot);
-    const long long budget = (long long)(0.05 * (double)tot / 80.0);
+    const long long budget = (long long)(0.05 * (double)tot / 88.0);
     const long long cap =
         std::max<long long>(1LL << 22, std::min<long long>(512LL * (long long)npts, budget)) & ~1LL;
     ctx->unit_cap = cap;
     RP_CUDA(cudaMalloc(&ctx->unit_key, cap * sizeof(unsigned long long)));
     RP_CUDA(cudaMalloc(&ctx->unit_key_sorted, cap * sizeof(unsigned long long)));
+    RP_CUDA(cudaMalloc(&ctx->unit_okey, cap * sizeof(unsigned long long)));
     RP_CUDA(cudaMalloc(&ctx->unit_iota, cap * sizeof(int32_t)));
     RP_CUDA(cudaMalloc(&ctx->unit_perm, cap * sizeof(int32_t)));
     RP_CUDA(cudaMalloc(&ctx->unit_val, cap * sizeof(double4)));
@@ -1202,7 +1216,24 @@ static int launch_integrate(rp_ctx* ctx, const Params& P) {
   }
   ctx->last_units = (int64_t)nu;
   ProfScope pu(ctx, PK_UNITS);
-  rc = launch_integrate_one<KIND, VAR, true>(ctx, P);
+  {
+    // longest-predicted-first order of the units (ctx->unit_key_sorted / unit_perm are free
+    // until the merge sort below)
+    k_unit_order_keys<<<(unsigned)((nu + 255) / 256), 256, 0, st>>>(
+        (long long)nu, ctx->unit_key, ctx->cost_prev, ctx->unit_okey);
+    RP_CHECK_LAUNCH();
+    size_t tmp = 0;
+    RP_CUDA(cub::DeviceRadixSort::SortPairs(nullptr, tmp, ctx->unit_okey, ctx->unit_key_sorted,
+                                            ctx->unit_iota, ctx->unit_perm, (int)nu, 0, 48, st));
+    rc = rp_ensure_cub_tmp(ctx, tmp);
+    if (rc) return rc;
+    tmp = ctx->cub_tmp_bytes;
+    RP_CUDA(cub::DeviceRadixSort::SortPairs(ctx->cub_tmp, tmp, ctx->unit_okey, ctx->unit_key_sorted,
+                                            ctx->unit_iota, ctx->unit_perm, (int)nu, 0, 48, st));
+  }
+  Params PU = P;
+  PU.unit_order = ctx->unit_perm;
+  rc = launch_integrate_one<KIND, VAR, true>(ctx, PU);
   if (rc) return rc;
   size_t tmp = 0;
   RP_CUDA(cub::DeviceRadixSort::SortPairs(nullptr, tmp, ctx->unit_key, ctx->unit_key_sorted,
@@ -1327,7 +1358,7 @@ int rp_potentials_impl(rp_ctx* ctx, int kind, const double src[6], int32_t rank,
   P.slot_doubles = ctx->slot_doubles; P.ring = ctx->ring; P.frames = ctx->frames_dev;
   P.amp = ctx->amp_dev;
   P.bp = nullptr; P.bp_off = nullptr; P.cluster = nullptr;
-  P.split_level = 0; P.split_j = 0; P.unit_budget = 0; P.unit_cap = 0; P.unit_key = nullptr; P.unit_val = nullptr;
+  P.split_level = 0; P.split_j = 0; P.unit_budget = 0; P.unit_cap = 0; P.unit_order = nullptr; P.unit_key = nullptr; P.unit_val = nullptr;
   P.unit_cnt = nullptr; P.unit_aux = nullptr;
   P.sx0 = src ? src[0] : 0; P.sy0 = src ? src[1] : 0; P.swidth = src ? src[2] : 0;
   P.sq = src ? src[3] : 0; P.sbx = src ? src[4] : 0; P.sby = src ? src[5] : 0;

@@ -55,7 +55,7 @@ void free_all(rp_ctx* c) {
                   c->point_key, c->point_key_sorted, c->point_idx, c->point_order,
                   c->point_owner, c->nseg_prev_pt, c->hx_d, c->hy_d, c->hux_d, c->huy_d,
                   c->mesh_d, c->leaves_prev, c->cluster_dev, c->bp_off_dev, c->bp_dev,
-                  c->unit_key, c->unit_key_sorted, c->unit_iota, c->unit_perm, c->unit_val,
+                  c->unit_key, c->unit_key_sorted, c->unit_okey, c->unit_iota, c->unit_perm, c->unit_val,
                   c->unit_cnt, c->unit_aux};
   for (void* p : ptrs)
     if (p) cudaFree(p);

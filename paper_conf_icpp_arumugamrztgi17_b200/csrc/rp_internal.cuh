@@ -80,6 +80,7 @@ struct rp_ctx {
   long long unit_cap = 0;           // even
   unsigned long long* unit_key = nullptr;
   unsigned long long* unit_key_sorted = nullptr;
+  unsigned long long* unit_okey = nullptr;  // launch-order keys of the units
   int32_t* unit_iota = nullptr;
   int32_t* unit_perm = nullptr;
   double4* unit_val = nullptr;
