@@ -65,4 +65,4 @@ for v in variants:
     print(f"variant {v}: integrate ms/step {[round(x, 2) for x in ms]} "
           f"(steps 2+: {np.mean(ms[2:]) if len(ms) > 2 else np.mean(ms):.2f}); "
           f"ps/eval {[round(1e9 * m / e, 2) for m, e in zip(ms, ev)]}; "
-          f"evals {info.evals}; bit-identical to first: {same}", flush=True)
+          f"evals/step (1e9) {[round(e / 1e9, 3) for e in ev]}; bit-identical to first: {same}", flush=True)
