@@ -360,6 +360,7 @@ def run_e2e(cfg, args, dev):
 # ---------------------------------------------------------------------------- oracle arm
 def _oracle_state(cfg):
     import oracle
+    oracle.set_threads(_cores())  # all host cores, whatever OMP_NUM_THREADS torchrun set
     x, y, ux, uy = W.particles(cfg)
     q = 1.0 / len(x)
     t0 = time.perf_counter()

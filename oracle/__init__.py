@@ -67,6 +67,17 @@ class Result(C.Structure):
 _lib = None
 
 
+def set_threads(n: int) -> int:
+    """Set the OpenMP thread count of the oracle's parallel loops (the calling thread's
+    nthreads ICV).  torchrun exports OMP_NUM_THREADS=1 and torch loads libgomp.so.1 before
+    the oracle, so the environment cannot be changed after the fact; bench.py calls this with
+    the host cores it reports.  Returns the count in effect."""
+    lib()
+    gomp = C.CDLL("libgomp.so.1")  # the instance already loaded (shared by soname)
+    gomp.omp_set_num_threads(C.c_int(int(n)))
+    return int(gomp.omp_get_max_threads())
+
+
 def lib():
     global _lib
     if _lib is None:

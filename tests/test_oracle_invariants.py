@@ -125,3 +125,18 @@ def test_rigid_ring_carries_the_tangent_current_of_each_level():
         np.testing.assert_allclose(R[..., 2], g * b * s, rtol=0, atol=1e-15 * g.max())
     # the oldest level (l = -61, psi = -0.12 rad) is rotated, not copied
     assert np.abs(ring[1, ..., 2]).max() > 0.1 * b * g.max()
+
+
+def test_oracle_thread_count_overrides_the_environment():
+    """bench.py's oracle legs run on all host cores even under torchrun, which exports
+    OMP_NUM_THREADS=1 before torch loads libgomp; the result does not depend on the count."""
+    cfg = _bend_small()
+    import bench
+    pts = np.arange(0, cfg.nx * cfg.ny, 97, dtype=np.int32)
+    P, _ = bench._oracle_state(cfg)
+    assert oracle.set_threads(1) == 1
+    r1 = P.potentials(pts)
+    assert oracle.set_threads(2) == 2
+    r2 = P.potentials(pts)
+    assert oracle.set_threads(bench._cores()) == bench._cores()
+    assert len(r1) == len(pts) and r1.tobytes() == r2.tobytes()
