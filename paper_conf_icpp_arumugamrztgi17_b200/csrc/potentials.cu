@@ -835,8 +835,8 @@ __global__ void __launch_bounds__(32 * kWarps) k_integrate(
         else r = __dadd_rn(m, __dmul_rn(hw, c_xgk[i]));
         double cu, cv, w0, w1, w2;
         centre_at(it, P, r, cu, cv, w0, w1, w2);
-        double th1[kMaxArcs], dth[kMaxArcs];
-        int na = arcs<KIND>(it, P, cu, cv, r, th1, dth);
+        // arcs written straight into the warp's shared block (no local-memory staging)
+        int na = arcs<KIND>(it, P, cu, cv, r, S.th1[lane], S.dth[lane]);
         NodeRec nr;
         nr.r = r; nr.cu = cu; nr.cv = cv; nr.w0 = w0; nr.w1 = w1; nr.w2 = w2;
         if (P.rule == RP_RULE_SIMPSON) {  // Boole h/90 (7,32,12,32,7); Simpson h/12 (1,4,2,4,1)
@@ -849,10 +849,6 @@ __global__ void __launch_bounds__(32 * kWarps) k_integrate(
         }
         S.node[lane] = nr;
         S.na[lane] = na;
-        for (int q = 0; q < (na > 0 ? na : 0); ++q) {
-          S.th1[lane][q] = th1[q];
-          S.dth[lane][q] = dth[q];
-        }
         cnt = na < 0 ? N : na * (N + 1);
         full = na < 0;
         if (KIND == RP_SRC_GRID && VAR >= 4 && na > 0) {  // interior nodes (R-24, R-25b)
