@@ -1,0 +1,26 @@
+"""bench.py --impl reference (the oracle arm) as the driver launches it for
+N > 1: under torchrun, rank 0 alone times the oracle on all host cores and prints one JSON
+line; the other ranks exit 0 without work.  CPU only."""
+import json
+import os
+import subprocess
+import sys
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+
+
+def test_reference_arm_under_torchrun_two_ranks():
+    env = dict(os.environ)
+    env.pop("OMP_NUM_THREADS", None)  # torchrun sets it to 1 for its children
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", "--nproc-per-node", "2",
+           "--master-addr", "127.0.0.1", "--master-port", "29561", "bench.py", "--impl",
+           "reference", "--gpus", "2", "--config", "1", "--steps", "1", "--warmup", "1"]
+    p = subprocess.run(cmd, cwd=ROOT, env=env, capture_output=True, text=True, timeout=600)
+    assert p.returncode == 0, p.stderr[-2000:]
+    lines = [ln for ln in p.stdout.splitlines() if ln.startswith("{")]
+    assert len(lines) == 1, p.stdout
+    d = json.loads(lines[0])
+    assert d["impl"] == "reference" and d["n_gpus"] == 2 and d["value"] > 0
+    assert d["cpu_baseline"]["kind"] == "oracle"
+    assert d["cpu_baseline"]["cores"] == len(os.sched_getaffinity(0))
+    assert d["e2e"]["h2d_bytes_per_step"] == 0 and d["e2e"]["value"] == d["value"]
