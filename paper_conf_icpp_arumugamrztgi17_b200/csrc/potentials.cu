@@ -17,6 +17,7 @@
 //   k_reduce     per point, sum the items in j order -> phi, A, err, nseg; counts.
 // FP64 throughout.  No tensor cores: the work is an irregular gather stencil,
 // not a dense contraction.
+#include <math_constants.h>
 #include <cub/device/device_radix_sort.cuh>
 #include <math.h>
 
@@ -388,13 +389,15 @@ __device__ int arcs(const Item& it, const Params& P, double cu, double cv, doubl
     dth[0] = ((ph + al) - (ph - al)) / N;
     return 1;
   }
-  // Crossings of the circle with the 4 edge lines that lie on the edge (kept compact: the
-  // node phase runs on 15 lanes once per segment, so code size matters more than ILP).
+  // Crossings of the circle with the 4 edge lines that lie on the edge.  Edge e's two
+  // crossings sit in fixed slots 2e, 2e + 1 (+inf when absent), sorted by a 19-comparator
+  // network and consumed through a register shift, so nothing goes to local memory.
   double t[8];
   int n = 0;
   const double rinv = 1.0 / r;
 #pragma unroll
   for (int e = 0; e < 4; ++e) {  // the 4 edges are independent: unrolled for ILP
+    t[2 * e] = t[2 * e + 1] = CUDART_INF;
     const bool vert = e < 2;
     const double edge = e == 0 ? it.U0 : e == 1 ? it.U1 : e == 2 ? it.V0 : it.V1;
     const double d = (edge - (vert ? cu : cv)) * rinv;
@@ -411,27 +414,30 @@ __device__ int arcs(const Item& it, const Params& P, double cu, double cv, doubl
       c1 = be < 0.0 ? be + kTwoPi : be;
       c2 = M_PI - be;
     }
-    if (o1 >= lo && o1 <= hi) t[n++] = c1;
-    if (o2 >= lo && o2 <= hi) t[n++] = c2;
+    if (o1 >= lo && o1 <= hi) { t[2 * e] = c1; ++n; }
+    if (o2 >= lo && o2 <= hi) { t[2 * e + 1] = c2; ++n; }
   }
   if (n == 0) return in_rect(cu + r, cv, it) ? -1 : 0;
-#pragma unroll 1
-  for (int i = 1; i < n; ++i) {  // insertion sort (n <= 8)
-    double x = t[i];
-    int k = i - 1;
-    while (k >= 0 && t[k] > x) {
-      t[k + 1] = t[k];
-      --k;
-    }
-    t[k + 1] = x;
+  constexpr int kNet[19][2] = {{0, 1}, {2, 3}, {4, 5}, {6, 7}, {0, 2}, {1, 3}, {4, 6},
+                               {5, 7}, {1, 2}, {5, 6}, {0, 4}, {1, 5}, {2, 6}, {3, 7},
+                               {2, 4}, {3, 5}, {1, 2}, {3, 4}, {5, 6}};
+#pragma unroll
+  for (int c = 0; c < 19; ++c) {
+    const double x = t[kNet[c][0]], y = t[kNet[c][1]];
+    const bool sw = y < x;
+    t[kNet[c][0]] = sw ? y : x;
+    t[kNet[c][1]] = sw ? x : y;
   }
   // unique crossings u_0 < u_1 < ...; keep the intervals (u_i, u_{i+1}) and
   // (u_last, u_0 + 2 pi) whose midpoint lies inside the rectangle
   int na = 0;
-  double prev = t[0];
+  const double first = t[0];
+  double prev = first;
 #pragma unroll 1
   for (int i = 1; i <= n; ++i) {
-    const double cur = i < n ? t[i] : t[0] + kTwoPi;
+    const double cur = i < n ? t[1] : first + kTwoPi;
+#pragma unroll
+    for (int q = 1; q < 7; ++q) t[q] = t[q + 1];
     if (i < n && cur == prev) continue;
     double sm, cm;
     sincos_b(0.5 * (prev + cur), &sm, &cm);
