@@ -3,17 +3,24 @@ N > 1: under torchrun, rank 0 alone times the oracle on all host cores and print
 line; the other ranks exit 0 without work.  CPU only."""
 import json
 import os
+import socket
 import subprocess
 import sys
 
 ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 
 
+def _free_port() -> int:
+    with socket.socket() as sk:
+        sk.bind(("127.0.0.1", 0))
+        return sk.getsockname()[1]
+
+
 def test_reference_arm_under_torchrun_two_ranks():
     env = dict(os.environ)
     env.pop("OMP_NUM_THREADS", None)  # torchrun sets it to 1 for its children
     cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", "--nproc-per-node", "2",
-           "--master-addr", "127.0.0.1", "--master-port", "29561", "bench.py", "--impl",
+           "--master-addr", "127.0.0.1", "--master-port", str(_free_port()), "bench.py", "--impl",
            "reference", "--gpus", "2", "--config", "1", "--steps", "1", "--warmup", "1"]
     p = subprocess.run(cmd, cwd=ROOT, env=env, capture_output=True, text=True, timeout=600)
     assert p.returncode == 0, p.stderr[-2000:]
