@@ -166,6 +166,8 @@ def run_ours(args):
     sched = args.schedule
     if sched == "index":
         rp.rp_set_schedule(sim.ctx, rp.RP_SCHED_INDEX, 1)
+    elif sched == "subregion":
+        rp.rp_set_schedule(sim.ctx, rp.RP_SCHED_SUBREGION, 1)
     elif sched.startswith("knn"):
         rp.rp_set_schedule(sim.ctx, rp.RP_SCHED_KNN, int(sched[3:]))
     dev = torch.device("cuda", local)

@@ -246,10 +246,15 @@ int rp_debug_potentials_analytic(rp_ctx* ctx, int32_t kind, double x0, double y0
  *   RP_SCHED_KNN          kNN regression over mesh points: predicted cost of (p, j) =
  *                         mean of last step's cost of (q, j) over the k nearest mesh points q
  *                         of the comoving mesh (k in {1, 5, 9, 25}; 1 = persistence).
+ *   RP_SCHED_SUBREGION    persistence forecast, items ordered subregion-major (j ascending) and
+ *                         longest-predicted-first within each subregion, so the warps running
+ *                         at any moment share one subregion's three history levels (L2 reuse
+ *                         when the ring is larger than L2, configs 4-5).
  * Items are then run longest-predicted-first (LPT). */
 #define RP_SCHED_INDEX 0
 #define RP_SCHED_PERSISTENCE 1
 #define RP_SCHED_KNN 2
+#define RP_SCHED_SUBREGION 3
 int rp_set_schedule(rp_ctx* ctx, int32_t policy, int32_t k);
 
 /* Predictive-RP variant: the paper's own COMPUTE-POTENTIALS (Algorithm 1; DESIGN

@@ -107,6 +107,7 @@ def lib():
             "orc_merge_partitions": (i64, [P(Params), pu16, pi32, i32, i32, pi64, pd]),
             "orc_clip_at": (i32, [P(Params), P(Hist), P(Source), d, d, i32, pd, pd]),
             "orc_dists_at": (None, [P(Params), P(Hist), P(Source), d, d, i32, d, pd, pd]),
+            "orc_centre_at": (None, [P(Params), P(Hist), P(Source), d, d, i32, d, pd, pd, pd]),
             "orc_inner_at": (i64, [P(Params), P(Hist), P(Source), d, d, i32, d, pd]),
             "orc_integrand_at": (None, [P(Params), P(Hist), P(Source), i32, d, d, d, pd]),
             "orc_gk15_at": (None, [P(Params), P(Hist), P(Source), d, d, i32, d, d, pd, pd, pd]),
@@ -260,6 +261,13 @@ class Problem:
         lib().orc_dists_at(C.byref(self.params), C.byref(self.hist), C.byref(self.source),
                            px, py, j, r, C.byref(a), C.byref(b))
         return a.value, b.value
+
+    def centre(self, px, py, j, r):
+        """Frame-local circle centre at radius r of subregion j and the time weights."""
+        cu, cv, w = C.c_double(), C.c_double(), np.zeros(3)
+        lib().orc_centre_at(C.byref(self.params), C.byref(self.hist), C.byref(self.source),
+                            px, py, j, r, C.byref(cu), C.byref(cv), _pd(w))
+        return cu.value, cv.value, w
 
     def inner(self, px, py, j, r):
         out = np.zeros(3)

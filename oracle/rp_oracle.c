@@ -878,6 +878,16 @@ void orc_dists_at(const orc_params* P, const orc_hist* Hh, const orc_source* S, 
   dists_at(&X, r, dmin2, dmax2);
 }
 
+/* Frame-local centre (c_u, c_v) of the circle about lab point p at radius r of subregion j,
+ * i.e. p in the frame interpolated to the retarded time t' = k dt - r/c (R-7), and the time
+ * weights of levels (l0, l1, l2) there. */
+void orc_centre_at(const orc_params* P, const orc_hist* Hh, const orc_source* S, double px,
+                   double py, int32_t j, double r, double* cu, double* cv, double* w) {
+  subctx X;
+  setup_sub(&X, P, Hh, S, px, py, j);
+  centre_at(&X, r, cu, cv, w);
+}
+
 int64_t orc_inner_at(const orc_params* P, const orc_hist* Hh, const orc_source* S, double px,
                      double py, int32_t j, double r, double* out) {
   subctx X;

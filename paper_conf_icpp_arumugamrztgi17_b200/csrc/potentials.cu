@@ -46,6 +46,7 @@ enum : int { C_ITEMS = 0, C_NEXT = 1, C_EVALS = 2, C_SEGS = 3, C_LEAVES = 4, C_C
              C_TIES = 6, C_MAXLEV = 7, C_NODES = 8, C_NOUT = 9, C_SKIP = 10, C_UNITS = 11,
              C_NEXT_U = 12, C_UOVF = 13, C_COUNT = 16 };
 constexpr int kUnitShift = 20;  // unit key = item << 20 | index of the subtree root at its level
+constexpr uint32_t kEmptyKey = 0xFFFFFFFFu;  // schedule key of an item without support
 
 constexpr double kTwoPi = 6.283185307179586476925286766559;
 constexpr int kMaxArcs = 8;
@@ -209,14 +210,14 @@ template <int KIND>
 __global__ void k_clip(Params P, const int32_t* __restrict__ owner, int rank,
                        const uint16_t* __restrict__ cost_prev, int policy, int knn,
                        double2* __restrict__ AB,
-                       uint16_t* __restrict__ key, int32_t* __restrict__ iota,
+                       uint32_t* __restrict__ key, int32_t* __restrict__ iota,
                        unsigned long long* __restrict__ counters) {
   int64_t id = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
   int64_t total = (int64_t)P.npts * P.kmax;
   if (id >= total) return;
   iota[id] = (int32_t)id;
   int p = (int)(id / P.kmax), j = (int)(id % P.kmax);
-  uint16_t kk = 0xFFFF;
+  uint32_t kk = kEmptyKey;
   double A = 0.0, B = 0.0;
   if (j < P.kap && (owner == nullptr || owner[p] == rank)) {
     Item it;
@@ -259,14 +260,18 @@ __global__ void k_clip(Params P, const int32_t* __restrict__ owner, int rank,
         // (DESIGN.md sec. 3), so run it first; later steps use last step's counts
         unsigned c = cost_prev ? forecast(cost_prev, p, j, P.nx, P.ny, P.kmax, policy, knn)
                                : (policy == RP_SCHED_INDEX ? 0u : (j == 0 ? 1u : 0u));
-        kk = (uint16_t)(0xFFFEu - (c < 0xFFFEu ? c : 0xFFFEu));
+        kk = 0xFFFEu - (c < 0xFFFEu ? c : 0xFFFEu);
+        // subregion-major order (j ascending, longest-predicted-first within j): concurrent
+        // warps share the 3 history levels of one subregion, so the slab stays L2-resident
+        // when the ring does not fit in L2 (configs 4-5)
+        if (policy == RP_SCHED_SUBREGION) kk |= (uint32_t)min(j, 0xFFFE) << 16;
       }
     }
   }
   AB[id] = make_double2(A, B);
   key[id] = kk;
   // count items: warp aggregate then one atomic per warp (integer -> deterministic)
-  unsigned m = __ballot_sync(__activemask(), kk != 0xFFFF);
+  unsigned m = __ballot_sync(__activemask(), kk != kEmptyKey);
   if ((threadIdx.x & 31) == (__ffs(__activemask()) - 1) && m)
     atomicAdd(&counters[C_ITEMS], (unsigned long long)__popc(m));
 }
@@ -1025,7 +1030,7 @@ __global__ void k_merge_units(long long n, const unsigned long long* __restrict_
 }
 
 // ------------------------------------------------------------- k_reduce
-__global__ void k_reduce(int npts, int kmax, int kap, const uint16_t* __restrict__ key,
+__global__ void k_reduce(int npts, int kmax, int kap, const uint32_t* __restrict__ key,
                          const double4* __restrict__ val, const int4* __restrict__ cnt,
                          const uint2* __restrict__ aux, const int32_t* __restrict__ owner,
                          int rank, const int32_t* __restrict__ row_of, int world,
@@ -1043,7 +1048,7 @@ __global__ void k_reduce(int npts, int kmax, int kap, const uint16_t* __restrict
   int ml = 0;
   for (int j = 0; j < kmax; ++j) {
     size_t id = (size_t)p * kmax + j;
-    if (j >= kap || key[id] == 0xFFFF) {
+    if (j >= kap || key[id] == kEmptyKey) {
       cost[id] = 0;
       leaves[id] = 0;
       continue;
@@ -1126,8 +1131,8 @@ int rp_alloc_potential_scratch(rp_ctx* ctx) {
   const rp_config& c = ctx->cfg;
   size_t npts = (size_t)c.nx * c.ny, nd = npts * c.history_depth;
   RP_CUDA(cudaMalloc(&ctx->clipAB, nd * sizeof(double2)));
-  RP_CUDA(cudaMalloc(&ctx->sched_key, nd * sizeof(uint16_t)));
-  RP_CUDA(cudaMalloc(&ctx->sched_key_sorted, nd * sizeof(uint16_t)));
+  RP_CUDA(cudaMalloc(&ctx->sched_key, nd * sizeof(uint32_t)));
+  RP_CUDA(cudaMalloc(&ctx->sched_key_sorted, nd * sizeof(uint32_t)));
   RP_CUDA(cudaMalloc(&ctx->sched_idx, nd * sizeof(int32_t)));
   RP_CUDA(cudaMalloc(&ctx->sched_order, nd * sizeof(int32_t)));
   RP_CUDA(cudaMalloc(&ctx->cost_prev, nd * sizeof(uint16_t)));
@@ -1297,15 +1302,16 @@ static int run_potentials(rp_ctx* ctx, Params P, int32_t rank, int32_t world,
     }
     {
       ProfScope ps(ctx, PK_SORT);
+      const int kbits = ctx->sched_policy == RP_SCHED_SUBREGION ? 32 : 16;
       size_t tmp = 0;
       RP_CUDA(cub::DeviceRadixSort::SortPairs(nullptr, tmp, ctx->sched_key, ctx->sched_key_sorted,
-                                              ctx->sched_idx, ctx->sched_order, (int)nd, 0, 16, st));
+                                              ctx->sched_idx, ctx->sched_order, (int)nd, 0, kbits, st));
       int rc = rp_ensure_cub_tmp(ctx, tmp);
       if (rc) return rc;
       tmp = ctx->cub_tmp_bytes;
       RP_CUDA(cub::DeviceRadixSort::SortPairs(ctx->cub_tmp, tmp, ctx->sched_key,
                                               ctx->sched_key_sorted, ctx->sched_idx,
-                                              ctx->sched_order, (int)nd, 0, 16, st));
+                                              ctx->sched_order, (int)nd, 0, kbits, st));
     }
     const int var = KIND != RP_SRC_GRID ? 0 : (P.interp == RP_INTERP_LAGRANGE3 ? 6 : ctx->eval_variant);
     ctx->pred_info.active = 0;

@@ -91,7 +91,7 @@ int64_t rp_launch_count(const rp_ctx* ctx) { return ctx ? ctx->launches : 0; }
 
 int rp_set_schedule(rp_ctx* ctx, int32_t policy, int32_t k) {
   if (!ctx) return RP_EINVAL;
-  if (policy < RP_SCHED_INDEX || policy > RP_SCHED_KNN) return rp_fail(ctx, RP_EINVAL, "set_schedule: policy");
+  if (policy < RP_SCHED_INDEX || policy > RP_SCHED_SUBREGION) return rp_fail(ctx, RP_EINVAL, "set_schedule: policy");
   if (policy == RP_SCHED_KNN && k != 1 && k != 5 && k != 9 && k != 25)
     return rp_fail(ctx, RP_EINVAL, "set_schedule: k must be 1, 5, 9 or 25");
   ctx->sched_policy = policy;

@@ -47,8 +47,8 @@ struct rp_ctx {
 
   // potentials scratch: dense (point, subregion) arrays of npts * kappa_max
   double2* clipAB = nullptr;        // [A, B] per (p, j)
-  uint16_t* sched_key = nullptr;    // sort keys (0xFFFF = empty)
-  uint16_t* sched_key_sorted = nullptr;
+  uint32_t* sched_key = nullptr;    // sort keys (0xFFFFFFFF = empty)
+  uint32_t* sched_key_sorted = nullptr;
   int32_t* sched_idx = nullptr;     // iota
   int32_t* sched_order = nullptr;   // sorted item ids (p * kappa_max + j)
   uint16_t* cost_prev = nullptr;    // forecast: previous step's segments per (p, j)

@@ -17,7 +17,7 @@ _HERE = os.path.dirname(os.path.abspath(__file__))
 LIB_PATH = os.path.join(_HERE, "librp.so")
 
 RP_SRC_GRID, RP_SRC_GAUSS, RP_SRC_DISK = 0, 1, 2
-RP_SCHED_INDEX, RP_SCHED_PERSISTENCE, RP_SCHED_KNN = 0, 1, 2
+RP_SCHED_INDEX, RP_SCHED_PERSISTENCE, RP_SCHED_KNN, RP_SCHED_SUBREGION = 0, 1, 2, 3
 RP_RULE_GK15, RP_RULE_SIMPSON = 0, 1
 
 
