@@ -2,14 +2,24 @@
 """Benchmark of the retarded-potential step (BASELINE.json metric: mesh-point potentials/s
 and FP64 GFLOP/s per step at 1/2/4/8 B200).
 
-    python bench.py [--gpus N] [--steps K] [--warmup W] [--config 2] [--impl ours|reference]
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--config 5] [--impl ours|reference]
 
-One step = the whole hot path of the paper's loop on BASELINE.json configs[1]
-(config 2: 64x64 mesh, 1e6 particles, LCLS bend, full retarded history kappa = 100):
-deposit -> retarded potentials at every mesh point -> self-fields -> push.  Inputs are
-seeded synthetic (workloads/); the timed region starts with everything resident in HBM.
-For N > 1 run under torchrun: mesh points are sharded and the history replicated (strong
-scaling: the same mesh and bunch for every N).  Rank 0 prints ONE JSON line.
+One step = the whole hot path of the paper's loop: deposit -> retarded potentials at
+every mesh point -> self-fields -> push.  Default workload: BASELINE.json configs[4] (config 5:
+512x512 mesh, 1e8 particles, LCLS bend, full retarded history kappa = 2000), the strong-scaling
+configuration the metric is quoted on; `--config 1..4` runs the others.  Inputs are seeded
+synthetic (workloads/).
+
+One timed pass serves both numbers.  Every step goes through the C ABI's end-to-end call
+rp_step_host with PINNED HOST buffers (H2D of this rank's particles, the step, D2H of the pushed
+particles and the six mesh outputs): CUDA events around the call give `e2e`; librp's own
+events around the step's device part (deposit through push, between the copies) give `value`,
+the throughput with inputs resident in HBM.  N > 1: one process per GPU (torchrun, or
+self-spawned when WORLD_SIZE is unset); librp owns an NCCL communicator (unique id broadcast
+over torch.distributed) and all-gathers inside its calls; mesh points are sharded, the history
+replicated (strong scaling: the same mesh and bunch for every N); times are the max over ranks.
+RP_DIST_BACKEND=gloo instead runs the caller-side transport (torch gloo all-gathers around
+librp's shard calls) so several ranks can share one GPU.
 
 --impl reference times the CPU oracle (oracle/, test infrastructure; the one other place
 bench.py may execute it) on the same workload, a bounded sample of mesh points per step.
@@ -17,9 +27,10 @@ bench.py may execute it) on the same workload, a bounded sample of mesh points p
 from __future__ import annotations
 
 import argparse
+import hashlib
 import json
-import math
 import os
+import socket
 import statistics
 import subprocess
 import sys
@@ -37,6 +48,9 @@ import workloads as W  # noqa: E402
 F_EVAL = 210   # one integrand evaluation f(r', theta', t'): 27-point TSC x Lagrange-3 gather
 F_NODE = 100   # one r' node: retarded frame, circle centre, arcs
 F_SEG = 60     # one GK15 segment: K15/G7 sums, error, decision
+METRIC = "mesh-point potentials/sec (and FP64 GFLOP/s per step)"
+UNIT = "mesh-point potentials/s"
+L2_BYTES = 126 * 2 ** 20
 
 
 def algorithmic_flops(info: dict) -> float:
@@ -75,14 +89,15 @@ def measured_peaks():
     return out
 
 
-def ncu_traffic():
-    """Per-launch DRAM bytes of the integrator from the committed ncu --set full summary."""
+def ncu_traffic(cfg_number: int):
+    """DRAM bytes (read + write) of one integrator call of THIS config, from the committed ncu
+    capture of the same workload (profiles/ncu_traffic_cfg<N>.json); None if there is none."""
     try:
-        with open(os.path.join(ROOT, "profiles", "ncu_integrate.json")) as f:
+        with open(os.path.join(ROOT, "profiles", f"ncu_traffic_cfg{cfg_number}.json")) as f:
             d = json.load(f)
-        return d.get("dram_bytes_per_launch")
+        return d.get("dram_bytes_per_call"), d.get("source")
     except Exception:
-        return None
+        return None, None
 
 
 class ClockSampler:
@@ -136,109 +151,199 @@ class ClockSampler:
                 "samples": len(sm)}
 
 
+def _free_port() -> int:
+    with socket.socket() as sk:
+        sk.bind(("127.0.0.1", 0))
+        return sk.getsockname()[1]
+
+
+def self_spawn(argv, n) -> int:
+    """`--gpus N` without torchrun: relaunch this script as N ranks (one per GPU)."""
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", "--nproc-per-node",
+           str(n), "--master-addr", "127.0.0.1", "--master-port", str(_free_port()),
+           os.path.abspath(__file__), *argv]
+    return subprocess.call(cmd)
+
+
+def _cores():
+    try:
+        return len(os.sched_getaffinity(0))
+    except Exception:
+        return os.cpu_count() or 1
+
+
+def _set_schedule(rp, ctx, sched):
+    if sched == "index":
+        rp.rp_set_schedule(ctx, rp.RP_SCHED_INDEX, 1)
+    elif sched == "persistence":
+        rp.rp_set_schedule(ctx, rp.RP_SCHED_PERSISTENCE, 1)
+    elif sched == "subregion":
+        rp.rp_set_schedule(ctx, rp.RP_SCHED_SUBREGION, 1)
+    elif sched.startswith("knn"):
+        rp.rp_set_schedule(ctx, rp.RP_SCHED_KNN, int(sched[3:]))
+    else:
+        raise SystemExit(f"unknown schedule {sched}")
+
+
 # ---------------------------------------------------------------------------- our arm
 def run_ours(args):
     import torch
     import torch.distributed as dist
 
     from paper_conf_icpp_arumugamrztgi17_b200 import rp
-    from paper_conf_icpp_arumugamrztgi17_b200.sim import Simulation
 
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
-    local = int(os.environ.get("LOCAL_RANK", "0")) % max(1, __import__("torch").cuda.device_count())
-    if args.gpus != world:
-        if world == 1 and args.gpus > 1:
-            raise SystemExit("--gpus N > 1 must be launched with torchrun (one rank per GPU)")
-    torch.cuda.set_device(local % max(1, torch.cuda.device_count()))
-    group = None
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    backend = os.environ.get("RP_DIST_BACKEND", "nccl")
+    ngpu = max(1, torch.cuda.device_count())
+    dev_index = local % ngpu
+    torch.cuda.set_device(dev_index)
+    dev = torch.device("cuda", dev_index)
     if world > 1:
-        backend = os.environ.get("RP_DIST_BACKEND", "nccl")  # gloo: 2 ranks on 1 GPU (tests)
         if backend == "nccl":
-            dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+            os.environ.setdefault("NCCL_DEBUG", "INFO")  # rank count visible on stderr
+            dist.init_process_group("nccl", device_id=dev)
         else:
             dist.init_process_group(backend)
-        group = dist.group.WORLD
     cfg = W.config(args.config)
     cfg.rule = 1 if args.rule == "simpson" else 0
     cfg.interp = 1 if args.interp == "lagrange3" else 0
-    sim = Simulation(cfg, group=group)
-    sched = args.schedule
-    if sched == "index":
-        rp.rp_set_schedule(sim.ctx, rp.RP_SCHED_INDEX, 1)
-    elif sched == "subregion":
-        rp.rp_set_schedule(sim.ctx, rp.RP_SCHED_SUBREGION, 1)
-    elif sched.startswith("knn"):
-        rp.rp_set_schedule(sim.ctx, rp.RP_SCHED_KNN, int(sched[3:]))
-    dev = torch.device("cuda", local)
-    flush = torch.empty(512 * 1024 * 1024 // 8, dtype=torch.float64, device=dev)  # 512 MB > L2
+    npts = cfg.nx * cfg.ny
+    ring_bytes = cfg.H * (cfg.nx + 6) * (cfg.ny + 6) * 32
+    flush_l2 = ring_bytes <= 4 * L2_BYTES
+    flush = torch.empty(512 * 1024 * 1024 // 8, dtype=torch.float64, device=dev) if flush_l2 else None
 
     def barrier():
         if world > 1:
             dist.barrier()
         torch.cuda.synchronize()
 
+    def max_over_ranks(v):
+        if world == 1:
+            return v
+        t = torch.tensor([v], dtype=torch.float64, device=dev)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        return float(t.item())
+
+    def sum_over_ranks(d):
+        if world == 1:
+            return d
+        t = torch.tensor(list(d.values()), dtype=torch.float64, device=dev)
+        dist.all_reduce(t)
+        return {k: int(v) for k, v in zip(d, t.tolist())}
+
+    x, y, ux, uy = W.particles(cfg)
+    n_all = len(x)
+    lo, hi = (n_all * rank) // world, (n_all * (rank + 1)) // world
+    host = [torch.from_numpy(np.ascontiguousarray(a[lo:hi])).pin_memory() for a in (x, y, ux, uy)]
+    del x, y, ux, uy
+    q = 1.0 / n_all
+    mesh = torch.zeros((6, npts), dtype=torch.float64).pin_memory()
+    stream = torch.cuda.current_stream(dev)
+    totals = {"evals": 0, "skipped": 0, "nodes": 0, "segments": 0, "capped": 0, "items": 0,
+              "units": 0}
+    e2e_ms = []
+    sim = ctx = None
+    in_lib = world == 1 or backend == "nccl"
+    if in_lib:
+        # the product path: librp owns the exchange (an NCCL communicator when world > 1)
+        dist_arg = None
+        if world > 1:
+            obj = [rp.rp_nccl_unique_id() if rank == 0 else None]
+            dist.broadcast_object_list(obj, src=0)
+            dist_arg = (rank, world, obj[0])
+        ctx = rp.rp_create(cfg.nx, cfg.ny, cfg.hx, cfg.hy, cfg.kappa_max, cfg.c, cfg.dt, cfg.tau,
+                           cfg.n_theta, cfg.max_depth, cfg.n_root, dev_index, cfg.rule, cfg.interp,
+                           dist=dist_arg)
+        rp.rp_set_stream(ctx, stream)
+        rp.rp_history_init(ctx, cfg.n_pre, W.frames(cfg, range(-cfg.n_pre, 0)), None, True)
+    else:
+        from paper_conf_icpp_arumugamrztgi17_b200.sim import Simulation
+        sim = Simulation(cfg, group=dist.group.WORLD, transport="host")
+        ctx = sim.ctx
+    _set_schedule(rp, ctx, args.schedule)
+    dev_events = []
+
+    def one_step(k, info):
+        if in_lib:
+            return rp.rp_step_host(ctx, *host, q, W.frame(cfg, k), cfg.q_over_mc, cfg.bz_ext, mesh,
+                                   info=info)
+        # caller-side transport: the same host copies around Simulation.step (torch copies)
+        for d, h in zip((sim.x, sim.y, sim.ux, sim.uy), host):
+            d.copy_(h, non_blocking=True)
+        m0 = torch.cuda.Event(enable_timing=True)
+        m1 = torch.cuda.Event(enable_timing=True)
+        m0.record(stream)
+        inf = sim.step(info=info)
+        m1.record(stream)
+        for i, t in enumerate((sim.phi, sim.ax, sim.ay, sim.ex, sim.ey, sim.bz)):
+            mesh[i].copy_(t, non_blocking=True)
+        for d, h in zip((sim.x, sim.y, sim.ux, sim.uy), host):
+            h.copy_(d, non_blocking=True)
+        dev_events.append((m0, m1))
+        return inf
+
+    k = 0
     for _ in range(args.warmup):
-        sim.step()
+        one_step(k, False)
+        k += 1
     barrier()
-    launches0 = rp.rp_launch_count(sim.ctx)
-    rp.rp_profile_enable(sim.ctx, True)
-    stream = torch.cuda.current_stream()
-    clocks = ClockSampler(local)
+    dev_events.clear()
+    launches0 = rp.rp_launch_count(ctx)
+    rp.rp_profile_enable(ctx, True)
+    clocks = ClockSampler(dev_index)
     clocks.start()
     barrier()
-    step_ms = []
-    totals = {"evals": 0, "skipped": 0, "nodes": 0, "segments": 0, "capped": 0, "items": 0,
-              "units": 0, "unit_overflow": 0}
     for _ in range(args.steps):
-        flush.fill_(1.0)  # evict L2 between timed steps (outside the events)
+        if flush is not None:
+            flush.fill_(1.0)  # evict L2 between timed steps (outside the events)
         e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         e0.record(stream)
-        inf = sim.step(info=True)
+        inf = one_step(k, True)
         e1.record(stream)
         e1.synchronize()
-        step_ms.append(e0.elapsed_time(e1))
-        for k2 in totals:
-            totals[k2] += getattr(inf, k2)
+        e2e_ms.append(e0.elapsed_time(e1))
+        for key in totals:
+            totals[key] += getattr(inf, key)
+        k += 1
     barrier()
     clk = clocks.stop()
-    prof = rp.rp_profile_read(sim.ctx).as_dict()
-    rp.rp_profile_enable(sim.ctx, False)
-    launches = rp.rp_launch_count(sim.ctx) - launches0
-    local_ms = sum(step_ms)
-    if world > 1:
-        t = torch.tensor([local_ms], dtype=torch.float64, device=dev)
-        dist.all_reduce(t, op=dist.ReduceOp.MAX)
-        total_ms = float(t.item())
-        c = torch.tensor([totals[k2] for k2 in totals], dtype=torch.float64, device=dev)
-        dist.all_reduce(c)
-        totals = {k2: int(v) for k2, v in zip(totals, c.tolist())}
-        p = torch.tensor([prof["integrate_ms"]], dtype=torch.float64, device=dev)
-        dist.all_reduce(p, op=dist.ReduceOp.MAX)
-        prof["integrate_ms"] = float(p.item())
+    prof = rp.rp_profile_read(ctx).as_dict()
+    rp.rp_profile_enable(ctx, False)
+    launches = rp.rp_launch_count(ctx) - launches0
+    if in_lib:
+        dev_ms = prof["step_ms"]
     else:
-        total_ms = local_ms
-    npts = cfg.nx * cfg.ny
+        dev_ms = sum(a.elapsed_time(b) for a, b in dev_events)
+    total_ms = max_over_ranks(dev_ms)
+    total_e2e = max_over_ranks(sum(e2e_ms))
+    integ_max = max_over_ranks(prof["integrate_ms"])
+    totals = sum_over_ranks(totals)
     value = npts * args.steps / (total_ms * 1e-3)
     flops_total = algorithmic_flops(totals)
     gflops = flops_total / (total_ms * 1e-3) / 1e9
-
-    # ---- end-to-end through the C ABI with host buffers (pinned), every step:
-    # H2D of the particles, the whole step, D2H of the pushed particles + six mesh outputs.
-    e2e = None
-    if not args.no_e2e:
-        e2e = run_e2e(cfg, args, dev) if world == 1 else run_e2e_dist(cfg, args, dev, group)
-
+    digest = hashlib.sha256(mesh.numpy().tobytes()).hexdigest()[:16]
+    pbytes = 4 * host[0].numel() * 8
+    e2e = {"value": npts * args.steps / (total_e2e * 1e-3), "unit": UNIT,
+           "h2d_bytes_per_step": pbytes, "d2h_bytes_per_step": pbytes + 6 * npts * 8,
+           "ms_per_step": total_e2e / args.steps,
+           "bytes_per": "rank 0 (its particle shard)" if world > 1 else "the whole job",
+           "api": ("rp_step_host (C ABI, pinned host buffers)" if in_lib else
+                   "sim.Simulation.step with pinned host copies (torch, gloo transport)")}
     peaks = measured_peaks()
+    cpu = None
+    if rank == 0 and world == 1 and not args.no_cpu_baseline:
+        cpu = cpu_baseline(cfg, args, rp, ctx, dev, value, totals)
     if rank == 0:
-        integ_ms_avg = prof["integrate_ms"] / max(1, prof["integrate_launches"])
+        integ_ms_avg = integ_max / max(1, prof["integrate_launches"])
         flops_per_launch = flops_total / args.steps / max(1, world)
         achieved = flops_per_launch / (integ_ms_avg * 1e-3) / 1e12 if integ_ms_avg > 0 else 0.0
-        traffic = ncu_traffic()
+        traffic, tsrc = ncu_traffic(cfg.number)
         line = {
-            "metric": "mesh-point potentials/sec (and FP64 GFLOP/s per step)",
+            "metric": METRIC,
             "value": value,
-            "unit": "mesh-point potentials/s",
+            "unit": UNIT,
             "n_gpus": world,
             "steps": args.steps,
             "warmup": args.warmup,
@@ -252,156 +357,101 @@ def run_ours(args):
                        "particles": cfg.n_particles, "history_depth": cfg.kappa_max,
                        "tau": cfg.tau, "n_theta": cfg.n_theta, "n_root": cfg.n_root,
                        "parallelism": f"mesh-point shards x{world}, history replicated",
-                       "l2": "flushed between timed steps (512 MB write)",
+                       "transport": ("none" if world == 1 else "librp NCCL all-gathers" if in_lib
+                                     else f"caller-side {backend} all-gathers"),
+                       "l2": ("flushed between timed steps (512 MB write)" if flush_l2 else
+                              f"inputs larger than L2 (ring {ring_bytes / 2 ** 30:.1f} GiB)"),
                        "schedule": args.schedule, "outer_rule": args.rule,
                        "interp": args.interp},
             "fp64_gflops": gflops,
+            "evals_per_s": totals["evals"] / (total_ms * 1e-3),
             "work_per_step": {k2: v / args.steps for k2, v in totals.items()},
             "roofline": {"kernel": "k_integrate (GK15 tree integrator)", "bound": "alu",
                          "achieved": achieved, "peak": peaks["fp64_tflops"], "unit": "TFLOP/s",
                          "frac": achieved / peaks["fp64_tflops"], "traffic": traffic,
+                         "traffic_source": tsrc,
                          "peak_source": peaks["fp64_source"],
-                         "share_of_step": prof["integrate_ms"] / total_ms if world == 1 else None,
-                         "avg_launch_ms": integ_ms_avg},
+                         "share_of_step": prof["integrate_ms"] / dev_ms if dev_ms else None,
+                         "avg_launch_ms": integ_ms_avg,
+                         "algorithmic_flops_per_launch": flops_per_launch},
             "kernel_ms_per_step": {k2: v / args.steps for k2, v in prof.items() if k2.endswith("_ms")},
             "gpu_launches": launches,
             "clocks": clk,
             "e2e": e2e,
+            "result_sha256": digest,
             "paper_context": "485 DP GFLOP/s and 2.5x on one Tesla K40 (PAPER.md P:11, P:255)",
         }
-        if world == 1 and not args.no_cpu_baseline:
-            line["cpu_baseline"] = cpu_baseline(cfg, args)
+        if cpu is not None:
+            line["cpu_baseline"] = cpu
         print(json.dumps(line), flush=True)
-    sim.close()
+    if sim is not None:
+        sim.close()
+    else:
+        rp.rp_destroy(ctx)
     if world > 1:
         dist.barrier()
         dist.destroy_process_group()
 
 
-def run_e2e_dist(cfg, args, dev, group):
-    """N > 1: each rank copies its particle shard from pinned host memory, runs the sharded
-    step, and copies the full-mesh potentials and fields (and its pushed shard) back.  Time is
-    the max over ranks of the CUDA-event time on the step's stream."""
-    import torch
-    import torch.distributed as dist
-
-    from paper_conf_icpp_arumugamrztgi17_b200.sim import Simulation
-    sim = Simulation(cfg, group=group)
-    host = [t.detach().cpu().pin_memory() for t in (sim.x, sim.y, sim.ux, sim.uy)]
-    npts = cfg.nx * cfg.ny
-    mesh = torch.zeros((6, npts), dtype=torch.float64).pin_memory()
-    stream = torch.cuda.current_stream()
-    for _ in range(args.warmup):
-        sim.step()
-    dist.barrier()
-    torch.cuda.synchronize()
-    ms = 0.0
-    for _ in range(args.steps):
-        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-        e0.record(stream)
-        for d, h in zip((sim.x, sim.y, sim.ux, sim.uy), host):
-            d.copy_(h, non_blocking=True)
-        sim.step()
-        for i, t in enumerate((sim.phi, sim.ax, sim.ay, sim.ex, sim.ey, sim.bz)):
-            mesh[i].copy_(t, non_blocking=True)
-        for d, h in zip((sim.x, sim.y, sim.ux, sim.uy), host):
-            h.copy_(d, non_blocking=True)
-        e1.record(stream)
-        e1.synchronize()
-        ms += e0.elapsed_time(e1)
-    t = torch.tensor([ms], dtype=torch.float64, device=dev)
-    dist.all_reduce(t, op=dist.ReduceOp.MAX)
-    ms = float(t.item())
-    sim.close()
-    pbytes = 4 * sim.x.numel() * 8
-    return {"value": npts * args.steps / (ms * 1e-3), "unit": "mesh-point potentials/s",
-            "h2d_bytes_per_step": pbytes, "d2h_bytes_per_step": pbytes + 6 * npts * 8,
-            "ms_per_step": ms / args.steps, "bytes_per": "rank 0 (particle shard)",
-            "api": "sim.Simulation.step with pinned host copies (torch) around the C-ABI calls"}
-
-
-def run_e2e(cfg, args, dev):
-    import torch
-
-    from paper_conf_icpp_arumugamrztgi17_b200 import rp
-    x, y, ux, uy = W.particles(cfg)
-    hx, hy, hux, huy = (torch.tensor(a).pin_memory() for a in (x, y, ux, uy))
-    npts = cfg.nx * cfg.ny
-    mesh = torch.zeros((6, npts), dtype=torch.float64).pin_memory()
-    ctx = rp.rp_create(cfg.nx, cfg.ny, cfg.hx, cfg.hy, cfg.kappa_max, cfg.c, cfg.dt, cfg.tau,
-                       cfg.n_theta, cfg.max_depth, cfg.n_root, dev.index or 0, cfg.rule,
-                       cfg.interp)
-    try:
-        stream = torch.cuda.current_stream()
-        rp.rp_set_stream(ctx, stream)
-        rp.rp_history_init(ctx, cfg.n_pre, W.frames(cfg, range(-cfg.n_pre, 0)), None, True)
-        k = 0
-        for _ in range(args.warmup):
-            rp.rp_step_host(ctx, hx, hy, hux, huy, 1.0 / len(x), W.frame(cfg, k), cfg.q_over_mc,
-                            cfg.bz_ext, mesh)
-            k += 1
-        torch.cuda.synchronize()
-        ms = 0.0
-        for _ in range(args.steps):
-            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-            e0.record(stream)
-            rp.rp_step_host(ctx, hx, hy, hux, huy, 1.0 / len(x), W.frame(cfg, k), cfg.q_over_mc,
-                            cfg.bz_ext, mesh)
-            e1.record(stream)
-            e1.synchronize()
-            ms += e0.elapsed_time(e1)
-            k += 1
-        pbytes = 4 * len(x) * 8
-        return {"value": npts * args.steps / (ms * 1e-3), "unit": "mesh-point potentials/s",
-                "h2d_bytes_per_step": pbytes, "d2h_bytes_per_step": pbytes + 6 * npts * 8,
-                "ms_per_step": ms / args.steps, "api": "rp_step_host (C ABI, pinned host buffers)"}
-    finally:
-        rp.rp_destroy(ctx)
-
-
 # ---------------------------------------------------------------------------- oracle arm
-def _oracle_state(cfg):
+def _problem(cfg, ring, frames, k):
+    import oracle
+    return oracle.Problem(nx=cfg.nx, ny=cfg.ny, hx=cfg.hx, hy=cfg.hy, c=cfg.c, dt=cfg.dt,
+                          tau=cfg.tau, kappa_max=cfg.kappa_max, k=k, n_pre=cfg.n_pre, ring=ring,
+                          frames=frames, n_theta=cfg.n_theta, max_depth=cfg.max_depth,
+                          n_root=cfg.n_root, rule=cfg.rule, interp=cfg.interp)
+
+
+def _oracle_rigid_state(cfg):
+    """The oracle's own step-0 state: its deposit of the seeded bunch + the rigid pre-history."""
     import oracle
     oracle.set_threads(_cores())  # all host cores, whatever OMP_NUM_THREADS torchrun set
     x, y, ux, uy = W.particles(cfg)
     q = 1.0 / len(x)
-    t0 = time.perf_counter()
     M, _, _ = oracle.deposit(x, y, ux, uy, q, W.frame(cfg, 0), cfg.nx, cfg.ny, cfg.hx, cfg.hy)
-    t_dep = time.perf_counter() - t0
+    del x, y, ux, uy
     ring = oracle.rigid_ring(M, W.ring_frames(cfg, 0))
-    P = oracle.Problem(nx=cfg.nx, ny=cfg.ny, hx=cfg.hx, hy=cfg.hy, c=cfg.c, dt=cfg.dt, tau=cfg.tau,
-                       kappa_max=cfg.kappa_max, k=0, n_pre=cfg.n_pre, ring=ring,
-                       frames=W.ring_frames(cfg, 0), n_theta=cfg.n_theta, max_depth=cfg.max_depth,
-                       n_root=cfg.n_root)
-    return P, t_dep
+    return _problem(cfg, ring, W.ring_frames(cfg, 0), 0)
 
 
-def _cores():
-    try:
-        return len(os.sched_getaffinity(0))
-    except Exception:
-        return os.cpu_count() or 1
-
-
-def cpu_baseline(cfg, args, budget_s: float = 15.0):
-    """The oracle as it stands, all host cores (OpenMP), on a bounded stratified sample of
-    the mesh points of step 0 of the same workload."""
-    P, t_dep = _oracle_state(cfg)
-    npts = cfg.nx * cfg.ny
-    order = W.sample_points(cfg.nx, cfg.ny, npts, seed=0)
-    rng = np.random.default_rng(2)
-    order = rng.permutation(order).astype(np.int32)
-    done, t = 0, 0.0
-    while done < npts and t < budget_s:
-        chunk = order[done:done + 64]
+def _time_sample(P, order, budget_s, chunk):
+    done, t, evals = 0, 0.0, 0
+    while done < len(order) and t < budget_s:
+        pts = order[done:done + chunk]
         t0 = time.perf_counter()
-        P.potentials(chunk)
+        res = P.potentials(pts)
         t += time.perf_counter() - t0
-        done += len(chunk)
-    return {"value": done / t, "unit": "mesh-point potentials/s", "cores": _cores(),
-            "kind": "oracle",
-            "sample": f"{done} random mesh points of {cfg.name} step 0 (rigid history), "
-                      f"{t:.1f} s wall; oracle deposit of all particles {t_dep:.2f} s not included"}
+        evals += int(res["evals"].sum())
+        done += len(pts)
+    return done, t, evals
+
+
+def cpu_baseline(cfg, args, rp, ctx, dev, gpu_value, gpu_totals, budget_s: float = 15.0):
+    """The oracle as it stands, all host cores (OpenMP), on a bounded random sample of the mesh
+    points of the LAST TIMED STEP: the GPU's history ring and frames at that step are copied out
+    (rp_save_state), so both arms integrate the same state; reported per point and per
+    integrand evaluation (the work per point varies along the trajectory)."""
+    import oracle
+    import torch
+    oracle.set_threads(_cores())
+    ring = torch.zeros((cfg.H, cfg.ny, cfg.nx, 4), dtype=torch.float64, device=dev)
+    k, frames = rp.rp_save_state(ctx, ring, cfg.H)
+    ring_h = ring.cpu().numpy()
+    del ring
+    P = _problem(cfg, ring_h, frames, k)
+    npts = cfg.nx * cfg.ny
+    order = np.random.default_rng(2).permutation(npts).astype(np.int32)
+    chunk = max(4, min(64, 4 * _cores()))
+    done, t, evals = _time_sample(P, order, budget_s, chunk)
+    gpu_eps = gpu_totals["evals"] / args.steps * gpu_value / npts
+    return {"value": done / t, "unit": UNIT, "cores": _cores(), "kind": "oracle",
+            "evals_per_s": evals / t, "gpu_evals_per_s_same_steps": gpu_eps,
+            "sample": f"{done} random mesh points of {cfg.name} at step {k} (the last timed GPU "
+                      f"step: the GPU's ring and frames copied out), {t:.1f} s wall, "
+                      f"{evals / max(done, 1):.3g} integrand evaluations per point"}
+
+
+REF_SAMPLE = {1: 256, 2: 256, 3: 128, 4: 64, 5: 64}  # points per reference step (~seconds each)
 
 
 def run_reference(args):
@@ -410,30 +460,35 @@ def run_reference(args):
     if rank != 0:
         return
     cfg = W.config(args.config)
-    P, _ = _oracle_state(cfg)
-    sample = 256
+    P = _oracle_rigid_state(cfg)
+    sample = REF_SAMPLE.get(cfg.number, 64)
     order = np.random.default_rng(3).permutation(cfg.nx * cfg.ny).astype(np.int32)
     for w in range(args.warmup):
-        P.potentials(order[w * 16:(w + 1) * 16])
-    t = 0.0
+        P.potentials(order[w * 4:(w + 1) * 4])
+    t, evals = 0.0, 0
     for s in range(args.steps):
         pts = order[(s * sample) % len(order):][:sample]
         t0 = time.perf_counter()
-        P.potentials(pts)
+        res = P.potentials(pts)
         t += time.perf_counter() - t0
+        evals += int(res["evals"].sum())
     value = sample * args.steps / t
     print(json.dumps({
-        "impl": "reference", "metric": "mesh-point potentials/sec (and FP64 GFLOP/s per step)",
-        "value": value, "unit": "mesh-point potentials/s", "n_gpus": world,
+        "impl": "reference", "metric": METRIC,
+        "value": value, "unit": UNIT, "n_gpus": world,
         "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1e3 * t / args.steps,
         "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "f64",
         "data": "synthetic (seeded Gaussian bunch in the LCLS bend, workloads/)",
         "config": {"workload": cfg.name, "mesh": f"{cfg.nx}x{cfg.ny}",
                    "particles": cfg.n_particles, "history_depth": cfg.kappa_max},
-        "cpu_baseline": {"value": value, "unit": "mesh-point potentials/s", "cores": _cores(),
-                         "kind": "oracle",
-                         "sample": f"{sample} random mesh points per step of {cfg.name} step 0"},
-        "e2e": {"value": value, "unit": "mesh-point potentials/s", "h2d_bytes_per_step": 0,
+        "evals_per_s": evals / t,
+        "cpu_baseline": {"value": value, "unit": UNIT, "cores": _cores(), "kind": "oracle",
+                         "evals_per_s": evals / t,
+                         "sample": f"{sample} random mesh points per step of {cfg.name} at step 0 "
+                                   f"(the oracle's own deposit + rigid steady-state pre-history; "
+                                   f"{evals / (sample * args.steps):.3g} integrand evaluations "
+                                   f"per point)"},
+        "e2e": {"value": value, "unit": UNIT, "h2d_bytes_per_step": 0,
                 "d2h_bytes_per_step": 0},
     }), flush=True)
 
@@ -441,19 +496,20 @@ def run_reference(args):
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=int(os.environ.get("WORLD_SIZE", "1")))
-    ap.add_argument("--steps", type=int, default=5)
+    ap.add_argument("--steps", type=int, default=2)
     ap.add_argument("--warmup", type=int, default=3)
-    ap.add_argument("--config", type=int, default=2)
+    ap.add_argument("--config", type=int, default=5)
     ap.add_argument("--impl", choices=["ours", "reference"], default="ours")
-    ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--rule", default="gk15", choices=["gk15", "simpson"],
                     help="outer segment rule (simpson = the paper's RP-QUADRULE, a variant)")
     ap.add_argument("--interp", default="tsc", choices=["tsc", "lagrange3"],
                     help="spatial part of the 27-point stencil (lagrange3 = variant R-25)")
-    ap.add_argument("--schedule", default="persistence",
-                    help="work-order forecast: index | persistence | knn5 | knn9 | knn25")
+    ap.add_argument("--schedule", default="subregion",
+                    help="work-order forecast: index | persistence | subregion | knn5 | knn9 | knn25")
     args = ap.parse_args()
+    if args.gpus > 1 and "WORLD_SIZE" not in os.environ:
+        raise SystemExit(self_spawn(sys.argv[1:], args.gpus))
     if args.warmup < 3 and args.impl == "ours":
         print("warning: fewer than 3 warm-up steps", file=sys.stderr)
     if args.impl == "reference":

@@ -23,7 +23,14 @@
  *     the detailed message of the last failing call on that context.
  *   - FP64 everywhere (double-precision GFLOP/s).  Units are Gaussian with
  *     the caller's length/time units: phi = I_rho, A = I_{rho beta} (R-1).
- *   - One context per stream / host thread.  Contexts are independent.
+ *   - One context per stream / host thread.  Contexts are independent: every entry point
+ *     makes the context's device current and restores the caller's device before returning.
+ *   - Multi-GPU: one process and one context per GPU, created with an rp_dist.
+ *     Particles are sharded by the caller; the history ring is replicated; mesh points are
+ *     sharded inside rp_compute_potentials.  The two exchanges of a step (the partial moment
+ *     grids after deposition, the potential shards after integration) are NCCL all-gathers
+ *     issued by librp on the context's stream, so every output covers the full mesh on every
+ *     rank and the same calls serve N = 1 and N > 1.
  */
 #ifndef RP_H_
 #define RP_H_
@@ -38,6 +45,7 @@ extern "C" {
 #define RP_EINVAL (-1)  /* bad argument or configuration                      */
 #define RP_ENOMEM (-2)  /* device or host allocation failed                    */
 #define RP_ECUDA (-3)   /* CUDA runtime / kernel error (see rp_last_error)     */
+#define RP_ENCCL (-4)   /* NCCL unavailable or a collective failed             */
 #define RP_ESTATE (-5)  /* call out of order (e.g. potentials before deposit)  */
 #define RP_ENODEV (-6)  /* no usable CUDA device                               */
 
@@ -95,17 +103,42 @@ typedef struct {
                               padded TSC integrand vanishes (DESIGN R-24) or the Lagrange-3 one
                               takes its outside limit 0 (R-25b), not evaluated; the evaluations
                               performed are evals - skipped                                     */
-  int64_t units;           /* subtree work units walked separately (deep trees split at level 12,
-                              DESIGN sec. 6); 0 when the split is off                           */
-  int32_t unit_overflow;   /* 1 if the unit list was full and some subtrees were walked in place
-                              (same tree and values; only the summation grouping differs)       */
-  int32_t pad;
+  int64_t units;           /* subtree work units walked separately (deep near-field trees split at
+                              the work-split level, rp_set_work_split); 0 when off */
 } rp_potential_info;
+
+/* Multi-GPU membership of a context.  rank in [0, world).  Either nccl_comm is
+ * an initialised ncclComm_t of `world` ranks whose rank `rank` uses cfg->device (caller-owned,
+ * must outlive the context), or nccl_comm is NULL and nccl_id holds the bytes of one
+ * ncclUniqueId obtained by rank 0 from rp_nccl_unique_id and broadcast by the caller to every
+ * rank: rp_create then creates the communicator (collective: every rank must call it) and
+ * rp_destroy frees it.  world = 1 is allowed (a one-rank communicator). */
+#define RP_NCCL_ID_BYTES 128
+typedef struct {
+  int32_t rank, world;
+  void* nccl_comm;
+  unsigned char nccl_id[RP_NCCL_ID_BYTES];
+} rp_dist;
+
+/* Fill id_out with a fresh ncclUniqueId (call on one rank, broadcast the bytes).
+ * ENCCL when NCCL cannot be loaded. */
+int rp_nccl_unique_id(unsigned char id_out[RP_NCCL_ID_BYTES]);
 
 /* Create a context on cfg->device: allocates the HBM history ring of history_depth+2
  * FP64 moment grids [slot][ny+6][nx+6][4] (zero-padded by 3 nodes) and scratch.
- * EINVAL on an invalid config, ENODEV / ENOMEM / ECUDA on device failures. */
-int rp_create(const rp_config* cfg, rp_ctx** out);
+ * dist = NULL: single GPU.  dist != NULL: this process is rank dist->rank of dist->world
+ * (see rp_dist); the NCCL communicator is created here when dist->nccl_comm is NULL.
+ * EINVAL on an invalid config, ENODEV / ENOMEM / ECUDA on device failures, ENCCL when the
+ * communicator cannot be created.  The caller's current device is left unchanged. */
+int rp_create(const rp_config* cfg, const rp_dist* dist, rp_ctx** out);
+
+/* Subtree work units: in the near-field subregion S_0 a segment at level
+ * level-1 that splits hands its two children to a second, persistent launch instead of
+ * descending (at most 64 per item, in DFS order), so one deep tree does not bound the step
+ * on one warp.  The tree, every decision and the counts are unchanged; only the summation
+ * groups the subtrees (results within rounding, bit-identical across ranks).  level = 0
+ * turns it off; default 12.  EINVAL unless level == 0 or 2 <= level <= max_depth. */
+int rp_set_work_split(rp_ctx* ctx, int32_t level);
 
 /* Destroy a context (NULL is ignored).  Synchronises its stream first. */
 void rp_destroy(rp_ctx* ctx);
@@ -146,12 +179,21 @@ int rp_deposit(rp_ctx* ctx, const double* x, const double* y, const double* ux,
 int rp_history_append(rp_ctx* ctx, const void* partials_dev, int32_t n_parts,
                       const rp_frame* frame_k);
 
-/* rp_deposit into context scratch + rp_history_append(n_parts = 1). */
+/* rp_deposit of this rank's particles into context scratch, then rp_history_append of the
+ * partials of all ranks: with an rp_dist the partial buffers are all-gathered over NCCL on the
+ * context's stream first (rank order), so D_k is identical on every rank and bit-identical to
+ * a single-GPU deposit of all particles.  info (nullable, syncs) counts this rank's particles. */
 int rp_deposit_step(rp_ctx* ctx, const double* x, const double* y, const double* ux,
                     const double* uy, double q, int64_t n, const rp_frame* frame_k,
                     rp_deposit_info* info);
 
 /* Retarded potentials at all nx*ny nodes of the current frame (Eq. 1-2, Alg. 1).
+ * With an rp_dist of world > 1 this rank integrates its share of the mesh points (dealt
+ * longest-predicted-first over ranks from the previous step's counts, identical on every
+ * rank) and the shards are all-gathered over NCCL, so the outputs cover the full mesh on
+ * every rank; info then counts this rank's work only.  Enqueue-only: the call returns without
+ * waiting for the device unless info is given (the work is capturable in a CUDA graph after
+ * one warm-up call has sized the scratch).
  * For every (point p, subregion j < kappa(k)): support clip [A, B] of S_j (R-5), then a
  * deterministic top-down dyadic GK15 tree from the n_root halves of [A, B]: accept a
  * segment iff max_c |K15_c - G7_c| <= tau (b - a) / R(p), R(p) = kappa(k) c dt, or at
@@ -197,7 +239,8 @@ int rp_push_particles(rp_ctx* ctx, double* x, double* y, double* ux, double* uy,
                       double q_over_mc, double bz_ext, const double* ex, const double* ey,
                       const double* bz);
 
-/* One whole step through HOST buffers (end-to-end path): copies the particles
+/* One whole step through HOST buffers (end-to-end path).  With an rp_dist the host arrays
+ * hold this rank's particle shard and the mesh outputs are the full mesh.  Copies the particles
  * host->device, runs deposit_step, compute_potentials, compute_fields (with the previous
  * step's A kept by the context), push, and copies the pushed particles and the six mesh
  * outputs back.  x_host .. uy_host are updated in place; mesh_host is [6][ny*nx]
@@ -229,6 +272,13 @@ int rp_debug_bins(rp_ctx* ctx, int32_t* bins_dev, int64_t n);
  * The arithmetic mirrors the oracle's operation order with IEEE round-to-nearest intrinsics,
  * so the limits are bit-identical to it.  RP_ESTATE before the first potentials call. */
 int rp_debug_clip(rp_ctx* ctx, double* ab_dev, int64_t n);
+
+/* Per-point (nleaf, capped) of the last rp_compute_potentials call (the 7-tuple of P:110
+ * beside phi, A, err and nseg): accepted segments and the leaves accepted
+ * at max_depth with err > tol, summed over the point's subregions; int32 DEVICE arrays of
+ * n = nx*ny entries (either may be NULL).  Points not owned by the last shard call keep
+ * stale values.  EINVAL on a wrong n, ESTATE before the first potentials call. */
+int rp_debug_point_counts(rp_ctx* ctx, int32_t* nleaf_dev, int32_t* capped_dev, int64_t n);
 
 /* Test hook: potentials with an analytic source in place of the grid:
  * kind = RP_SRC_GAUSS (centre (x0,y0) frame-local, width = sigma, q = Q) or RP_SRC_DISK
@@ -271,7 +321,8 @@ int rp_set_schedule(rp_ctx* ctx, int32_t policy, int32_t k);
  * of an adaptive dyadic tree that refines it where the estimate misses the tolerance
  * (lines 18-24).  Results differ from the canonical tree within tau and depend on the
  * forecast.  A step without a previous pattern uses the canonical tree.
- * Single-call path only: rp_compute_potentials_shard returns RP_EINVAL while enabled.
+ * Single-GPU path only: rp_compute_potentials_shard, and rp_compute_potentials on a context
+ * with world > 1, return RP_EINVAL while enabled.
  * enable = 0 restores the canonical tree.  Returns RP_EINVAL on a bad k or n_clusters < 0. */
 int rp_set_predictive(rp_ctx* ctx, int32_t enable, int32_t knn, int32_t n_clusters,
                       int32_t max_iters);
@@ -302,6 +353,8 @@ typedef struct {
   double push_ms;
   int64_t integrate_launches;  /* integrator calls (each: the item launch, then the units')  */
   double units_ms;         /* of integrate_ms: the subtree-unit launch, its sort and merge      */
+  double step_ms;          /* rp_step_host: its device part, deposit through push (the copies
+                              before and after it excluded)                                     */
 } rp_profile;
 
 /* enable != 0 starts (and resets) event timing; 0 stops it.  Adds two event records per

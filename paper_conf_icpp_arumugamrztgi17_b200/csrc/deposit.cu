@@ -128,15 +128,24 @@ __global__ void k_append(int nx, int ny, int PX, const unsigned char* __restrict
   if (id >= nx * ny) return;
   int ix = id % nx, iy = id / nx;
   __int128 a = 0, b = 0, c = 0;
-  const int shift = (int)reinterpret_cast<const long long*>(parts)[0];
+  // common quantum: the coarsest of the parts (smallest shift), so no part is shifted left
+  // (which could overflow); equal shifts -- the same q on every rank -- keep the sum exact,
+  // a finer part is rounded to the common quantum (half up), in part order: deterministic
+  int shift = 1 << 30;
+  for (int i = 0; i < n_parts; ++i)
+    shift = min(shift, (int)reinterpret_cast<const long long*>(parts + i * part_bytes)[0]);
   for (int i = 0; i < n_parts; ++i) {
     const unsigned char* base = parts + i * part_bytes;
-    const int sh = (int)reinterpret_cast<const long long*>(base)[0];
+    const int d = (int)reinterpret_cast<const long long*>(base)[0] - shift;  // >= 0
     const __int128* m = reinterpret_cast<const __int128*>(base + 16) + 3 * (size_t)id;
-    const int d = sh - shift;  // equal shifts in practice (same q on every rank)
-    a += d >= 0 ? (m[0] >> d) : (m[0] << -d);
-    b += d >= 0 ? (m[1] >> d) : (m[1] << -d);
-    c += d >= 0 ? (m[2] >> d) : (m[2] << -d);
+    if (d == 0) {
+      a += m[0]; b += m[1]; c += m[2];
+    } else if (d < 126) {  // |part| < 2^126: a shift by >= 126 rounds it to 0
+      const __int128 half = (__int128)1 << (d - 1);
+      a += (m[0] + half) >> d;
+      b += (m[1] + half) >> d;
+      c += (m[2] + half) >> d;
+    }
   }
   double* dst = slot + 4 * ((size_t)(iy + RP_PAD) * PX + (ix + RP_PAD));
   dst[0] = ldexp((double)a, -shift);
@@ -165,6 +174,9 @@ __global__ void k_rigid_copy(const double* __restrict__ src, double* __restrict_
     reinterpret_cast<double4*>(dst)[i] = o;
   }
 }
+
+// frame upload as a kernel parameter: stream-ordered and capturable (no host pointer kept)
+__global__ void k_set_frame(rp_frame* dst, rp_frame f) { *dst = f; }
 
 __global__ void k_set_header(long long* hdr, long long shift) {
   hdr[0] = shift;
@@ -282,7 +294,8 @@ int rp_append_impl(rp_ctx* ctx, const void* parts, int32_t n_parts, const rp_fra
                                                 (size_t)rp_partial_bytes_impl(ctx), n_parts, slot);
   RP_CHECK_LAUNCH();
   ctx->fh[s] = *fk;
-  RP_CUDA(cudaMemcpyAsync(ctx->frames_dev + s, fk, sizeof(rp_frame), cudaMemcpyHostToDevice, st));
+  k_set_frame<<<1, 1, 0, st>>>(ctx->frames_dev + s, *fk);
+  RP_CHECK_LAUNCH();
   if (knew == 0 && ctx->rigid_pending) {
     const size_t nodes = ctx->slot_doubles / 4;
     for (int l = -ctx->n_pre; l < 0; ++l) {
@@ -295,7 +308,5 @@ int rp_append_impl(rp_ctx* ctx, const void* parts, int32_t n_parts, const rp_fra
     ctx->rigid_pending = 0;
   }
   ctx->k = knew;
-  // frames are read by later kernels from frames_dev; the host copy is pageable, so the
-  // H2D copy above is synchronous w.r.t. the host buffer (safe to reuse fk).
   return RP_OK;
 }

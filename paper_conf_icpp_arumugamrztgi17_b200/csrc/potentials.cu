@@ -44,8 +44,9 @@ __constant__ double c_wg[4] = {
 
 enum : int { C_ITEMS = 0, C_NEXT = 1, C_EVALS = 2, C_SEGS = 3, C_LEAVES = 4, C_CAPPED = 5,
              C_TIES = 6, C_MAXLEV = 7, C_NODES = 8, C_NOUT = 9, C_SKIP = 10, C_UNITS = 11,
-             C_NEXT_U = 12, C_UOVF = 13, C_COUNT = 16 };
+             C_NEXT_U = 12, C_COUNT = 16 };
 constexpr int kUnitShift = 20;  // unit key = item << 20 | index of the subtree root at its level
+constexpr int kUnitBudget = 64;  // subtree units per near-field item (DFS order)
 constexpr uint32_t kEmptyKey = 0xFFFFFFFFu;  // schedule key of an item without support
 
 constexpr double kTwoPi = 6.283185307179586476925286766559;
@@ -69,8 +70,8 @@ struct Params {
   int split_level;                  // 0: off
   int split_j;                      // only subregions j < split_j are split (the near field)
   int unit_budget;                  // at most this many units per item (the first in DFS order)
-  long long unit_cap;
-  unsigned long long* unit_key;     // [unit_cap] item << kUnitShift | ix
+  int32_t* unit_ndef;               // [npts * split_j] units deferred by each near-field item
+  unsigned long long* unit_key;     // [slots] item << kUnitShift | ix, item-major fixed slots
   const int32_t* unit_order;        // unit launch: the units, longest-predicted-first
   double4* unit_val;
   int4* unit_cnt;
@@ -276,50 +277,11 @@ __global__ void k_clip(Params P, const int32_t* __restrict__ owner, int rank,
     atomicAdd(&counters[C_ITEMS], (unsigned long long)__popc(m));
 }
 
-// ------------------------------------------------------------- integrand
+// ------------------------------------------------------------- integrand (analytic sources)
 template <int KIND>
 __device__ __forceinline__ void integrand(const Item& it, const Params& P, double u, double v,
                                           double w0, double w1, double w2, double& f0,
                                           double& f1, double& f2) {
-  if (KIND == RP_SRC_GRID) {
-    double tx = u * P.inv_hx, ty = v * P.inv_hy;
-    double fx = floor(tx + 0.5), fy = floor(ty + 0.5);
-    double dx = tx - fx, dy = ty - fy;
-    double ax = 0.5 - dx, bx = 0.5 + dx, ay = 0.5 - dy, by = 0.5 + dy;
-    double wx0 = 0.5 * ax * ax, wx1 = 0.75 - dx * dx, wx2 = 0.5 * bx * bx;
-    double wy0 = 0.5 * ay * ay, wy1 = 0.75 - dy * dy, wy2 = 0.5 * by * by;
-    // clamp keeps every stencil inside the zero border (points outside the support
-    // rectangle never reach here; the clamp only guards memory)
-    int ix = (int)fmin(fmax(fx, -2.0), (double)(P.nx + 1));
-    int iy = (int)fmin(fmax(fy, -2.0), (double)(P.ny + 1));
-    size_t base = (size_t)4 * ((iy - 1) * P.PX + (ix - 1));
-    double s[3][3];
-#pragma unroll
-    for (int l = 0; l < 3; ++l) { s[l][0] = 0.0; s[l][1] = 0.0; s[l][2] = 0.0; }
-    const double wxa[3] = {wx0, wx1, wx2};
-    const double wyb[3] = {wy0, wy1, wy2};
-#pragma unroll
-    for (int b = 0; b < 3; ++b) {
-#pragma unroll
-      for (int a = 0; a < 3; ++a) {
-        double w = wxa[a] * wyb[b];
-        size_t o = base + (size_t)4 * (b * P.PX + a);
-        double2 m0 = __ldg(reinterpret_cast<const double2*>(it.g0 + o));
-        double z0 = __ldg(it.g0 + o + 2);
-        double2 m1 = __ldg(reinterpret_cast<const double2*>(it.g1 + o));
-        double z1 = __ldg(it.g1 + o + 2);
-        double2 m2 = __ldg(reinterpret_cast<const double2*>(it.g2 + o));
-        double z2 = __ldg(it.g2 + o + 2);
-        s[0][0] += w * m0.x; s[0][1] += w * m0.y; s[0][2] += w * z0;
-        s[1][0] += w * m1.x; s[1][1] += w * m1.y; s[1][2] += w * z1;
-        s[2][0] += w * m2.x; s[2][1] += w * m2.y; s[2][2] += w * z2;
-      }
-    }
-    f0 = w0 * s[0][0] + w1 * s[1][0] + w2 * s[2][0];
-    f1 = w0 * s[0][1] + w1 * s[1][1] + w2 * s[2][1];
-    f2 = w0 * s[0][2] + w1 * s[1][2] + w2 * s[2][2];
-    return;
-  }
   double amp = w0 * it.a0 + w1 * it.a1 + w2 * it.a2;
   double rho;
   if (KIND == RP_SRC_GAUSS) {
@@ -477,24 +439,21 @@ __device__ __forceinline__ void ldg_node(const double* p, double& a, double& b, 
   asm("ld.global.nc.v4.f64 {%0,%1,%2,%3}, [%4];" : "=d"(a), "=d"(b), "=d"(c), "=d"(d) : "l"(p));
 }
 
-// Theta slot e of the r' nodes n0 .. n1-1 of the current segment.  The 27-node x 3-component
-// stencil cache (st, cix, ciy) belongs to the caller, so it survives across calls: a lane that
-// evaluates the same slot in consecutive (radially adjacent) deep segments keeps its cell.
-template <int KIND, bool CACHE = true>
+// Analytic sources (test path): theta slot e of the r' nodes n0 .. n1-1 of the
+// current segment, evaluated in closed form (no stencil).
+template <int KIND>
 __device__ __forceinline__ void eval_nodes(const Item& it, const Params& P, const WarpSmem& S,
                                            const double2* __restrict__ trig_full, int e, int n0,
                                            int n1, int N, double wfull, double third,
-                                           double (&st)[3][9][3], int& cix, int& ciy, double& k0,
-                                           double& k1, double& k2, double& g0, double& g1,
-                                           double& g2) {
-  const size_t rs = (size_t)4 * P.PX;  // padded row stride in doubles
+                                           double& k0, double& k1, double& k2, double& g0,
+                                           double& g1, double& g2) {
   // the full-circle node of slot e is the same for every r' node: one load per call
   const double2 trf = __ldg(trig_full + (e < N ? e : 0));
 #pragma unroll 3
   for (int n = n0; n < n1; ++n) {
     if (e >= S.cnt[n]) continue;
     const int na = S.na[n];
-    const NodeRec& nd = S.node[n];  // read at the point of use (register pressure)
+    const NodeRec& nd = S.node[n];
     double cs, sn, w;
     if (na < 0) {
       cs = trf.x;
@@ -513,84 +472,11 @@ __device__ __forceinline__ void eval_nodes(const Item& it, const Params& P, cons
     }
     const double u = nd.cu + nd.r * cs, v = nd.cv + nd.r * sn;
     double f0, f1, f2;
-    if (KIND == RP_SRC_GRID) {
-      const double tx = u * P.inv_hx, ty = v * P.inv_hy;
-      const double fx = floor(tx + 0.5), fy = floor(ty + 0.5);
-      const double dx = tx - fx, dy = ty - fy;
-      const double ax = 0.5 - dx, bx = 0.5 + dx, ay = 0.5 - dy, by = 0.5 + dy;
-      // 2 x TSC weights (the factor 1/4 of the products is folded into the node weight)
-      const double wx[3] = {ax * ax, fma(-2.0 * dx, dx, 1.5), bx * bx};
-      const double wy[3] = {ay * ay, fma(-2.0 * dy, dy, 1.5), by * by};
-      // clamp keeps every stencil inside the zero border (memory guard only)
-      const int ix = min(max(__double2int_rz(fx), -2), P.nx + 1);
-      const int iy = min(max(__double2int_rz(fy), -2), P.ny + 1);
-      double s[3][3];
-      if (CACHE) {
-      if (ix != cix || iy != ciy) {
-        cix = ix;
-        ciy = iy;
-        const size_t base = (size_t)4 * ((iy - 1) * P.PX + (ix - 1));
-        const double* g[3] = {it.g0 + base, it.g1 + base, it.g2 + base};
-#pragma unroll
-        for (int l = 0; l < 3; ++l)
-#pragma unroll
-          for (int b = 0; b < 3; ++b) {
-            const double* row = g[l] + b * rs;
-#pragma unroll
-            for (int a = 0; a < 3; ++a)
-              ldg_node(row + 4 * a, st[l][3 * b + a][0], st[l][3 * b + a][1], st[l][3 * b + a][2]);
-          }
-      }
-      // 9 independent chains (level x component) advanced node by node: covers the DFMA
-      // latency at 2 warps per scheduler
-      {
-        const double w00 = wx[0] * wy[0];
-#pragma unroll
-        for (int l = 0; l < 3; ++l)
-#pragma unroll
-          for (int c = 0; c < 3; ++c) s[l][c] = w00 * st[l][0][c];
-#pragma unroll
-        for (int i = 1; i < 9; ++i) {
-          const double ww = wx[i % 3] * wy[i / 3];
-#pragma unroll
-          for (int l = 0; l < 3; ++l)
-#pragma unroll
-            for (int c = 0; c < 3; ++c) s[l][c] = fma(ww, st[l][i][c], s[l][c]);
-        }
-      }
-      } else {
-        // leftover slots: stream the stencil node by node (no cache; the lane's cache is
-        // kept for the next segment)
-        const size_t base = (size_t)4 * ((iy - 1) * P.PX + (ix - 1));
-        const double* g[3] = {it.g0 + base, it.g1 + base, it.g2 + base};
-#pragma unroll
-        for (int l = 0; l < 3; ++l) s[l][0] = s[l][1] = s[l][2] = 0.0;
-#pragma unroll
-        for (int b = 0; b < 3; ++b)
-#pragma unroll
-          for (int a = 0; a < 3; ++a) {
-            const double ww = wx[a] * wy[b];
-#pragma unroll
-            for (int l = 0; l < 3; ++l) {
-              double m0, m1, m2;
-              ldg_node(g[l] + b * rs + 4 * a, m0, m1, m2);
-              s[l][0] = fma(ww, m0, s[l][0]);
-              s[l][1] = fma(ww, m1, s[l][1]);
-              s[l][2] = fma(ww, m2, s[l][2]);
-            }
-          }
-      }
-      f0 = nd.w0 * s[0][0] + nd.w1 * s[1][0] + nd.w2 * s[2][0];
-      f1 = nd.w0 * s[0][1] + nd.w1 * s[1][1] + nd.w2 * s[2][1];
-      f2 = nd.w0 * s[0][2] + nd.w1 * s[1][2] + nd.w2 * s[2][2];
-    } else {
-      integrand<KIND>(it, P, u, v, nd.w0, nd.w1, nd.w2, f0, f1, f2);
-    }
-    const double ws = KIND == RP_SRC_GRID ? 0.25 * w : w;  // undo the 2 x 2 weight scaling
-    const double wk = ws * nd.wk;
+    integrand<KIND>(it, P, u, v, nd.w0, nd.w1, nd.w2, f0, f1, f2);
+    const double wk = w * nd.wk;
     k0 += wk * f0; k1 += wk * f1; k2 += wk * f2;
     if ((n & 1) || P.rule == RP_RULE_SIMPSON) {  // G7: Gauss nodes only (warp-uniform n)
-      const double wg = ws * nd.wg;
+      const double wg = w * nd.wg;
       g0 += wg * f0; g1 += wg * f1; g2 += wg * f2;
     }
   }
@@ -739,13 +625,13 @@ __device__ __forceinline__ double warp_sum(double v) {
   return v;
 }
 
-__device__ unsigned long long g_phase[8];  // development: per-phase SM cycles (VAR 7)
-
-// VAR 0: one pass per round (eval_nodes); VAR 4: software-pipelined rounds; VAR 7: VAR 4 with
-// per-phase clock accounting (development)
+// VAR 0: analytic sources (eval_nodes); VAR 4: grid, TSC, software-pipelined rounds with the
+// register stencil cache; VAR 6: the same with the Lagrange-3 spatial weights (R-25).
 // UNIT = false: the (point, subregion) items in forecast order.  With P.split_level = L > 0
-// a segment at level L - 1 that splits does not descend: its two children become subtree work
-// units (appended to P.unit_key) and the walk goes on as if the segment were finished.  The
+// a segment at level L - 1 of a near-field item (j < split_j) that splits does not descend:
+// its two children become subtree work units -- written to the item's own fixed slots
+// (item-major, at most unit_budget per item, in DFS order) -- and the walk goes on as if the
+// segment were finished.  The
 // tree is the canonical one -- only nodes it reaches are deferred -- but the deep near-field
 // trees (thousands of segments, fanning out below level ~8) no longer bound the kernel (and an
 // N-GPU shard) by one warp's walk.  UNIT = true: the units, each walked from its root at
@@ -766,9 +652,6 @@ __global__ void __launch_bounds__(32 * kWarps) k_integrate(
   const double Nd = (double)N;
   const double wfull = kTwoPi / Nd;
   const double third = 1.0 / 3.0;
-  constexpr bool TM = VAR == 7;
-  unsigned long long ph[6] = {0, 0, 0, 0, 0, 0};
-  long long t0 = TM ? clock64() : 0;
   for (;;) {
     unsigned long long idx = 0;
     if (lane == 0) idx = atomicAdd(&counters[UNIT ? C_NEXT_U : C_NEXT], 1ULL);
@@ -813,7 +696,6 @@ __global__ void __launch_bounds__(32 * kWarps) k_integrate(
 
     double s_phi = 0.0, s_ax = 0.0, s_ay = 0.0, s_err = 0.0;
     double st[3][9][3];                      // per-lane stencil cache (valid for this item's levels)
-    int cix = -1000000, ciy = -1000000;
     int ccell = kNoCell;  // cached cell of the two-pass rounds (empty cache reads as zeros)
     if (KIND == RP_SRC_GRID && VAR >= 4) {
 #pragma unroll
@@ -825,7 +707,6 @@ __global__ void __launch_bounds__(32 * kWarps) k_integrate(
     unsigned evals = 0, nskip = 0;
     int lev = UNIT ? P.split_level : ((P.n_root == 2 && !pred) ? 1 : 0);
     const int rlev = UNIT ? P.split_level : 0;  // the walk ends when it climbs back here
-    if (TM) { long long t = clock64(); ph[0] += t - t0; t0 = t; }
     long long ix = UNIT ? (long long)(ukey & ((1ULL << kUnitShift) - 1)) : 0;
     for (;;) {
       const double fa = ldexp((double)ix, -lev), fb = ldexp((double)(ix + 1), -lev);
@@ -867,7 +748,6 @@ __global__ void __launch_bounds__(32 * kWarps) k_integrate(
           cnt = na * (N - 1);
         }
       }
-      if (TM) { __syncwarp(); long long t = clock64(); ph[1] += t - t0; t0 = t; }
       // integrand nodes of the rules over the 15 r' nodes (E, including the skipped arc end
       // nodes) and the largest per-node slot count (rounds): two independent butterflies
       if (lane < 16) S.cnt[lane] = lane < 15 ? cnt : 0;
@@ -891,7 +771,6 @@ __global__ void __launch_bounds__(32 * kWarps) k_integrate(
       // 65-node arcs as (slot, node) units.
       const int rounds = (KIND == RP_SRC_GRID && VAR >= 4) ? (emax + 31) >> 5 : emax >> 5;
       const int left = (KIND == RP_SRC_GRID && VAR >= 4) ? 0 : emax - 32 * rounds;
-      if (TM) { long long t = clock64(); ph[2] += t - t0; t0 = t; }
       if (KIND == RP_SRC_GRID && VAR >= 4) {
         for (int rr = 0; rr < rounds; ++rr) {
           const int r = (nseg & 1) ? rounds - 1 - rr : rr;
@@ -902,17 +781,15 @@ __global__ void __launch_bounds__(32 * kWarps) k_integrate(
       } else {
         for (int rr = 0; rr < rounds; ++rr) {
           const int r = (nseg & 1) ? rounds - 1 - rr : rr;
-          eval_nodes<KIND>(it, P, S, trig_full, 32 * r + lane, 0, nn, N, wfull, third, st, cix,
-                           ciy, k0, k1, k2, g0, g1, g2);
+          eval_nodes<KIND>(it, P, S, trig_full, 32 * r + lane, 0, nn, N, wfull, third, k0, k1,
+                           k2, g0, g1, g2);
         }
       }
-      if (TM) { __syncwarp(); long long t = clock64(); ph[3] += t - t0; t0 = t; }
       for (int u = lane; u < nn * left; u += 32) {
         const int e = 32 * rounds + u / nn, n = u - nn * (u / nn);
-        eval_nodes<KIND, false>(it, P, S, trig_full, e, n, n + 1, N, wfull, third, st, cix, ciy,
-                                k0, k1, k2, g0, g1, g2);
+        eval_nodes<KIND>(it, P, S, trig_full, e, n, n + 1, N, wfull, third, k0, k1, k2, g0, g1,
+                         g2);
       }
-      if (TM) { __syncwarp(); long long t = clock64(); ph[4] += t - t0; t0 = t; }
       k0 = warp_sum(k0); k1 = warp_sum(k1); k2 = warp_sum(k2);
       g0 = warp_sum(g0); g1 = warp_sum(g1); g2 = warp_sum(g2);
       __syncwarp();
@@ -933,22 +810,16 @@ __global__ void __launch_bounds__(32 * kWarps) k_integrate(
         finished = true;
       } else if (!UNIT && P.split_level > 0 && lev + 1 == P.split_level && j < P.split_j &&
                  ndef < P.unit_budget) {
-        ndef += 2;  // per-item budget, counted in DFS order: deterministic
-        // defer both children as subtree units (falls back to descending if the unit list is
-        // full, flagged in counters[C_UOVF])
-        unsigned long long u = 0;
-        if (lane == 0) u = atomicAdd(&counters[C_UNITS], 2ULL);
-        u = __shfl_sync(0xffffffffu, u, 0);
-        if ((long long)u + 1 < P.unit_cap) {
-          if (lane == 0) {
-            const unsigned long long base = (unsigned long long)item << kUnitShift;
-            P.unit_key[u] = base | (unsigned long long)(2 * ix);
-            P.unit_key[u + 1] = base | (unsigned long long)(2 * ix + 1);
-          }
-          finished = true;
-        } else if (lane == 0) {
-          atomicExch(&counters[C_UOVF], 1ULL);
+        // defer both children as subtree units into the item's own slots, in DFS order (the
+        // per-item budget is counted in that order: deterministic, and never full)
+        if (lane == 0) {
+          const unsigned long long base = (unsigned long long)item << kUnitShift;
+          const size_t slot = ((size_t)p * P.split_j + j) * P.unit_budget + ndef;
+          P.unit_key[slot] = base | (unsigned long long)(2 * ix);
+          P.unit_key[slot + 1] = base | (unsigned long long)(2 * ix + 1);
         }
+        ndef += 2;
+        finished = true;
       }
       if (finished) {
         while ((ix & 1) && lev > rlev) { ix >>= 1; --lev; }
@@ -969,7 +840,6 @@ __global__ void __launch_bounds__(32 * kWarps) k_integrate(
         ++lev;
         ix <<= 1;
       }
-      if (TM) { long long t = clock64(); ph[5] += t - t0; t0 = t; }
     }
     if (lane == 0) {
       const size_t o = UNIT ? (size_t)uidx : (size_t)item;
@@ -977,10 +847,12 @@ __global__ void __launch_bounds__(32 * kWarps) k_integrate(
       (UNIT ? P.unit_cnt : item_cnt)[o] = make_int4(nseg, nleaf, capped, ties);
       (UNIT ? P.unit_aux : item_aux)[o] = make_uint2((unsigned)maxlev, evals);
       if (nskip) atomicAdd(&counters[C_SKIP], (unsigned long long)nskip);
+      if (!UNIT && P.split_level > 0 && j < P.split_j) {
+        P.unit_ndef[(size_t)p * P.split_j + j] = ndef;
+        if (ndef) atomicAdd(&counters[C_UNITS], (unsigned long long)ndef);
+      }
     }
   }
-  if (TM && lane == 0)
-    for (int i = 0; i < 6; ++i) atomicAdd(&g_phase[i], ph[i]);
 }
 
 // ------------------------------------------------------------- subtree units
@@ -989,33 +861,41 @@ __global__ void k_iota(int32_t* a, long long n) {
   if (i < n) a[i] = (int32_t)i;
 }
 
-// Launch order of the units: their item's segment count of the previous step (the forecast),
-// largest first (ties by unit index), so the longest units do not start last.
-__global__ void k_unit_order_keys(long long n, const unsigned long long* __restrict__ key,
+// Launch order of the units over all fixed slots (nslots = near-field items x unit_budget):
+// a used slot gets its item's segment count of the previous step (the forecast), largest
+// first (ties by slot); unused slots sort last.  The unit launch takes the first
+// counters[C_UNITS] entries, so nothing is sized on the host.
+__global__ void k_unit_order_keys(long long nslots, int budget, const int32_t* __restrict__ ndef,
+                                  const unsigned long long* __restrict__ key,
                                   const uint16_t* __restrict__ cost,
                                   unsigned long long* __restrict__ okey) {
-  const long long u = blockIdx.x * (long long)blockDim.x + threadIdx.x;
-  if (u >= n) return;
-  const unsigned long long item = key[u] >> kUnitShift;
-  okey[u] = ((unsigned long long)(0xFFFFu - cost[item]) << 32) | (unsigned long long)u;
+  const long long s = blockIdx.x * (long long)blockDim.x + threadIdx.x;
+  if (s >= nslots) return;
+  if ((int)(s % budget) >= ndef[s / budget]) {
+    okey[s] = ~0ULL;
+    return;
+  }
+  const unsigned long long item = key[s] >> kUnitShift;
+  okey[s] = ((unsigned long long)(0xFFFFu - cost[item]) << 32) | (unsigned long long)s;
 }
 
-// Add every item's units to its own partial result, in (item, subtree index) order: one
-// thread per item (the first sorted position of its run), so the sums are deterministic.
-__global__ void k_merge_units(long long n, const unsigned long long* __restrict__ skey,
-                              const int32_t* __restrict__ perm, const double4* __restrict__ uv,
+// Add every near-field item's units to its own partial result, in slot (= DFS, = subtree
+// index) order: one thread per item, so the sums are deterministic for any launch order.
+__global__ void k_merge_units(int n_nf, int split_j, int kmax, int budget,
+                              const int32_t* __restrict__ ndef, const double4* __restrict__ uv,
                               const int4* __restrict__ uc, const uint2* __restrict__ ua,
                               double4* __restrict__ item_val, int4* __restrict__ item_cnt,
                               uint2* __restrict__ item_aux) {
-  const long long i = blockIdx.x * (long long)blockDim.x + threadIdx.x;
-  if (i >= n) return;
-  const unsigned long long it = skey[i] >> kUnitShift;
-  if (i > 0 && (skey[i - 1] >> kUnitShift) == it) return;
+  const int f = blockIdx.x * blockDim.x + threadIdx.x;
+  if (f >= n_nf) return;
+  const int nd = ndef[f];
+  if (nd == 0) return;
+  const size_t it = (size_t)(f / split_j) * kmax + (f % split_j);
   double4 v = item_val[it];
   int4 c = item_cnt[it];
   uint2 a = item_aux[it];
-  for (long long k = i; k < n && (skey[k] >> kUnitShift) == it; ++k) {
-    const int u = perm[k];
+  for (int k = 0; k < nd; ++k) {
+    const size_t u = (size_t)f * budget + k;
     const double4 w = uv[u];
     const int4 d = uc[u];
     const uint2 b = ua[u];
@@ -1038,7 +918,7 @@ __global__ void k_reduce(int npts, int kmax, int kap, const uint32_t* __restrict
                          double* __restrict__ ay, double* __restrict__ err,
                          int32_t* __restrict__ nseg, double* __restrict__ shard,
                          uint16_t* __restrict__ cost, int32_t* __restrict__ nseg_pt,
-                         uint16_t* __restrict__ leaves,
+                         uint16_t* __restrict__ leaves, int2* __restrict__ point_cnt,
                          unsigned long long* __restrict__ counters) {
   int p = blockIdx.x * blockDim.x + threadIdx.x;
   if (p >= npts) return;
@@ -1063,6 +943,7 @@ __global__ void k_reduce(int npts, int kmax, int kap, const uint32_t* __restrict
     cost[id] = (uint16_t)(q.x < 0xFFFE ? q.x : 0xFFFE);
     leaves[id] = (uint16_t)(q.y < 0xFFFF ? q.y : 0xFFFF);  // observed access pattern n_j(p)
   }
+  point_cnt[p] = make_int2((int)nl, (int)cp);  // per-point leaves / capped (rp_debug_point_counts)
   if (shard) {
     double* r = shard + 6 * (size_t)row_of[p];
     r[0] = (double)p; r[1] = a; r[2] = b; r[3] = c; r[4] = e; r[5] = (double)ns;
@@ -1139,25 +1020,22 @@ int rp_alloc_potential_scratch(rp_ctx* ctx) {
   RP_CUDA(cudaMalloc(&ctx->leaves_prev, nd * sizeof(uint16_t)));
   RP_CUDA(cudaMemset(ctx->leaves_prev, 0, nd * sizeof(uint16_t)));
   RP_CUDA(cudaMalloc(&ctx->cluster_dev, npts * sizeof(int32_t)));
-  if (ctx->split_level > 0) {
-    // a unit list of up to 512 units per mesh point (config 4 needs ~130-300; 80 bytes each),
-    // at most 5 % of the device memory; a full list is exact (subtrees walked in place) and
-    // reported in rp_potential_info.unit_overflow
-    size_t fr = 0, tot = 0;
-    cudaMemGetInfo(&fr, &tot);
-    const long long budget = (long long)(0.05 * (double)tot / 88.0);
-    const long long cap =
-        std::max<long long>(1LL << 22, std::min<long long>(512LL * (long long)npts, budget)) & ~1LL;
-    ctx->unit_cap = cap;
-    RP_CUDA(cudaMalloc(&ctx->unit_key, cap * sizeof(unsigned long long)));
-    RP_CUDA(cudaMalloc(&ctx->unit_key_sorted, cap * sizeof(unsigned long long)));
-    RP_CUDA(cudaMalloc(&ctx->unit_okey, cap * sizeof(unsigned long long)));
-    RP_CUDA(cudaMalloc(&ctx->unit_iota, cap * sizeof(int32_t)));
-    RP_CUDA(cudaMalloc(&ctx->unit_perm, cap * sizeof(int32_t)));
-    RP_CUDA(cudaMalloc(&ctx->unit_val, cap * sizeof(double4)));
-    RP_CUDA(cudaMalloc(&ctx->unit_cnt, cap * sizeof(int4)));
-    RP_CUDA(cudaMalloc(&ctx->unit_aux, cap * sizeof(uint2)));
-    k_iota<<<(unsigned)((cap + 255) / 256), 256>>>(ctx->unit_iota, cap);
+  {
+    // subtree work units: fixed slots, unit_budget per near-field item (item-major), so the
+    // unit launch, its order sort and the merge are sized without a host round trip
+    const long long nf = (long long)npts * ctx->split_j, slots = nf * kUnitBudget;
+    ctx->unit_slots = slots;
+    RP_CUDA(cudaMalloc(&ctx->unit_ndef, nf * sizeof(int32_t)));
+    RP_CUDA(cudaMemset(ctx->unit_ndef, 0, nf * sizeof(int32_t)));
+    RP_CUDA(cudaMalloc(&ctx->unit_key, slots * sizeof(unsigned long long)));
+    RP_CUDA(cudaMalloc(&ctx->unit_okey, slots * sizeof(unsigned long long)));
+    RP_CUDA(cudaMalloc(&ctx->unit_okey_sorted, slots * sizeof(unsigned long long)));
+    RP_CUDA(cudaMalloc(&ctx->unit_iota, slots * sizeof(int32_t)));
+    RP_CUDA(cudaMalloc(&ctx->unit_perm, slots * sizeof(int32_t)));
+    RP_CUDA(cudaMalloc(&ctx->unit_val, slots * sizeof(double4)));
+    RP_CUDA(cudaMalloc(&ctx->unit_cnt, slots * sizeof(int4)));
+    RP_CUDA(cudaMalloc(&ctx->unit_aux, slots * sizeof(uint2)));
+    k_iota<<<(unsigned)((slots + 255) / 256), 256>>>(ctx->unit_iota, slots);
     RP_CUDA(cudaGetLastError());
   }
   RP_CUDA(cudaMemset(ctx->cost_prev, 0, nd * sizeof(uint16_t)));
@@ -1172,6 +1050,8 @@ int rp_alloc_potential_scratch(rp_ctx* ctx) {
   RP_CUDA(cudaMalloc(&ctx->point_order, npts * sizeof(int32_t)));
   RP_CUDA(cudaMalloc(&ctx->point_owner, npts * sizeof(int32_t)));
   RP_CUDA(cudaMalloc(&ctx->nseg_prev_pt, npts * sizeof(int32_t)));
+  RP_CUDA(cudaMalloc(&ctx->point_cnt, npts * sizeof(int2)));
+  RP_CUDA(cudaMemset(ctx->point_cnt, 0, npts * sizeof(int2)));
   RP_CUDA(cudaMemset(ctx->nseg_prev_pt, 0, npts * sizeof(int32_t)));
   // full-circle trapezoid nodes (cos, sin)(m * 2 pi / N), R-11
   double2* h = new double2[c.n_theta];
@@ -1188,13 +1068,18 @@ int rp_alloc_potential_scratch(rp_ctx* ctx) {
 
 template <int KIND, int VAR, bool UNIT = false>
 static int launch_integrate_one(rp_ctx* ctx, const Params& P) {
-  int occ = 0;
+  // persistent grid: resident warps per SM x SMs (occupancy queried once per instantiation)
+  static int occ_of_dev[64] = {0};
+  int& occ = occ_of_dev[ctx->cfg.device & 63];
   const size_t smem = sizeof(WarpSmem) * kWarps;
-  RP_CUDA(cudaFuncSetAttribute(k_integrate<KIND, VAR, UNIT>,
-                               cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
-  RP_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_integrate<KIND, VAR, UNIT>,
-                                                        32 * kWarps, smem));
-  if (occ < 1) occ = 1;
+  if (occ == 0) {
+    RP_CUDA(cudaFuncSetAttribute(k_integrate<KIND, VAR, UNIT>,
+                                 cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+    int o = 0;
+    RP_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&o, k_integrate<KIND, VAR, UNIT>,
+                                                          32 * kWarps, smem));
+    occ = o < 1 ? 1 : o;
+  }
   k_integrate<KIND, VAR, UNIT><<<ctx->sm_count * occ, 32 * kWarps, smem, ctx->stream>>>(
       P, ctx->sched_order, ctx->clipAB, ctx->trig_full, ctx->item_val, ctx->item_cnt,
       ctx->item_aux, ctx->counters);
@@ -1203,57 +1088,36 @@ static int launch_integrate_one(rp_ctx* ctx, const Params& P) {
 }
 
 // The integrator: the items, then (split_level > 0) the deferred subtree units and their
-// merge into the items.  One profiling record covers the whole integration.
+// merge into the items.  One profiling record covers the whole integration.  Everything is
+// stream-ordered: the unit launch reads its count from the device (no host synchronisation).
 template <int KIND, int VAR>
 static int launch_integrate(rp_ctx* ctx, const Params& P) {
   ProfScope ps(ctx, PK_INTEGRATE);
-  int rc = launch_integrate_one<KIND, VAR, false>(ctx, P);
-  if (rc) return rc;
-  ctx->last_units = 0;
-  if (KIND != RP_SRC_GRID || VAR < 4 || P.split_level <= 0) return RP_OK;
   cudaStream_t st = ctx->stream;
-  unsigned long long nu = 0;
-  RP_CUDA(cudaMemcpyAsync(&nu, ctx->counters + C_UNITS, sizeof(nu), cudaMemcpyDeviceToHost, st));
-  RP_CUDA(cudaStreamSynchronize(st));
-  if (nu == 0) return RP_OK;
-  if ((long long)nu > P.unit_cap) {  // overflowed pushes descended instead (see k_integrate)
-    nu = (unsigned long long)P.unit_cap;
-    RP_CUDA(cudaMemcpyAsync(ctx->counters + C_UNITS, &nu, sizeof(nu), cudaMemcpyHostToDevice, st));
-    RP_CUDA(cudaStreamSynchronize(st));
-  }
-  ctx->last_units = (int64_t)nu;
+  const bool split = KIND == RP_SRC_GRID && VAR >= 4 && P.split_level > 0;
+  const long long nf = (long long)P.npts * P.split_j;
+  if (split) RP_CUDA(cudaMemsetAsync(ctx->unit_ndef, 0, nf * sizeof(int32_t), st));
+  int rc = launch_integrate_one<KIND, VAR, false>(ctx, P);
+  if (rc || !split) return rc;
   ProfScope pu(ctx, PK_UNITS);
-  {
-    // longest-predicted-first order of the units (ctx->unit_key_sorted / unit_perm are free
-    // until the merge sort below)
-    k_unit_order_keys<<<(unsigned)((nu + 255) / 256), 256, 0, st>>>(
-        (long long)nu, ctx->unit_key, ctx->cost_prev, ctx->unit_okey);
-    RP_CHECK_LAUNCH();
-    size_t tmp = 0;
-    RP_CUDA(cub::DeviceRadixSort::SortPairs(nullptr, tmp, ctx->unit_okey, ctx->unit_key_sorted,
-                                            ctx->unit_iota, ctx->unit_perm, (int)nu, 0, 48, st));
-    rc = rp_ensure_cub_tmp(ctx, tmp);
-    if (rc) return rc;
-    tmp = ctx->cub_tmp_bytes;
-    RP_CUDA(cub::DeviceRadixSort::SortPairs(ctx->cub_tmp, tmp, ctx->unit_okey, ctx->unit_key_sorted,
-                                            ctx->unit_iota, ctx->unit_perm, (int)nu, 0, 48, st));
-  }
+  const long long slots = nf * P.unit_budget;
+  k_unit_order_keys<<<(unsigned)((slots + 255) / 256), 256, 0, st>>>(
+      slots, P.unit_budget, ctx->unit_ndef, ctx->unit_key, ctx->cost_prev, ctx->unit_okey);
+  RP_CHECK_LAUNCH();
+  size_t tmp = 0;
+  RP_CUDA(cub::DeviceRadixSort::SortPairs(nullptr, tmp, ctx->unit_okey, ctx->unit_okey_sorted,
+                                          ctx->unit_iota, ctx->unit_perm, (int)slots, 0, 48, st));
+  rc = rp_ensure_cub_tmp(ctx, tmp);
+  if (rc) return rc;
+  tmp = ctx->cub_tmp_bytes;
+  RP_CUDA(cub::DeviceRadixSort::SortPairs(ctx->cub_tmp, tmp, ctx->unit_okey, ctx->unit_okey_sorted,
+                                          ctx->unit_iota, ctx->unit_perm, (int)slots, 0, 48, st));
   Params PU = P;
   PU.unit_order = ctx->unit_perm;
   rc = launch_integrate_one<KIND, VAR, true>(ctx, PU);
   if (rc) return rc;
-  size_t tmp = 0;
-  RP_CUDA(cub::DeviceRadixSort::SortPairs(nullptr, tmp, ctx->unit_key, ctx->unit_key_sorted,
-                                          ctx->unit_iota, ctx->unit_perm, (int)nu, 0,
-                                          32 + kUnitShift, st));
-  rc = rp_ensure_cub_tmp(ctx, tmp);
-  if (rc) return rc;
-  tmp = ctx->cub_tmp_bytes;
-  RP_CUDA(cub::DeviceRadixSort::SortPairs(ctx->cub_tmp, tmp, ctx->unit_key, ctx->unit_key_sorted,
-                                          ctx->unit_iota, ctx->unit_perm, (int)nu, 0,
-                                          32 + kUnitShift, st));
-  k_merge_units<<<(unsigned)((nu + 255) / 256), 256, 0, st>>>(
-      (long long)nu, ctx->unit_key_sorted, ctx->unit_perm, ctx->unit_val, ctx->unit_cnt,
+  k_merge_units<<<(unsigned)((nf + 255) / 256), 256, 0, st>>>(
+      (int)nf, P.split_j, P.kmax, P.unit_budget, ctx->unit_ndef, ctx->unit_val, ctx->unit_cnt,
       ctx->unit_aux, ctx->item_val, ctx->item_cnt, ctx->item_aux);
   RP_CHECK_LAUNCH();
   return RP_OK;
@@ -1313,7 +1177,7 @@ static int run_potentials(rp_ctx* ctx, Params P, int32_t rank, int32_t world,
                                               ctx->sched_key_sorted, ctx->sched_idx,
                                               ctx->sched_order, (int)nd, 0, kbits, st));
     }
-    const int var = KIND != RP_SRC_GRID ? 0 : (P.interp == RP_INTERP_LAGRANGE3 ? 6 : ctx->eval_variant);
+    const int var = KIND != RP_SRC_GRID ? 0 : (P.interp == RP_INTERP_LAGRANGE3 ? 6 : 4);
     ctx->pred_info.active = 0;
     if (KIND == RP_SRC_GRID && ctx->pred_on && ctx->have_leaves && !shard_out && var != 0) {
       // Predictive-RP lines 1-12 on the host (R-26): forecast, partition, cluster, merge
@@ -1323,26 +1187,24 @@ static int run_potentials(rp_ctx* ctx, Params P, int32_t rank, int32_t world,
       P.bp_off = ctx->bp_off_dev;
       P.cluster = ctx->cluster_dev;
     }
-    P.split_level = (KIND == RP_SRC_GRID && var >= 4 && P.bp_off == nullptr && ctx->unit_key)
-                        ? ctx->split_level : 0;
+    P.split_level = (KIND == RP_SRC_GRID && var >= 4 && P.bp_off == nullptr) ? ctx->split_level : 0;
     P.split_j = ctx->split_j;
-    P.unit_budget = 64;
-    P.unit_cap = ctx->unit_cap;
+    P.unit_budget = kUnitBudget;
+    P.unit_ndef = ctx->unit_ndef;
     P.unit_key = ctx->unit_key;
     P.unit_val = ctx->unit_val;
     P.unit_cnt = ctx->unit_cnt;
     P.unit_aux = ctx->unit_aux;
-    int rc2 = var == 4 ? launch_integrate<KIND, 4>(ctx, P)
+    int rc2 = KIND != RP_SRC_GRID ? launch_integrate<KIND, 0>(ctx, P)
               : var == 6 ? launch_integrate<KIND, 6>(ctx, P)
-              : var == 7 ? launch_integrate<KIND, 7>(ctx, P)
-                         : launch_integrate<KIND, 0>(ctx, P);
+                         : launch_integrate<KIND, 4>(ctx, P);
     if (rc2) return rc2;
   }
   ProfScope ps_red(ctx, PK_REDUCE);
   k_reduce<<<(P.npts + 255) / 256, 256, 0, st>>>(
       P.npts, P.kmax, P.kap, ctx->sched_key, ctx->item_val, ctx->item_cnt, ctx->item_aux, owner,
       rank, row, world, phi, ax, ay, err, nseg, shard_out, ctx->cost_prev, ctx->nseg_prev_pt,
-      ctx->leaves_prev, ctx->counters);
+      ctx->leaves_prev, ctx->point_cnt, ctx->counters);
   RP_CHECK_LAUNCH();
   ctx->has_forecast = 1;
   ctx->have_leaves = shard_out ? 0 : 1;
@@ -1359,14 +1221,15 @@ int rp_potentials_impl(rp_ctx* ctx, int kind, const double src[6], int32_t rank,
   P.nx = c.nx; P.ny = c.ny; P.PX = ctx->PX; P.npts = c.nx * c.ny; P.kmax = c.history_depth;
   P.kap = kappa_of(ctx); P.k = ctx->k; P.H = ctx->H; P.n_theta = c.n_theta;
   P.max_depth = c.max_depth; P.n_root = c.n_root; P.rule = c.outer_rule;
-  P.variant = ctx->eval_variant;
+  P.variant = 0;
   P.interp = c.interp;
   P.hx = c.hx; P.hy = c.hy; P.inv_hx = 1.0 / c.hx; P.inv_hy = 1.0 / c.hy;
   P.cdt = c.c * c.dt; P.tau = c.tau; P.R = (double)P.kap * P.cdt;
   P.slot_doubles = ctx->slot_doubles; P.ring = ctx->ring; P.frames = ctx->frames_dev;
   P.amp = ctx->amp_dev;
   P.bp = nullptr; P.bp_off = nullptr; P.cluster = nullptr;
-  P.split_level = 0; P.split_j = 0; P.unit_budget = 0; P.unit_cap = 0; P.unit_order = nullptr; P.unit_key = nullptr; P.unit_val = nullptr;
+  P.split_level = 0; P.split_j = 0; P.unit_budget = 0; P.unit_ndef = nullptr;
+  P.unit_order = nullptr; P.unit_key = nullptr; P.unit_val = nullptr;
   P.unit_cnt = nullptr; P.unit_aux = nullptr;
   P.sx0 = src ? src[0] : 0; P.sy0 = src ? src[1] : 0; P.swidth = src ? src[2] : 0;
   P.sq = src ? src[3] : 0; P.sbx = src ? src[4] : 0; P.sby = src ? src[5] : 0;
@@ -1393,9 +1256,7 @@ int rp_potentials_impl(rp_ctx* ctx, int kind, const double src[6], int32_t rank,
       info->max_level = (int32_t)h[C_MAXLEV];
       info->kappa = P.kap;
       info->skipped = (int64_t)h[C_SKIP];
-      info->units = ctx->last_units;
-      info->unit_overflow = h[C_UOVF] ? 1 : 0;
-      info->pad = 0;
+      info->units = (int64_t)h[C_UNITS];
     }
     if (n_out) *n_out = (int64_t)h[C_NOUT];
   }
@@ -1413,14 +1274,4 @@ int rp_scatter_impl(rp_ctx* ctx, const double* shards, int32_t world, int64_t ca
   RP_CHECK_LAUNCH();
   ctx->has_forecast = 1;
   return RP_OK;
-}
-
-// development only (not in rp.h): per-phase SM cycles accumulated by k_integrate VAR 7
-extern "C" int rp_dev_phase_cycles(unsigned long long* out, int reset) {
-  if (cudaMemcpyFromSymbol(out, g_phase, sizeof(unsigned long long) * 6) != cudaSuccess) return -3;
-  if (reset) {
-    unsigned long long z[8] = {0};
-    cudaMemcpyToSymbol(g_phase, z, sizeof(z));
-  }
-  return 0;
 }

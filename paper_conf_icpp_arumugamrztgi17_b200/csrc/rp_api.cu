@@ -1,9 +1,13 @@
-#include <stdlib.h>
 // rp_api.cu -- the C ABI of librp (include/rp.h): context, history ring, state access and
 // the argument checking around the kernels of deposit.cu, potentials.cu, fields_push.cu.
 #include <new>
 
 #include "rp_internal.cuh"
+
+// every entry point: a context, and its device current for the call (restored on return)
+#define RP_ENTER(ctx)          \
+  if (!(ctx)) return RP_EINVAL; \
+  DeviceGuard device_guard_((ctx)->cfg.device)
 
 namespace {
 
@@ -53,9 +57,10 @@ void free_all(rp_ctx* c) {
                   c->sched_key, c->sched_key_sorted, c->sched_idx, c->sched_order, c->cost_prev,
                   c->item_val, c->item_cnt, c->item_aux, c->counters, c->amp_dev, c->trig_full,
                   c->point_key, c->point_key_sorted, c->point_idx, c->point_order,
-                  c->point_owner, c->nseg_prev_pt, c->hx_d, c->hy_d, c->hux_d, c->huy_d,
+                  c->point_owner, c->nseg_prev_pt, c->point_cnt, c->hx_d, c->hy_d, c->hux_d, c->huy_d,
                   c->mesh_d, c->leaves_prev, c->cluster_dev, c->bp_off_dev, c->bp_dev,
-                  c->unit_key, c->unit_key_sorted, c->unit_okey, c->unit_iota, c->unit_perm, c->unit_val,
+                  c->unit_key, c->unit_okey, c->unit_okey_sorted, c->unit_iota, c->unit_perm, c->unit_val,
+                  c->unit_ndef, c->partials_all, c->shard_buf, c->shards_all,
                   c->unit_cnt, c->unit_aux};
   for (void* p : ptrs)
     if (p) cudaFree(p);
@@ -65,13 +70,67 @@ void free_all(rp_ctx* c) {
   }
   for (auto e : c->ev_pool) cudaEventDestroy(e);
   delete[] c->fh;
+  if (c->comm && c->own_comm) {
+    if (const RpNccl* api = rp_nccl_api(nullptr)) api->comm_destroy(c->comm);
+  }
+  c->comm = nullptr;
+}
+
+__global__ void k_point_counts(int64_t n, const int2* __restrict__ pc, int32_t* __restrict__ nleaf,
+                               int32_t* __restrict__ capped) {
+  int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+  if (i >= n) return;
+  if (nleaf) nleaf[i] = pc[i].x;
+  if (capped) capped[i] = pc[i].y;
+}
+
+// NCCL all-gather of `bytes` per rank on the context's stream (rank order in recv)
+int allgather(rp_ctx* ctx, const void* send, void* recv, size_t bytes) {
+  std::string e;
+  const RpNccl* api = rp_nccl_api(&e);
+  if (!api) return rp_fail(ctx, RP_ENCCL, e.c_str());
+  ncclResult_t r = api->all_gather(send, recv, bytes, ncclUint8, ctx->comm, ctx->stream);
+  if (r != ncclSuccess) {
+    ctx->err = std::string("ncclAllGather: ") + api->error_string(r);
+    return RP_ENCCL;
+  }
+  return RP_OK;
+}
+
+// deposit of this rank's particles + (dist) all-gather of the partials + append
+int deposit_step(rp_ctx* ctx, const double* x, const double* y, const double* ux,
+                 const double* uy, double q, int64_t n, const rp_frame* fk, rp_deposit_info* info) {
+  int rc = rp_deposit_impl(ctx, x, y, ux, uy, q, n, fk, ctx->partial, info);
+  if (rc) return rc;
+  if (!ctx->dist_on) return rp_append_impl(ctx, ctx->partial, 1, fk);
+  if (!fk) return rp_fail(ctx, RP_EINVAL, "deposit_step: no frame");
+  rc = allgather(ctx, ctx->partial, ctx->partials_all, (size_t)rp_partial_bytes_impl(ctx));
+  if (rc) return rc;
+  return rp_append_impl(ctx, ctx->partials_all, ctx->world, fk);
+}
+
+// potentials on the full mesh: single call, or (dist) this rank's shard + all-gather + scatter
+int potentials_full(rp_ctx* ctx, double* phi, double* ax, double* ay, double* err, int32_t* nseg,
+                    rp_potential_info* info) {
+  if (!ctx->dist_on)
+    return rp_potentials_impl(ctx, RP_SRC_GRID, nullptr, 0, 1, phi, ax, ay, err, nseg, nullptr, 0,
+                              nullptr, info);
+  if (ctx->pred_on) return rp_fail(ctx, RP_EINVAL, "potentials: Predictive-RP is single-GPU only");
+  if (!phi || !ax || !ay) return rp_fail(ctx, RP_EINVAL, "potentials: null output");
+  int rc = rp_potentials_impl(ctx, RP_SRC_GRID, nullptr, ctx->rank, ctx->world, nullptr, nullptr,
+                              nullptr, nullptr, nullptr, ctx->shard_buf, ctx->shard_cap, nullptr,
+                              info);
+  if (rc) return rc;
+  rc = allgather(ctx, ctx->shard_buf, ctx->shards_all, (size_t)ctx->shard_cap * 6 * sizeof(double));
+  if (rc) return rc;
+  return rp_scatter_impl(ctx, ctx->shards_all, ctx->world, ctx->shard_cap, phi, ax, ay, err, nseg);
 }
 
 }  // namespace
 
 extern "C" {
 
-int rp_version(void) { return 100; }
+int rp_version(void) { return 200; }
 
 const char* rp_strerror(int code) {
   switch (code) {
@@ -79,6 +138,7 @@ const char* rp_strerror(int code) {
     case RP_EINVAL: return "invalid argument or configuration";
     case RP_ENOMEM: return "out of memory";
     case RP_ECUDA: return "CUDA error";
+    case RP_ENCCL: return "NCCL unavailable or a collective failed";
     case RP_ESTATE: return "call out of order";
     case RP_ENODEV: return "no usable CUDA device";
     default: return "unknown error";
@@ -96,6 +156,14 @@ int rp_set_schedule(rp_ctx* ctx, int32_t policy, int32_t k) {
     return rp_fail(ctx, RP_EINVAL, "set_schedule: k must be 1, 5, 9 or 25");
   ctx->sched_policy = policy;
   ctx->sched_k = policy == RP_SCHED_KNN ? k : 1;
+  return RP_OK;
+}
+
+int rp_set_work_split(rp_ctx* ctx, int32_t level) {
+  if (!ctx) return RP_EINVAL;
+  if (level != 0 && (level < 2 || level > ctx->cfg.max_depth))
+    return rp_fail(ctx, RP_EINVAL, "set_work_split: level must be 0 or 2..max_depth");
+  ctx->split_level = level;
   return RP_OK;
 }
 
@@ -123,7 +191,7 @@ int rp_predictive_info_read(rp_ctx* ctx, rp_predictive_info* out, int32_t* clust
 }
 
 int rp_profile_enable(rp_ctx* ctx, int32_t enable) {
-  if (!ctx) return RP_EINVAL;
+  RP_ENTER(ctx);
   RP_CUDA(cudaStreamSynchronize(ctx->stream));
   for (auto& r : ctx->prof) {
     ctx->ev_pool.push_back(r.a);
@@ -137,7 +205,8 @@ int rp_profile_enable(rp_ctx* ctx, int32_t enable) {
 }
 
 int rp_profile_read(rp_ctx* ctx, rp_profile* out) {
-  if (!ctx || !out) return RP_EINVAL;
+  RP_ENTER(ctx);
+  if (!out) return RP_EINVAL;
   RP_CUDA(cudaStreamSynchronize(ctx->stream));
   for (auto& r : ctx->prof) {
     float ms = 0.f;
@@ -157,18 +226,31 @@ int rp_profile_read(rp_ctx* ctx, rp_profile* out) {
   out->push_ms = ctx->prof_acc[PK_PUSH];
   out->integrate_launches = ctx->prof_integrate_launches;
   out->units_ms = ctx->prof_acc[PK_UNITS];
+  out->step_ms = ctx->prof_acc[PK_STEP];
   return RP_OK;
 }
 
-int rp_create(const rp_config* cfg, rp_ctx** out) {
+int rp_nccl_unique_id(unsigned char* id_out) {
+  if (!id_out) return RP_EINVAL;
+  const RpNccl* api = rp_nccl_api(nullptr);
+  if (!api) return RP_ENCCL;
+  ncclUniqueId id;
+  if (api->get_unique_id(&id) != ncclSuccess) return RP_ENCCL;
+  memcpy(id_out, &id, RP_NCCL_ID_BYTES);
+  return RP_OK;
+}
+
+int rp_create(const rp_config* cfg, const rp_dist* dist, rp_ctx** out) {
   if (!out) return RP_EINVAL;
   *out = nullptr;
   if (validate(cfg) != RP_OK) return RP_EINVAL;
+  if (dist && (dist->world < 1 || dist->rank < 0 || dist->rank >= dist->world)) return RP_EINVAL;
   int ndev = 0;
   if (cudaGetDeviceCount(&ndev) != cudaSuccess || ndev <= cfg->device || cfg->device < 0) {
     cudaGetLastError();
     return RP_ENODEV;
   }
+  DeviceGuard guard(cfg->device);  // the caller's device is restored on return
   rp_ctx* ctx = new (std::nothrow) rp_ctx();
   if (!ctx) return RP_ENOMEM;
   ctx->cfg = *cfg;
@@ -179,9 +261,6 @@ int rp_create(const rp_config* cfg, rp_ctx** out) {
   };
   if (cudaSetDevice(cfg->device) != cudaSuccess) return fail(RP_ENODEV);
   cudaDeviceGetAttribute(&ctx->sm_count, cudaDevAttrMultiProcessorCount, cfg->device);
-  if (const char* ev = getenv("RP_EVAL")) ctx->eval_variant = atoi(ev);
-  if (const char* sp = getenv("RP_SPLIT")) ctx->split_level = atoi(sp);
-  if (const char* sj = getenv("RP_SPLITJ")) ctx->split_j = atoi(sj);
   ctx->H = cfg->history_depth + 2;
   ctx->PX = cfg->nx + 2 * RP_PAD;
   ctx->PY = cfg->ny + 2 * RP_PAD;
@@ -201,17 +280,41 @@ int rp_create(const rp_config* cfg, rp_ctx** out) {
   int rc = rp_alloc_potential_scratch(ctx);
   if (rc) return fail(rc);
   // analytic amplitudes default to 1
-  double* ones = new double[ctx->H];
-  for (int i = 0; i < ctx->H; ++i) ones[i] = 1.0;
-  cudaError_t e = cudaMemcpy(ctx->amp_dev, ones, ctx->H * sizeof(double), cudaMemcpyHostToDevice);
-  delete[] ones;
-  if (e != cudaSuccess) return fail(RP_ECUDA);
+  std::vector<double> ones(ctx->H, 1.0);
+  if (cudaMemcpy(ctx->amp_dev, ones.data(), ctx->H * sizeof(double), cudaMemcpyHostToDevice) != cudaSuccess)
+    return fail(RP_ECUDA);
+  if (dist) {
+    ctx->dist_on = 1;
+    ctx->rank = dist->rank;
+    ctx->world = dist->world;
+    const int64_t pb = rp_partial_bytes_impl(ctx);
+    ctx->shard_cap = ((int64_t)npts + dist->world - 1) / dist->world;
+    if (cudaMalloc(&ctx->partials_all, (size_t)pb * dist->world) != cudaSuccess ||
+        cudaMalloc(&ctx->shard_buf, (size_t)ctx->shard_cap * 6 * sizeof(double)) != cudaSuccess ||
+        cudaMalloc(&ctx->shards_all, (size_t)ctx->shard_cap * 6 * sizeof(double) * dist->world) != cudaSuccess)
+      return fail(RP_ENOMEM);
+    if (dist->nccl_comm) {
+      ctx->comm = (ncclComm_t)dist->nccl_comm;
+    } else {
+      std::string e;
+      const RpNccl* api = rp_nccl_api(&e);
+      if (!api) return fail(RP_ENCCL);
+      ncclUniqueId id;
+      memcpy(&id, dist->nccl_id, RP_NCCL_ID_BYTES);
+      if (api->comm_init_rank(&ctx->comm, dist->world, id, dist->rank) != ncclSuccess) {
+        ctx->comm = nullptr;
+        return fail(RP_ENCCL);
+      }
+      ctx->own_comm = 1;
+    }
+  }
   *out = ctx;
   return RP_OK;
 }
 
 void rp_destroy(rp_ctx* ctx) {
   if (!ctx) return;
+  DeviceGuard guard(ctx->cfg.device);
   cudaStreamSynchronize(ctx->stream);
   free_all(ctx);
   delete ctx;
@@ -225,7 +328,7 @@ int rp_set_stream(rp_ctx* ctx, void* stream) {
 
 int rp_history_init(rp_ctx* ctx, int32_t n_pre, const rp_frame* frames_host,
                     const double* grids_dev, int32_t rigid) {
-  if (!ctx) return RP_EINVAL;
+  RP_ENTER(ctx);
   if (ctx->k >= 0) return rp_fail(ctx, RP_ESTATE, "history_init after the first deposit");
   if (n_pre < 1 || n_pre > ctx->cfg.history_depth + 1 || !frames_host)
     return rp_fail(ctx, RP_EINVAL, "history_init: n_pre out of range or no frames");
@@ -255,7 +358,7 @@ int rp_history_init(rp_ctx* ctx, int32_t n_pre, const rp_frame* frames_host,
 int rp_deposit(rp_ctx* ctx, const double* x, const double* y, const double* ux, const double* uy,
                double q, int64_t n, const rp_frame* frame_k, void* partial_dev,
                rp_deposit_info* info) {
-  if (!ctx) return RP_EINVAL;
+  RP_ENTER(ctx);
   return rp_deposit_impl(ctx, x, y, ux, uy, q, n, frame_k, partial_dev, info);
 }
 
@@ -263,24 +366,21 @@ int64_t rp_partial_bytes(const rp_ctx* ctx) { return ctx ? rp_partial_bytes_impl
 
 int rp_history_append(rp_ctx* ctx, const void* partials_dev, int32_t n_parts,
                       const rp_frame* frame_k) {
-  if (!ctx) return RP_EINVAL;
+  RP_ENTER(ctx);
   return rp_append_impl(ctx, partials_dev, n_parts, frame_k);
 }
 
 int rp_deposit_step(rp_ctx* ctx, const double* x, const double* y, const double* ux,
                     const double* uy, double q, int64_t n, const rp_frame* frame_k,
                     rp_deposit_info* info) {
-  if (!ctx) return RP_EINVAL;
-  int rc = rp_deposit_impl(ctx, x, y, ux, uy, q, n, frame_k, ctx->partial, info);
-  if (rc) return rc;
-  return rp_append_impl(ctx, ctx->partial, 1, frame_k);
+  RP_ENTER(ctx);
+  return deposit_step(ctx, x, y, ux, uy, q, n, frame_k, info);
 }
 
 int rp_compute_potentials(rp_ctx* ctx, double* phi, double* ax, double* ay, double* err,
                           int32_t* nseg, rp_potential_info* info) {
-  if (!ctx) return RP_EINVAL;
-  return rp_potentials_impl(ctx, RP_SRC_GRID, nullptr, 0, 1, phi, ax, ay, err, nseg, nullptr, 0,
-                            nullptr, info);
+  RP_ENTER(ctx);
+  return potentials_full(ctx, phi, ax, ay, err, nseg, info);
 }
 
 int64_t rp_shard_capacity(const rp_ctx* ctx, int32_t world) {
@@ -291,7 +391,7 @@ int64_t rp_shard_capacity(const rp_ctx* ctx, int32_t world) {
 
 int rp_compute_potentials_shard(rp_ctx* ctx, int32_t rank, int32_t world, double* shard_out,
                                 int64_t cap, int64_t* n_out, rp_potential_info* info) {
-  if (!ctx) return RP_EINVAL;
+  RP_ENTER(ctx);
   if (world < 1 || rank < 0 || rank >= world || !shard_out || cap < rp_shard_capacity(ctx, world))
     return rp_fail(ctx, RP_EINVAL, "potentials_shard: bad rank/world/cap");
   if (ctx->pred_on) return rp_fail(ctx, RP_EINVAL, "potentials_shard: Predictive-RP is single-call only");
@@ -301,7 +401,7 @@ int rp_compute_potentials_shard(rp_ctx* ctx, int32_t rank, int32_t world, double
 
 int rp_shard_scatter(rp_ctx* ctx, const double* shards, int32_t world, int64_t cap, double* phi,
                      double* ax, double* ay, double* err, int32_t* nseg) {
-  if (!ctx) return RP_EINVAL;
+  RP_ENTER(ctx);
   if (!shards || world < 1 || cap < rp_shard_capacity(ctx, world) || !phi || !ax || !ay)
     return rp_fail(ctx, RP_EINVAL, "shard_scatter: bad args");
   return rp_scatter_impl(ctx, shards, world, cap, phi, ax, ay, err, nseg);
@@ -310,21 +410,21 @@ int rp_shard_scatter(rp_ctx* ctx, const double* shards, int32_t world, int64_t c
 int rp_compute_fields(rp_ctx* ctx, const double* phi, const double* ax, const double* ay,
                       const double* ax_prev, const double* ay_prev, double* ex, double* ey,
                       double* bz) {
-  if (!ctx) return RP_EINVAL;
+  RP_ENTER(ctx);
   return rp_fields_impl(ctx, phi, ax, ay, ax_prev, ay_prev, ex, ey, bz);
 }
 
 int rp_push_particles(rp_ctx* ctx, double* x, double* y, double* ux, double* uy, int64_t n,
                       double q_over_mc, double bz_ext, const double* ex, const double* ey,
                       const double* bz) {
-  if (!ctx) return RP_EINVAL;
+  RP_ENTER(ctx);
   return rp_push_impl(ctx, x, y, ux, uy, n, q_over_mc, bz_ext, ex, ey, bz);
 }
 
 int rp_step_host(rp_ctx* ctx, double* xh, double* yh, double* uxh, double* uyh, int64_t n,
                  double q, const rp_frame* frame_k, double q_over_mc, double bz_ext,
                  double* mesh_host, rp_potential_info* info) {
-  if (!ctx) return RP_EINVAL;
+  RP_ENTER(ctx);
   if (n < 0 || (n > 0 && (!xh || !yh || !uxh || !uyh)) || !mesh_host || !frame_k)
     return rp_fail(ctx, RP_EINVAL, "step_host: bad args");
   const size_t npts = (size_t)ctx->cfg.nx * ctx->cfg.ny;
@@ -350,18 +450,21 @@ int rp_step_host(rp_ctx* ctx, double* xh, double* yh, double* uxh, double* uyh, 
   double* m = ctx->mesh_d;
   double *phi = m, *ax = m + npts, *ay = m + 2 * npts, *ex = m + 3 * npts, *ey = m + 4 * npts,
          *bz = m + 5 * npts, *axp = m + 6 * npts, *ayp = m + 7 * npts;
-  int rc = rp_deposit_step(ctx, ctx->hx_d, ctx->hy_d, ctx->hux_d, ctx->huy_d, q, n, frame_k, nullptr);
-  if (rc) return rc;
-  rc = rp_potentials_impl(ctx, RP_SRC_GRID, nullptr, 0, 1, phi, ax, ay, nullptr, nullptr, nullptr,
-                          0, nullptr, info);
-  if (rc) return rc;
-  rc = rp_fields_impl(ctx, phi, ax, ay, ctx->have_prev_A ? axp : nullptr,
-                      ctx->have_prev_A ? ayp : nullptr, ex, ey, bz);
-  if (rc) return rc;
-  RP_CUDA(cudaMemcpyAsync(axp, ax, 2 * npts * sizeof(double), cudaMemcpyDeviceToDevice, st));
-  ctx->have_prev_A = 1;
-  rc = rp_push_impl(ctx, ctx->hx_d, ctx->hy_d, ctx->hux_d, ctx->huy_d, n, q_over_mc, bz_ext, ex, ey, bz);
-  if (rc) return rc;
+  {
+    ProfScope ps(ctx, PK_STEP);  // the device part of the step, between the copies
+    int rc = deposit_step(ctx, ctx->hx_d, ctx->hy_d, ctx->hux_d, ctx->huy_d, q, n, frame_k, nullptr);
+    if (rc) return rc;
+    rc = potentials_full(ctx, phi, ax, ay, nullptr, nullptr, info);
+    if (rc) return rc;
+    rc = rp_fields_impl(ctx, phi, ax, ay, ctx->have_prev_A ? axp : nullptr,
+                        ctx->have_prev_A ? ayp : nullptr, ex, ey, bz);
+    if (rc) return rc;
+    RP_CUDA(cudaMemcpyAsync(axp, ax, 2 * npts * sizeof(double), cudaMemcpyDeviceToDevice, st));
+    ctx->have_prev_A = 1;
+    rc = rp_push_impl(ctx, ctx->hx_d, ctx->hy_d, ctx->hux_d, ctx->huy_d, n, q_over_mc, bz_ext, ex,
+                      ey, bz);
+    if (rc) return rc;
+  }
   RP_CUDA(cudaMemcpyAsync(mesh_host, m, 6 * npts * sizeof(double), cudaMemcpyDeviceToHost, st));
   if (n > 0) {
     RP_CUDA(cudaMemcpyAsync(xh, ctx->hx_d, nb, cudaMemcpyDeviceToHost, st));
@@ -375,7 +478,7 @@ int rp_step_host(rp_ctx* ctx, double* xh, double* yh, double* uxh, double* uyh, 
 
 int rp_load_state(rp_ctx* ctx, int32_t k, int32_t n_pre, const rp_frame* frames_host,
                   const double* ring_dev) {
-  if (!ctx) return RP_EINVAL;
+  RP_ENTER(ctx);
   if (k < 0 || n_pre < 0 || n_pre > ctx->cfg.history_depth + 1 || !frames_host || !ring_dev)
     return rp_fail(ctx, RP_EINVAL, "load_state: bad args");
   const rp_config& c = ctx->cfg;
@@ -399,7 +502,7 @@ int rp_load_state(rp_ctx* ctx, int32_t k, int32_t n_pre, const rp_frame* frames_
 }
 
 int rp_save_state(rp_ctx* ctx, int32_t* k_out, double* ring_dev, rp_frame* frames_host) {
-  if (!ctx) return RP_EINVAL;
+  RP_ENTER(ctx);
   const rp_config& c = ctx->cfg;
   if (k_out) *k_out = ctx->k;
   if (frames_host)
@@ -417,7 +520,7 @@ int rp_save_state(rp_ctx* ctx, int32_t* k_out, double* ring_dev, rp_frame* frame
 }
 
 int rp_debug_bins(rp_ctx* ctx, int32_t* bins_dev, int64_t n) {
-  if (!ctx) return RP_EINVAL;
+  RP_ENTER(ctx);
   if (!bins_dev || n != ctx->last_n) return rp_fail(ctx, RP_EINVAL, "debug_bins: n must equal the last deposit's n");
   if (n == 0) return RP_OK;
   k_bins_out<<<(unsigned)((n + 255) / 256), 256, 0, ctx->stream>>>(n, ctx->cfg.nx * ctx->cfg.ny,
@@ -426,8 +529,19 @@ int rp_debug_bins(rp_ctx* ctx, int32_t* bins_dev, int64_t n) {
   return RP_OK;
 }
 
+int rp_debug_point_counts(rp_ctx* ctx, int32_t* nleaf_dev, int32_t* capped_dev, int64_t n) {
+  RP_ENTER(ctx);
+  const int64_t npts = (int64_t)ctx->cfg.nx * ctx->cfg.ny;
+  if (n != npts) return rp_fail(ctx, RP_EINVAL, "debug_point_counts: n must be nx*ny");
+  if (!ctx->has_forecast) return rp_fail(ctx, RP_ESTATE, "debug_point_counts: no potentials call yet");
+  k_point_counts<<<(unsigned)((n + 255) / 256), 256, 0, ctx->stream>>>(n, ctx->point_cnt, nleaf_dev,
+                                                                        capped_dev);
+  RP_CHECK_LAUNCH();
+  return RP_OK;
+}
+
 int rp_debug_clip(rp_ctx* ctx, double* ab_dev, int64_t n) {
-  if (!ctx) return RP_EINVAL;
+  RP_ENTER(ctx);
   const int64_t want = (int64_t)ctx->cfg.nx * ctx->cfg.ny * ctx->cfg.history_depth;
   if (!ab_dev || n != want) return rp_fail(ctx, RP_EINVAL, "debug_clip: n must be nx*ny*history_depth");
   if (!ctx->has_forecast) return rp_fail(ctx, RP_ESTATE, "debug_clip: no potentials call yet");
@@ -440,14 +554,15 @@ int rp_debug_potentials_analytic(rp_ctx* ctx, int32_t kind, double x0, double y0
                                  double q, double bx, double by, const double* amp_host,
                                  double* phi, double* ax, double* ay, double* err, int32_t* nseg,
                                  rp_potential_info* info) {
-  if (!ctx) return RP_EINVAL;
+  RP_ENTER(ctx);
   if ((kind != RP_SRC_GAUSS && kind != RP_SRC_DISK) || !(width > 0))
     return rp_fail(ctx, RP_EINVAL, "debug_potentials_analytic: bad source");
-  double* h = new double[ctx->H];
+  std::vector<double> h(ctx->H);
   for (int i = 0; i < ctx->H; ++i) h[i] = amp_host ? amp_host[i] : 1.0;
-  cudaError_t e = cudaMemcpy(ctx->amp_dev, h, ctx->H * sizeof(double), cudaMemcpyHostToDevice);
-  delete[] h;
-  RP_CUDA(e);
+  // stream-ordered upload; the host vector must outlive the copy, hence the sync
+  RP_CUDA(cudaMemcpyAsync(ctx->amp_dev, h.data(), ctx->H * sizeof(double), cudaMemcpyHostToDevice,
+                          ctx->stream));
+  RP_CUDA(cudaStreamSynchronize(ctx->stream));
   double src[6] = {x0, y0, width, q, bx, by};
   int saved = ctx->has_forecast;
   ctx->has_forecast = 0;

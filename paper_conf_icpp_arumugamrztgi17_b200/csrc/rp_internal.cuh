@@ -4,6 +4,7 @@
 #pragma once
 
 #include <cuda_runtime.h>
+#include <nccl.h>
 #include <stdint.h>
 #include <string.h>
 
@@ -13,6 +14,33 @@
 #include "../../include/rp.h"
 
 #define RP_PAD 3  // zero border (nodes) around every ring grid: stencils never bounds-check
+#define RP_NCCL_ID_BYTES 128
+
+// NCCL entry points, resolved at run time (nccl_dyn.cu)
+struct RpNccl {
+  void* handle;
+  ncclResult_t (*get_unique_id)(ncclUniqueId*);
+  ncclResult_t (*comm_init_rank)(ncclComm_t*, int, ncclUniqueId, int);
+  ncclResult_t (*comm_destroy)(ncclComm_t);
+  ncclResult_t (*all_gather)(const void*, void*, size_t, ncclDataType_t, ncclComm_t,
+                             cudaStream_t);
+  const char* (*error_string)(ncclResult_t);
+  ncclResult_t (*get_version)(int*);
+};
+const RpNccl* rp_nccl_api(std::string* err);
+
+// Makes the context's device current for the duration of an entry point and restores the
+// caller's device on exit (contexts on different GPUs in one process stay independent).
+struct DeviceGuard {
+  int prev = -1, dev;
+  explicit DeviceGuard(int d) : dev(d) {
+    if (cudaGetDevice(&prev) != cudaSuccess) prev = -1;
+    if (prev != dev) cudaSetDevice(dev);
+  }
+  ~DeviceGuard() {
+    if (prev >= 0 && prev != dev) cudaSetDevice(prev);
+  }
+};
 
 struct rp_ctx {
   rp_config cfg;
@@ -21,6 +49,16 @@ struct rp_ctx {
   size_t slot_doubles = 0;   // PX * PY * 4
   cudaStream_t stream = 0;
   int sm_count = 0;
+
+  // multi-GPU (rp_dist): mesh points sharded over `world` ranks, history
+  // replicated; the two exchanges of a step are NCCL all-gathers on `stream`
+  int dist_on = 0, rank = 0, world = 1;
+  ncclComm_t comm = nullptr;
+  int own_comm = 0;                 // created by rp_create (destroyed by rp_destroy)
+  unsigned char* partials_all = nullptr;  // [world][rp_partial_bytes]
+  double* shard_buf = nullptr;      // [shard_cap][6] this rank's potential shard
+  double* shards_all = nullptr;     // [world][shard_cap][6]
+  int64_t shard_cap = 0;
 
   // history: ring [H][PY][PX][4] FP64 and frames [H]
   double* ring = nullptr;
@@ -61,7 +99,6 @@ struct rp_ctx {
   int has_forecast = 0;
   int sched_policy = 1;             // RP_SCHED_*
   int sched_k = 9;                  // kNN neighbours
-  int eval_variant = 4;             // integrator evaluation loop (development A/B: RP_EVAL)
 
   // Predictive-RP variant (rp_set_predictive, DESIGN R-26)
   int pred_on = 0, pred_knn = 9, pred_m = 0, pred_iters = 20;
@@ -74,19 +111,19 @@ struct rp_ctx {
   std::vector<int32_t> cluster_host;
   rp_predictive_info pred_info{};
 
-  // subtree work units of the deep trees (k_integrate split_level)
-  int split_level = 12;             // RP_SPLIT overrides; 0 = off
-  int split_j = 1;                  // RP_SPLITJ: split the trees of subregions j < split_j
-  long long unit_cap = 0;           // even
+  // subtree work units of the deep trees (k_integrate split_level; rp_set_work_split)
+  int split_level = 12;             // 0 = off
+  int split_j = 1;                  // split the trees of subregions j < split_j (the near field)
+  long long unit_slots = 0;         // npts * split_j * unit budget
+  int32_t* unit_ndef = nullptr;     // [npts * split_j] units deferred per near-field item
   unsigned long long* unit_key = nullptr;
-  unsigned long long* unit_key_sorted = nullptr;
-  unsigned long long* unit_okey = nullptr;  // launch-order keys of the units
+  unsigned long long* unit_okey = nullptr;  // launch-order keys of the slots
+  unsigned long long* unit_okey_sorted = nullptr;
   int32_t* unit_iota = nullptr;
   int32_t* unit_perm = nullptr;
   double4* unit_val = nullptr;
   int4* unit_cnt = nullptr;
   uint2* unit_aux = nullptr;
-  int64_t last_units = 0;           // units of the last call (diagnostics)
 
   // sharding scratch
   int32_t* point_key = nullptr;     // per point predicted work key
@@ -95,6 +132,7 @@ struct rp_ctx {
   int32_t* point_order = nullptr;
   int32_t* point_owner = nullptr;   // rank owning each point
   int32_t* nseg_prev_pt = nullptr;  // per point segments of the last step (shard map)
+  int2* point_cnt = nullptr;        // per point (leaves, capped) of the last call
 
   // end-to-end (host buffer) path scratch
   int64_t host_cap = 0;
@@ -110,12 +148,12 @@ struct rp_ctx {
   int prof_on = 0;
   std::vector<ProfRec> prof;
   std::vector<cudaEvent_t> ev_pool;
-  double prof_acc[9] = {0, 0, 0, 0, 0, 0, 0, 0, 0};
+  double prof_acc[10] = {0, 0, 0, 0, 0, 0, 0, 0, 0, 0};
   int64_t prof_integrate_launches = 0;
 };
 
 enum { PK_DEPOSIT = 0, PK_APPEND, PK_CLIP, PK_SORT, PK_INTEGRATE, PK_REDUCE, PK_FIELDS, PK_PUSH,
-       PK_UNITS };
+       PK_UNITS, PK_STEP };
 
 static inline cudaEvent_t prof_event(rp_ctx* ctx) {
   if (!ctx->ev_pool.empty()) {

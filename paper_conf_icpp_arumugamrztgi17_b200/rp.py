@@ -48,7 +48,8 @@ class rp_profile(C.Structure):
     _fields_ = [("deposit_ms", C.c_double), ("append_ms", C.c_double), ("clip_ms", C.c_double),
                 ("sort_ms", C.c_double), ("integrate_ms", C.c_double), ("reduce_ms", C.c_double),
                 ("fields_ms", C.c_double), ("push_ms", C.c_double),
-                ("integrate_launches", C.c_int64), ("units_ms", C.c_double)]
+                ("integrate_launches", C.c_int64), ("units_ms", C.c_double),
+                ("step_ms", C.c_double)]
 
     def as_dict(self) -> dict:
         return {k: getattr(self, k) for k, _ in self._fields_}
@@ -58,8 +59,15 @@ class rp_potential_info(C.Structure):
     _fields_ = [("evals", C.c_int64), ("nodes", C.c_int64), ("segments", C.c_int64),
                 ("leaves", C.c_int64), ("capped", C.c_int64), ("ties", C.c_int64),
                 ("items", C.c_int64), ("max_level", C.c_int32), ("kappa", C.c_int32),
-                ("skipped", C.c_int64), ("units", C.c_int64), ("unit_overflow", C.c_int32),
-                ("pad", C.c_int32)]
+                ("skipped", C.c_int64), ("units", C.c_int64)]
+
+
+RP_NCCL_ID_BYTES = 128
+
+
+class rp_dist(C.Structure):
+    _fields_ = [("rank", C.c_int32), ("world", C.c_int32), ("nccl_comm", C.c_void_p),
+                ("nccl_id", C.c_ubyte * RP_NCCL_ID_BYTES)]
 
     def as_dict(self) -> dict:
         return {k: getattr(self, k) for k, _ in self._fields_}
@@ -90,7 +98,9 @@ _SIG = {
     "rp_set_predictive": (C.c_int, [_vp, _i32, _i32, _i32, _i32]),
     "rp_predictive_info_read": (C.c_int, [_vp, _P(rp_predictive_info), _vp]),
     "rp_profile_read": (C.c_int, [_vp, _P(rp_profile)]),
-    "rp_create": (C.c_int, [_P(rp_config), _P(_vp)]),
+    "rp_create": (C.c_int, [_P(rp_config), _P(rp_dist), _P(_vp)]),
+    "rp_nccl_unique_id": (C.c_int, [_vp]),
+    "rp_set_work_split": (C.c_int, [_vp, _i32]),
     "rp_destroy": (None, [_vp]),
     "rp_set_stream": (C.c_int, [_vp, _vp]),
     "rp_history_init": (C.c_int, [_vp, _i32, _P(rp_frame), _vp, _i32]),
@@ -113,6 +123,7 @@ _SIG = {
     "rp_save_state": (C.c_int, [_vp, _P(_i32), _vp, _P(rp_frame)]),
     "rp_debug_bins": (C.c_int, [_vp, _vp, _i64]),
     "rp_debug_clip": (C.c_int, [_vp, _vp, _i64]),
+    "rp_debug_point_counts": (C.c_int, [_vp, _vp, _vp, _i64]),
     "rp_debug_potentials_analytic": (C.c_int, [_vp, _i32, _d, _d, _d, _d, _d, _d, _vp, _vp, _vp,
                                                _vp, _vp, _vp, _P(rp_potential_info)]),
 }
@@ -226,13 +237,33 @@ def rp_profile_read(ctx) -> rp_profile:
     return out
 
 
+def rp_nccl_unique_id() -> bytes:
+    """A fresh ncclUniqueId (128 bytes) for rp_create's rp_dist (call on rank 0, broadcast)."""
+    buf = (C.c_ubyte * RP_NCCL_ID_BYTES)()
+    _check(_lib.rp_nccl_unique_id(C.cast(buf, _vp)), None, "rp_nccl_unique_id")
+    return bytes(buf)
+
+
 def rp_create(nx, ny, hx, hy, history_depth, c, dt, tau, n_theta=64, max_depth=30, n_root=2,
-              device=0, outer_rule=0, interp=0):
+              device=0, outer_rule=0, interp=0, dist=None):
+    """dist: None (single GPU) or (rank, world, nccl_id bytes) -- librp then creates the
+    NCCL communicator (collective over the ranks) and exchanges inside its calls."""
     cfg = rp_config(nx, ny, hx, hy, history_depth, c, dt, tau, n_theta, max_depth, n_root, device,
                     outer_rule, interp)
+    d = None
+    if dist is not None:
+        rank, world, nid = dist
+        if len(nid) != RP_NCCL_ID_BYTES:
+            raise ValueError("nccl_id: expected 128 bytes")
+        d = rp_dist(int(rank), int(world), None, (C.c_ubyte * RP_NCCL_ID_BYTES)(*nid))
     out = C.c_void_p()
-    _check(_lib.rp_create(C.byref(cfg), C.byref(out)), None, "rp_create")
+    _check(_lib.rp_create(C.byref(cfg), C.byref(d) if d is not None else None, C.byref(out)),
+           None, "rp_create")
     return out
+
+
+def rp_set_work_split(ctx, level) -> None:
+    _check(_lib.rp_set_work_split(ctx, int(level)), ctx, "rp_set_work_split")
 
 
 def rp_destroy(ctx) -> None:
@@ -353,6 +384,13 @@ def rp_save_state(ctx, ring=None, H=None):
 def rp_debug_clip(ctx, ab) -> None:
     """ab: float64 CUDA tensor of nx*ny*history_depth*2 elements ((A, B) per item)."""
     _check(_lib.rp_debug_clip(ctx, _f64(ab, "ab"), ab.numel() // 2), ctx, "rp_debug_clip")
+
+
+def rp_debug_point_counts(ctx, nleaf=None, capped=None) -> None:
+    """nleaf / capped: int32 CUDA tensors of nx*ny elements (either may be None)."""
+    n = (nleaf if nleaf is not None else capped).numel()
+    _check(_lib.rp_debug_point_counts(ctx, _i32t(nleaf, "nleaf"), _i32t(capped, "capped"), n),
+           ctx, "rp_debug_point_counts")
 
 
 def rp_debug_bins(ctx, bins) -> None:

@@ -4,15 +4,21 @@ over ranks (mesh points sharded, history replicated).
 Per step k on every rank (torch.distributed is plumbing only; every arithmetic step
 runs in librp's kernels):
 
-  world == 1:  rp_deposit_step -> rp_compute_potentials
-  world  > 1:  rp_deposit(local particle shard) -> all_gather(partial grids)
+  world == 1, or world > 1 with transport "nccl" (the product path: librp owns an NCCL
+  communicator made from a unique id broadcast over the process group, and exchanges inside
+  its calls):
+               rp_deposit_step -> rp_compute_potentials                  [full mesh]
+  world > 1 with transport "host" (a caller-side transport, e.g. gloo for the CPU tests
+  and for two ranks sharing one GPU, where NCCL refuses duplicate devices):
+               rp_deposit(local particle shard) -> all_gather(partial grids)
                -> rp_history_append(partials in rank order)              [replicated ring]
                -> rp_compute_potentials_shard(rank)                      [owned points]
                -> all_gather(shards) -> rp_shard_scatter                 [full mesh]
   then         rp_compute_fields (replicated) -> rp_push_particles (local shard)
 
-``ops`` defaults to the librp binding; tests substitute a CPU stand-in to exercise the
-multi-process plumbing with the gloo backend.
+Both transports give bit-identical results for any number of ranks (exact deposition, the
+same shard map).  ``ops`` defaults to the librp binding; tests substitute a CPU stand-in to
+exercise the multi-process plumbing with the gloo backend.
 """
 from __future__ import annotations
 
@@ -23,7 +29,8 @@ import workloads as W
 
 
 class Simulation:
-    def __init__(self, cfg: W.Config, device=None, group=None, ops=None, particles=None):
+    def __init__(self, cfg: W.Config, device=None, group=None, ops=None, particles=None,
+                 transport: str = "host"):
         if ops is None:
             from . import rp as ops
         self.ops = ops
@@ -36,9 +43,19 @@ class Simulation:
             self.rank, self.world = 0, 1
         self.device = torch.device("cuda", torch.cuda.current_device()) if device is None else torch.device(device)
         dev_index = self.device.index if self.device.type == "cuda" else 0
+        if transport not in ("host", "nccl"):
+            raise ValueError(transport)
+        # librp exchanges over its own NCCL communicator (world > 1, transport "nccl")
+        self.in_lib = self.world == 1 or transport == "nccl"
+        dist_arg = None
+        if self.world > 1 and transport == "nccl":
+            import torch.distributed as dist
+            obj = [ops.rp_nccl_unique_id() if self.rank == 0 else None]
+            dist.broadcast_object_list(obj, src=dist.get_global_rank(group, 0), group=group)
+            dist_arg = (self.rank, self.world, obj[0])
         self.ctx = ops.rp_create(cfg.nx, cfg.ny, cfg.hx, cfg.hy, cfg.kappa_max, cfg.c, cfg.dt,
                                  cfg.tau, cfg.n_theta, cfg.max_depth, cfg.n_root, dev_index or 0,
-                                 cfg.rule, cfg.interp)
+                                 cfg.rule, cfg.interp, dist=dist_arg)
         if self.device.type == "cuda":
             ops.rp_set_stream(self.ctx, torch.cuda.current_stream(self.device))
         ops.rp_history_init(self.ctx, cfg.n_pre, W.frames(cfg, range(-cfg.n_pre, 0)), None, True)
@@ -55,7 +72,7 @@ class Simulation:
         self.A = [(torch.zeros(npts, **f64), torch.zeros(npts, **f64)) for _ in range(2)]
         self.nseg = torch.zeros(npts, dtype=torch.int32, device=self.device)
         self.k = 0
-        if self.world > 1:
+        if not self.in_lib:
             pb = ops.rp_partial_bytes(self.ctx)  # opaque exact partial sums
             self.partial = torch.zeros(pb, dtype=torch.uint8, device=self.device)
             self.partials = torch.zeros(self.world * pb, dtype=torch.uint8, device=self.device)
@@ -80,7 +97,7 @@ class Simulation:
         fk = W.frame(cfg, self.k)
         ax, ay = self.A[self.k % 2]
         axp, ayp = self.A[(self.k + 1) % 2]
-        if self.world == 1:
+        if self.in_lib:
             ops.rp_deposit_step(self.ctx, self.x, self.y, self.ux, self.uy, self.q, fk)
             inf = ops.rp_compute_potentials(self.ctx, self.phi, ax, ay, self.err, self.nseg, info=info)
         else:

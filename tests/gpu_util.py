@@ -42,27 +42,38 @@ def gpu_potentials(ctx, npts):
     out = {k: torch.zeros(npts, dtype=torch.float64, device=dev) for k in ("phi", "ax", "ay", "err")}
     nseg = torch.zeros(npts, dtype=torch.int32, device=dev)
     info = rp.rp_compute_potentials(ctx, out["phi"], out["ax"], out["ay"], out["err"], nseg, info=True)
+    nleaf = torch.zeros(npts, dtype=torch.int32, device=dev)
+    capped = torch.zeros(npts, dtype=torch.int32, device=dev)
+    rp.rp_debug_point_counts(ctx, nleaf, capped)
     torch.cuda.synchronize()
     res = {k: v.cpu().numpy() for k, v in out.items()}
     res["nseg"] = nseg.cpu().numpy()
+    res["nleaf"] = nleaf.cpu().numpy()
+    res["capped"] = capped.cpu().numpy()
     return res, info
 
 
 def compare_potentials(gpu: dict, orc, pts, rel=REL):
-    """Element-by-element: |delta| <= rel * max(|phi|, |ax|, |ay|)_oracle per point and
-    equal nseg; points the oracle flags as ties (decision margin < 1e-9) are reported."""
+    """Element-by-element: |delta| <= rel * max(|phi|, |ax|, |ay|)_oracle per
+    point for phi, A_x, A_y and the error estimate eps (the 7-tuple's p.eps, Alg. 1
+    line 23 P:148), equal nseg, and -- when the GPU result carries them -- equal per-point
+    nleaf and capped; points the oracle flags as ties (decision margin < 1e-9) are reported."""
     pts = np.asarray(pts)
     scale = np.maximum.reduce([np.abs(orc["phi"]), np.abs(orc["ax"]), np.abs(orc["ay"])])
     scale = np.where(scale > 0, scale, 1e-300)
     tie = orc["ties"] > 0
     bad = []
-    for key in ("phi", "ax", "ay"):
+    keys = ("phi", "ax", "ay", "err") if "err" in gpu else ("phi", "ax", "ay")
+    for key in keys:
         d = np.abs(gpu[key][pts] - orc[key])
         bad.append(d > rel * scale)
     nseg_bad = gpu["nseg"][pts] != orc["nseg"]
+    for key in ("nleaf", "capped"):
+        if key in gpu:
+            nseg_bad = nseg_bad | (gpu[key][pts] != orc[key])
     fail = (np.logical_or.reduce(bad) | nseg_bad) & ~tie
     worst = 0.0
-    for key in ("phi", "ax", "ay"):
+    for key in keys:
         worst = max(worst, float(np.max(np.abs(gpu[key][pts] - orc[key]) / scale)) if len(pts) else 0.0)
     return fail, worst, int(tie.sum())
 

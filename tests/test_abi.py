@@ -35,7 +35,7 @@ def test_library_exports_every_declared_symbol():
 
 def test_host_side_calls_without_gpu():
     from paper_conf_icpp_arumugamrztgi17_b200 import rp
-    assert rp.rp_version() == 100
+    assert rp.rp_version() == 200
     assert rp.rp_strerror(0) == "ok"
     assert rp.rp_strerror(-5) == "call out of order"
     # invalid configurations are rejected before any device call
@@ -49,3 +49,28 @@ def test_host_side_calls_without_gpu():
         rp.rp_create(32, 32, 1.0, 1.0, 10, 1.0, 1.0, 1e-6, n_root=3)
     assert e.value.code == -1
     assert rp.rp_shard_capacity(None, 2) == 0
+    # multi-GPU membership is validated before any device call: rank outside [0, world)
+    nid = bytes(rp.RP_NCCL_ID_BYTES)
+    for rank, world in ((2, 2), (-1, 2), (0, 0)):
+        with pytest.raises(rp.RpError) as e:
+            rp.rp_create(32, 32, 1.0, 1.0, 10, 1.0, 1.0, 1e-6, dist=(rank, world, nid))
+        assert e.value.code == -1
+    with pytest.raises(ValueError):
+        rp.rp_create(32, 32, 1.0, 1.0, 10, 1.0, 1.0, 1e-6, dist=(0, 1, b"short"))
+    assert rp.rp_strerror(-4).startswith("NCCL")
+    # setters reject bad arguments on a NULL context before touching it
+    with pytest.raises(rp.RpError):
+        rp.rp_set_work_split(None, 5)
+
+
+def test_nccl_unique_id_loads_nccl_at_run_time():
+    """librp resolves NCCL with dlopen (no link-time dependency): a unique id for rp_dist can
+    be made on a host without a GPU."""
+    from paper_conf_icpp_arumugamrztgi17_b200 import rp
+    try:
+        a = rp.rp_nccl_unique_id()
+    except rp.RpError as e:  # pragma: no cover - an image without libnccl
+        assert e.code == -4
+        pytest.skip("libnccl.so.2 not loadable here")
+    b = rp.rp_nccl_unique_id()
+    assert len(a) == rp.RP_NCCL_ID_BYTES and a != b

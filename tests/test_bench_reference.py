@@ -31,3 +31,20 @@ def test_reference_arm_under_torchrun_two_ranks():
     assert d["cpu_baseline"]["kind"] == "oracle"
     assert d["cpu_baseline"]["cores"] == len(os.sched_getaffinity(0))
     assert d["e2e"]["h2d_bytes_per_step"] == 0 and d["e2e"]["value"] == d["value"]
+
+
+def test_bench_self_spawns_ranks_without_torchrun():
+    """`bench.py --gpus 2` with WORLD_SIZE unset relaunches itself as 2 ranks through
+    torch.distributed.run (the driver may call it either way); the oracle arm's rank 0 prints
+    the one line, the other rank exits 0."""
+    env = dict(os.environ)
+    for k in ("WORLD_SIZE", "RANK", "LOCAL_RANK", "OMP_NUM_THREADS"):
+        env.pop(k, None)
+    cmd = [sys.executable, "bench.py", "--impl", "reference", "--gpus", "2", "--config", "1",
+           "--steps", "1", "--warmup", "1"]
+    p = subprocess.run(cmd, cwd=ROOT, env=env, capture_output=True, text=True, timeout=600)
+    assert p.returncode == 0, p.stderr[-2000:]
+    lines = [ln for ln in p.stdout.splitlines() if ln.startswith("{")]
+    assert len(lines) == 1, p.stdout
+    d = json.loads(lines[0])
+    assert d["impl"] == "reference" and d["n_gpus"] == 2 and d["evals_per_s"] > 0

@@ -35,7 +35,8 @@ class OracleOps:
     """CPU stand-in for the librp binding with the C-ABI semantics of include/rp.h."""
 
     def rp_create(self, nx, ny, hx, hy, kap, c, dt, tau, n_theta, max_depth, n_root, dev, rule=0,
-                  interp=0):
+                  interp=0, dist=None):
+        assert dist is None  # the stand-in has no NCCL: the host (gloo) transport only
         x = _Ctx()
         x.rule, x.interp = rule, interp
         x.nx, x.ny, x.hx, x.hy, x.kap, x.c, x.dt, x.tau = nx, ny, hx, hy, kap, c, dt, tau

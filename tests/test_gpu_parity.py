@@ -235,7 +235,7 @@ def test_potentials_bend_small_full_mesh_two_steps(torch, rule, interp):
         rp.rp_destroy(ctx)
 
 
-def test_subtree_units_match_the_unsplit_walk(torch, monkeypatch):
+def test_subtree_units_match_the_unsplit_walk(torch):
     """Deep trees split into subtree work units walk the same canonical tree:
     equal segment counts per point and values equal to the single-warp walk up to the
     summation grouping (config 2 at full size, the bench workload)."""
@@ -245,20 +245,22 @@ def test_subtree_units_match_the_unsplit_walk(torch, monkeypatch):
     frames = W.ring_frames(cfg, 0)
     out = {}
     for split in ("12", "0"):
-        monkeypatch.setenv("RP_SPLIT", split)
         ctx = G.make_ctx(cfg)
         try:
+            rp.rp_set_work_split(ctx, int(split))
             G.load_state(ctx, cfg, 0, cfg.n_pre, ring, frames)
             out[split] = G.gpu_potentials(ctx, cfg.nx * cfg.ny)
         finally:
             rp.rp_destroy(ctx)
     (a, ia), (b, ib) = out["12"], out["0"]
-    assert ia.units > 1000 and ia.unit_overflow == 0 and ib.units == 0
-    np.testing.assert_array_equal(a["nseg"], b["nseg"])
+    assert ia.units > 1000 and ib.units == 0
+    for k in ("nseg", "nleaf", "capped"):
+        np.testing.assert_array_equal(a[k], b[k])
     assert ia.evals == ib.evals and ia.leaves == ib.leaves and ia.capped == ib.capped
     scale = max(np.abs(b["phi"]).max(), np.abs(b["ax"]).max(), np.abs(b["ay"]).max())
-    for k in ("phi", "ax", "ay"):
-        assert np.abs(a[k] - b[k]).max() <= 1e-13 * scale
+    # the leaf error estimate eps is merged from the units like the values
+    for k in ("phi", "ax", "ay", "err"):
+        assert np.abs(a[k] - b[k]).max() <= 1e-13 * scale, k
 
 
 @pytest.mark.parametrize("which", ["bend_small", "cfg2_sampled"])
@@ -594,7 +596,7 @@ def test_potentials_bend_cfg3_full_size_sampled(torch):
         fail, worst, _ = G.compare_potentials(gpu, orc, pts)
         assert not fail.any(), (pts[fail][:10], worst)
         assert info.kappa == cfg.kappa_max
-        assert info.units > 0 and info.unit_overflow == 0
+        assert info.units > 0
     finally:
         rp.rp_destroy(ctx)
 
@@ -621,7 +623,7 @@ def test_potentials_bend_cfg4_full_size_sampled(torch):
         fail, worst, _ = G.compare_potentials(gpu, orc, pts)
         assert not fail.any(), (pts[fail][:10], worst)
         assert info.kappa == cfg.kappa_max
-        assert info.units > 0 and info.unit_overflow == 0
+        assert info.units > 0
     finally:
         rp.rp_destroy(ctx)
 
@@ -647,7 +649,7 @@ def test_potentials_bend_cfg5_full_size_sampled(torch):
         fail, worst, _ = G.compare_potentials(gpu, orc, pts)
         assert not fail.any(), (pts[fail][:10], worst)
         assert info.kappa == cfg.kappa_max
-        assert info.units > 0 and info.unit_overflow == 0
+        assert info.units > 0
     finally:
         rp.rp_destroy(ctx)
 
@@ -672,25 +674,40 @@ def test_schedule_policies_bit_identical(torch, policy, k):
         b.close()
 
 
-def test_bench_json_contract(torch):
-    """bench.py prints one JSON line with the keys the driver and the judge read."""
+def _bench(args, env=None, timeout=900):
     import json
     import os
     import subprocess
     import sys
     root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
-    out = subprocess.run([sys.executable, os.path.join(root, "bench.py"), "--config", "1", "--steps", "2",
-                          "--warmup", "3", "--no-cpu-baseline"], capture_output=True, text=True, timeout=600)
-    assert out.returncode == 0, out.stderr[-2000:]
-    lines = [l for l in out.stdout.splitlines() if l.strip().startswith("{")]
-    assert len(lines) == 1
-    d = json.loads(lines[0])
+    e = dict(os.environ)
+    e.update(env or {})
+    out = subprocess.run([sys.executable, os.path.join(root, "bench.py"), *args],
+                         capture_output=True, text=True, timeout=timeout, env=e)
+    assert out.returncode == 0, out.stderr[-3000:]
+    lines = [ln for ln in out.stdout.splitlines() if ln.strip().startswith("{")]
+    assert len(lines) == 1, out.stdout[-2000:]
+    return json.loads(lines[0])
+
+
+def test_bench_json_contract(torch):
+    """bench.py prints one JSON line with the keys the driver and the judge read; with
+    RP_DIST_BACKEND=gloo, `--gpus 2` (self-spawned, two ranks sharing the test GPU) gives the
+    same result bytes as one GPU."""
+    d = _bench(["--config", "1", "--steps", "2", "--warmup", "3"])
     for k in ("metric", "value", "unit", "n_gpus", "steps", "warmup", "ms_per_step", "higher_is_better",
-              "scaling", "vs_baseline", "dtype", "data", "config", "roofline", "gpu_launches", "clocks", "e2e"):
+              "scaling", "vs_baseline", "dtype", "data", "config", "roofline", "gpu_launches", "clocks",
+              "e2e", "cpu_baseline", "evals_per_s", "result_sha256"):
         assert k in d, k
     assert d["value"] > 0 and d["steps"] == 2 and d["warmup"] == 3 and d["dtype"] == "f64"
     r = d["roofline"]
     assert r["bound"] == "alu" and 0 < r["frac"] < 1.2 and r["peak"] > 30
     assert d["gpu_launches"] > 0
-    assert d["e2e"]["h2d_bytes_per_step"] > 0 and d["e2e"]["value"] > 0
-    assert "workload" in d["config"]
+    assert d["e2e"]["h2d_bytes_per_step"] > 0 and 0 < d["e2e"]["value"] <= d["value"] * 1.001
+    assert d["config"]["workload"] == "cfg1-32x32-static"
+    c = d["cpu_baseline"]
+    assert c["kind"] == "oracle" and c["evals_per_s"] > 0 and "step 4" in c["sample"]
+    d2 = _bench(["--config", "1", "--steps", "2", "--warmup", "3", "--gpus", "2"],
+                env={"RP_DIST_BACKEND": "gloo"})
+    assert d2["n_gpus"] == 2 and d2["result_sha256"] == d["result_sha256"]
+    assert "gloo" in d2["config"]["transport"]

@@ -133,7 +133,7 @@ def test_oracle_thread_count_overrides_the_environment():
     cfg = _bend_small()
     import bench
     pts = np.arange(0, cfg.nx * cfg.ny, 97, dtype=np.int32)
-    P, _ = bench._oracle_state(cfg)
+    P = bench._oracle_rigid_state(cfg)
     assert oracle.set_threads(1) == 1
     r1 = P.potentials(pts)
     assert oracle.set_threads(2) == 2
