@@ -239,6 +239,14 @@ int rp_push_particles(rp_ctx* ctx, double* x, double* y, double* ux, double* uy,
                       double q_over_mc, double bz_ext, const double* ex, const double* ey,
                       const double* bz);
 
+/* Lorentz force per unit charge on n particles, F = E + beta x (B_z + bz_ext) z-hat (lab x, y
+ * components), from the same TSC gather of (E_x, E_y, B_z) on frame k as rp_push_particles
+ * (R-15): the particle-level forces F_i of the paper's validation (Fig. 2-3).
+ * beta = u / sqrt(1 + u^2).  fx, fy [n] DEVICE outputs. */
+int rp_particle_forces(rp_ctx* ctx, const double* x, const double* y, const double* ux,
+                       const double* uy, int64_t n, double bz_ext, const double* ex,
+                       const double* ey, const double* bz, double* fx, double* fy);
+
 /* One whole step through HOST buffers (end-to-end path).  With an rp_dist the host arrays
  * hold this rank's particle shard and the mesh outputs are the full mesh.  Copies the particles
  * host->device, runs deposit_step, compute_potentials, compute_fields (with the previous

@@ -112,6 +112,7 @@ def lib():
             "orc_integrand_at": (None, [P(Params), P(Hist), P(Source), i32, d, d, d, pd]),
             "orc_gk15_at": (None, [P(Params), P(Hist), P(Source), d, d, i32, d, d, pd, pd, pd]),
             "orc_fields": (None, [P(Params), P(Frame), P(Frame), pd, pd, pd, pd, pd, pd, pd, pd]),
+            "orc_forces": (None, [P(Params), P(Frame), i64, pd, pd, pd, pd, d, pd, pd, pd, pd, pd]),
             "orc_push": (None, [P(Params), P(Frame), i64, pd, pd, pd, pd, d, d, pd, pd, pd]),
         }
         for name, (res, args) in sig.items():
@@ -379,3 +380,14 @@ def push(nx, ny, hx, hy, c, dt, fk, x, y, ux, uy, q_over_mc, bz_ext, ex, ey, bz)
     lib().orc_push(C.byref(P), C.byref(frame(fk)), len(x), _pd(x), _pd(y), _pd(ux), _pd(uy),
                    q_over_mc, bz_ext, _pd(ex), _pd(ey), _pd(bz))
     return x, y, ux, uy
+
+
+def forces(nx, ny, hx, hy, fk, x, y, ux, uy, bz_ext, ex, ey, bz):
+    """Lorentz force per unit charge E + beta x B at each particle: (fx, fy)."""
+    P = Params(nx, ny, hx, hy, 1.0, 1.0, 1.0, 64, 30, 2, 1, 0)
+    x, y, ux, uy, ex, ey, bz = (np.ascontiguousarray(a, dtype=np.float64)
+                                for a in (x, y, ux, uy, ex, ey, bz))
+    fx, fy = np.zeros(len(x)), np.zeros(len(x))
+    lib().orc_forces(C.byref(P), C.byref(frame(fk)), len(x), _pd(x), _pd(y), _pd(ux), _pd(uy),
+                     bz_ext, _pd(ex), _pd(ey), _pd(bz), _pd(fx), _pd(fy))
+    return fx, fy

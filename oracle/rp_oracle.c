@@ -1009,3 +1009,32 @@ void orc_push(const orc_params* P, const orc_frame* Fk, int64_t n, double* x, do
     y[i] += P->c * P->dt * nuy / g;
   }
 }
+
+/* Lorentz force per unit charge on each particle (the particle-level force F_i of the paper's
+ * validation): F = E + beta x (B_z + B_ext) z-hat with (E, B_z) gathered at the
+ * particle by the push's TSC weights (R-15) and beta = u / gamma.
+ *   F_x = E_x + beta_y B_z,   F_y = E_y - beta_x B_z. */
+void orc_forces(const orc_params* P, const orc_frame* Fk, int64_t n, const double* x,
+                const double* y, const double* ux, const double* uy, double bz_ext,
+                const double* ex, const double* ey, const double* bz, double* fx, double* fy) {
+  for (int64_t i = 0; i < n; ++i) {
+    double u, v;
+    to_local(Fk, x[i], y[i], &u, &v);
+    double tx = u / P->hx, ty = v / P->hy;
+    double gx = floor(tx + 0.5), gy = floor(ty + 0.5);
+    double Ex = 0.0, Ey = 0.0, Bz = 0.0;
+    if (gx >= -2.0 && gx <= P->nx + 1.0 && gy >= -2.0 && gy <= P->ny + 1.0) {
+      double wx[3], wy[3];
+      orc_tsc_weights(tx - gx, wx);
+      orc_tsc_weights(ty - gy, wy);
+      int32_t ix = (int32_t)gx, iy = (int32_t)gy;
+      Ex = gather_tsc(P, ex, ix, iy, wx, wy);
+      Ey = gather_tsc(P, ey, ix, iy, wx, wy);
+      Bz = gather_tsc(P, bz, ix, iy, wx, wy);
+    }
+    Bz += bz_ext;
+    double g = sqrt(1.0 + ux[i] * ux[i] + uy[i] * uy[i]);
+    fx[i] = Ex + (uy[i] / g) * Bz;
+    fy[i] = Ey - (ux[i] / g) * Bz;
+  }
+}

@@ -42,7 +42,8 @@ def up_to_date() -> bool:
 
 def _compile(src: str) -> tuple[str, str]:
     obj = os.path.join(BUILD, os.path.basename(src).replace(".cu", ".o"))
-    cmd = [NVCC, *ARCH, *FLAGS, "-c", src, "-o", obj]
+    # RP_NVCC_EXTRA: extra nvcc flags for development builds of A/B variants (tools/variant.sh)
+    cmd = [NVCC, *ARCH, *FLAGS, *os.environ.get("RP_NVCC_EXTRA", "").split(), "-c", src, "-o", obj]
     p = subprocess.run(cmd, capture_output=True, text=True)
     if p.returncode != 0:
         raise RuntimeError(f"nvcc failed for {src}:\n{p.stderr}")

@@ -55,20 +55,20 @@ __device__ __forceinline__ void tsc(double d, double& wm, double& w0, double& wp
   wp = 0.5 * (b * b);
 }
 
-__global__ void k_push(int64_t n, double* __restrict__ x, double* __restrict__ y,
-                       double* __restrict__ ux, double* __restrict__ uy, rp_frame F, int nx,
-                       int ny, double inv_hx, double inv_hy, double c, double dt, double qmc,
-                       double bz_ext, const double* __restrict__ ex,
-                       const double* __restrict__ ey, const double* __restrict__ bz) {
-  int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
-  if (i >= n) return;
-  double X = x[i], Y = y[i];
+// TSC gather of (E_x, E_y, B_z) at lab point (X, Y) on frame F, with the deposition's weights
+// (R-15); nodes outside the grid contribute 0
+__device__ __forceinline__ void gather_eb(double X, double Y, const rp_frame& F, int nx, int ny,
+                                          double inv_hx, double inv_hy,
+                                          const double* __restrict__ ex,
+                                          const double* __restrict__ ey,
+                                          const double* __restrict__ bz, double& Ex, double& Ey,
+                                          double& Bz) {
   double dx = X - F.ox, dy = Y - F.oy;
   double u = F.cos_psi * dx + F.sin_psi * dy;
   double v = F.cos_psi * dy - F.sin_psi * dx;
   double tx = u * inv_hx, ty = v * inv_hy;
   double fx = floor(tx + 0.5), fy = floor(ty + 0.5);
-  double Ex = 0.0, Ey = 0.0, Bz = 0.0;
+  Ex = 0.0; Ey = 0.0; Bz = 0.0;
   if (fx >= -2.0 && fx <= nx + 1.0 && fy >= -2.0 && fy <= ny + 1.0) {
     double wx[3], wy[3];
     tsc(tx - fx, wx[0], wx[1], wx[2]);
@@ -90,6 +90,37 @@ __global__ void k_push(int64_t n, double* __restrict__ x, double* __restrict__ y
       }
     }
   }
+}
+
+// Lorentz force per unit charge on each particle, F = E + beta x (B_z + B_ext) z-hat, from the
+// push's gather: the particle-level force of the paper's validation
+__global__ void k_forces(int64_t n, const double* __restrict__ x, const double* __restrict__ y,
+                         const double* __restrict__ ux, const double* __restrict__ uy, rp_frame F,
+                         int nx, int ny, double inv_hx, double inv_hy, double bz_ext,
+                         const double* __restrict__ ex, const double* __restrict__ ey,
+                         const double* __restrict__ bz, double* __restrict__ fx,
+                         double* __restrict__ fy) {
+  int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+  if (i >= n) return;
+  double Ex, Ey, Bz;
+  gather_eb(x[i], y[i], F, nx, ny, inv_hx, inv_hy, ex, ey, bz, Ex, Ey, Bz);
+  Bz += bz_ext;
+  const double a = ux[i], b = uy[i];
+  const double g = sqrt(1.0 + a * a + b * b);
+  fx[i] = Ex + (b / g) * Bz;
+  fy[i] = Ey - (a / g) * Bz;
+}
+
+__global__ void k_push(int64_t n, double* __restrict__ x, double* __restrict__ y,
+                       double* __restrict__ ux, double* __restrict__ uy, rp_frame F, int nx,
+                       int ny, double inv_hx, double inv_hy, double c, double dt, double qmc,
+                       double bz_ext, const double* __restrict__ ex,
+                       const double* __restrict__ ey, const double* __restrict__ bz) {
+  int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+  if (i >= n) return;
+  double X = x[i], Y = y[i];
+  double Ex, Ey, Bz;
+  gather_eb(X, Y, F, nx, ny, inv_hx, inv_hy, ex, ey, bz, Ex, Ey, Bz);
   Bz += bz_ext;
   double h = 0.5 * qmc * dt;
   double umx = ux[i] + h * Ex, umy = uy[i] + h * Ey;
@@ -137,6 +168,23 @@ int rp_push_impl(rp_ctx* ctx, double* x, double* y, double* ux, double* uy, int6
   k_push<<<(unsigned)((n + 255) / 256), 256, 0, ctx->stream>>>(n, x, y, ux, uy, Fk, c.nx, c.ny,
                                                                 1.0 / c.hx, 1.0 / c.hy, c.c, c.dt,
                                                                 qmc, bz_ext, ex, ey, bz);
+  RP_CHECK_LAUNCH();
+  return RP_OK;
+}
+
+int rp_forces_impl(rp_ctx* ctx, const double* x, const double* y, const double* ux,
+                   const double* uy, int64_t n, double bz_ext, const double* ex, const double* ey,
+                   const double* bz, double* fx, double* fy) {
+  const rp_config& c = ctx->cfg;
+  if (ctx->k < 0) return rp_fail(ctx, RP_ESTATE, "forces before the first deposit");
+  if (n < 0) return rp_fail(ctx, RP_EINVAL, "forces: n < 0");
+  if (n == 0) return RP_OK;
+  if (!x || !y || !ux || !uy || !ex || !ey || !bz || !fx || !fy)
+    return rp_fail(ctx, RP_EINVAL, "forces: null array");
+  rp_frame Fk = ctx->fh[slot_of(ctx->k, ctx->H)];
+  k_forces<<<(unsigned)((n + 255) / 256), 256, 0, ctx->stream>>>(n, x, y, ux, uy, Fk, c.nx, c.ny,
+                                                                  1.0 / c.hx, 1.0 / c.hy, bz_ext,
+                                                                  ex, ey, bz, fx, fy);
   RP_CHECK_LAUNCH();
   return RP_OK;
 }

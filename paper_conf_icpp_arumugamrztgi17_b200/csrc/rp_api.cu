@@ -421,6 +421,13 @@ int rp_push_particles(rp_ctx* ctx, double* x, double* y, double* ux, double* uy,
   return rp_push_impl(ctx, x, y, ux, uy, n, q_over_mc, bz_ext, ex, ey, bz);
 }
 
+int rp_particle_forces(rp_ctx* ctx, const double* x, const double* y, const double* ux,
+                       const double* uy, int64_t n, double bz_ext, const double* ex,
+                       const double* ey, const double* bz, double* fx, double* fy) {
+  RP_ENTER(ctx);
+  return rp_forces_impl(ctx, x, y, ux, uy, n, bz_ext, ex, ey, bz, fx, fy);
+}
+
 int rp_step_host(rp_ctx* ctx, double* xh, double* yh, double* uxh, double* uyh, int64_t n,
                  double q, const rp_frame* frame_k, double q_over_mc, double bz_ext,
                  double* mesh_host, rp_potential_info* info) {

@@ -237,6 +237,9 @@ int rp_fields_impl(rp_ctx* ctx, const double* phi, const double* ax, const doubl
 int rp_push_impl(rp_ctx* ctx, double* x, double* y, double* ux, double* uy, int64_t n,
                  double qmc, double bz_ext, const double* ex, const double* ey,
                  const double* bz);
+int rp_forces_impl(rp_ctx* ctx, const double* x, const double* y, const double* ux,
+                   const double* uy, int64_t n, double bz_ext, const double* ex, const double* ey,
+                   const double* bz, double* fx, double* fy);
 int rp_scatter_impl(rp_ctx* ctx, const double* shards, int32_t world, int64_t cap,
                     double* phi, double* ax, double* ay, double* err, int32_t* nseg);
 int rp_alloc_potential_scratch(rp_ctx* ctx);

@@ -61,6 +61,9 @@ class rp_potential_info(C.Structure):
                 ("items", C.c_int64), ("max_level", C.c_int32), ("kappa", C.c_int32),
                 ("skipped", C.c_int64), ("units", C.c_int64)]
 
+    def as_dict(self) -> dict:
+        return {k: getattr(self, k) for k, _ in self._fields_}
+
 
 RP_NCCL_ID_BYTES = 128
 
@@ -117,6 +120,7 @@ _SIG = {
     "rp_shard_scatter": (C.c_int, [_vp, _vp, _i32, _i64, _vp, _vp, _vp, _vp, _vp]),
     "rp_compute_fields": (C.c_int, [_vp, _vp, _vp, _vp, _vp, _vp, _vp, _vp, _vp]),
     "rp_push_particles": (C.c_int, [_vp, _vp, _vp, _vp, _vp, _i64, _d, _d, _vp, _vp, _vp]),
+    "rp_particle_forces": (C.c_int, [_vp, _vp, _vp, _vp, _vp, _i64, _d, _vp, _vp, _vp, _vp, _vp]),
     "rp_step_host": (C.c_int, [_vp, _vp, _vp, _vp, _vp, _i64, _d, _P(rp_frame), _d, _d, _vp,
                                _P(rp_potential_info)]),
     "rp_load_state": (C.c_int, [_vp, _i32, _i32, _P(rp_frame), _vp]),
@@ -353,6 +357,13 @@ def rp_push_particles(ctx, x, y, ux, uy, q_over_mc, bz_ext, ex, ey, bz) -> None:
     _check(_lib.rp_push_particles(ctx, _f64(x), _f64(y), _f64(ux), _f64(uy), x.numel(),
                                   float(q_over_mc), float(bz_ext), _f64(ex), _f64(ey), _f64(bz)),
            ctx, "rp_push_particles")
+
+
+def rp_particle_forces(ctx, x, y, ux, uy, bz_ext, ex, ey, bz, fx, fy) -> None:
+    _check(_lib.rp_particle_forces(ctx, _f64(x, "x"), _f64(y, "y"), _f64(ux, "ux"), _f64(uy, "uy"),
+                                   x.numel(), float(bz_ext), _f64(ex, "ex"), _f64(ey, "ey"),
+                                   _f64(bz, "bz"), _f64(fx, "fx"), _f64(fy, "fy")), ctx,
+           "rp_particle_forces")
 
 
 def rp_step_host(ctx, x, y, ux, uy, q, frame_k, q_over_mc, bz_ext, mesh_out, info=False):

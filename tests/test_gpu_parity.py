@@ -466,6 +466,31 @@ def test_push_parity(torch):
         rp.rp_destroy(ctx)
 
 
+def test_particle_forces_parity(torch):
+    """rp_particle_forces (E + beta x B gathered at the particles) against orc_forces, the
+    particle-level force of the paper's validation; 1e-13 relative."""
+    from paper_conf_icpp_arumugamrztgi17_b200 import rp
+    cfg = W.config(2)
+    x, y, ux, uy = W.particles(cfg, n=200_000, seed=3)
+    rng = np.random.default_rng(6)
+    npts = cfg.nx * cfg.ny
+    ex, ey, bz = (1e3 * rng.standard_normal(npts) for _ in range(3))
+    fk = W.frame(cfg, 0)
+    want = oracle.forces(cfg.nx, cfg.ny, cfg.hx, cfg.hy, fk, x, y, ux, uy, cfg.bz_ext, ex, ey, bz)
+    ctx = G.make_ctx(cfg)
+    try:
+        ring = np.zeros((cfg.H, cfg.ny, cfg.nx, 4))
+        G.load_state(ctx, cfg, 0, 0, ring, W.ring_frames(cfg, 0))
+        xd, yd, uxd, uyd, exd, eyd, bzd = _dev_arrays(torch, x, y, ux, uy, ex, ey, bz)
+        fx, fy = (torch.zeros(len(x), dtype=torch.float64, device="cuda") for _ in range(2))
+        rp.rp_particle_forces(ctx, xd, yd, uxd, uyd, cfg.bz_ext, exd, eyd, bzd, fx, fy)
+        for g, w in zip((fx, fy), want):
+            g = g.cpu().numpy()
+            assert np.abs(g - w).max() <= 1e-13 * np.abs(w).max()
+    finally:
+        rp.rp_destroy(ctx)
+
+
 # ------------------------------------------------------------------ sharding, e2e, loop
 def test_shard_path_equals_full_mesh(torch):
     """Mesh-point sharding simulated on one GPU: ranks 0..W-1 each compute

@@ -139,3 +139,50 @@ def test_push_uniform_E_acceleration():
     assert abs(ux2[0] - (0.1 + 2.0 * 0.5 * 0.2)) < 1e-15
     g = math.sqrt(1 + ux2[0] ** 2)
     assert abs(x2[0] - (3.2 + 0.2 * ux2[0] / g)) < 1e-15
+
+
+def test_particle_forces_uniform_and_linear_fields():
+    """orc_forces (the particle-level force of the validation): with uniform fields
+    F = E + beta x B exactly (q > 0, beta along x, B_z > 0 pushes towards -y); with E_x linear
+    in the frame coordinate u the TSC gather reproduces it exactly at the particle (TSC weights
+    reproduce linear functions), on a rotated frame."""
+    nx, ny, h = 10, 9, 0.5
+    psi = 0.7
+    fk = (1.0, -2.0, math.cos(psi), math.sin(psi))
+    rng = np.random.default_rng(4)
+    u = rng.uniform(2 * h, (nx - 3) * h, 50)
+    v = rng.uniform(2 * h, (ny - 3) * h, 50)
+    x = fk[0] + u * fk[2] - v * fk[3]
+    y = fk[1] + u * fk[3] + v * fk[2]
+    ux, uy = rng.normal(0, 2, 50), rng.normal(0, 2, 50)
+    g = np.sqrt(1 + ux ** 2 + uy ** 2)
+    E0x, E0y, B0 = 0.3, -0.2, 0.7
+    ones = np.ones((ny, nx))
+    fx, fy = oracle.forces(nx, ny, h, h, fk, x, y, ux, uy, 0.25, E0x * ones, E0y * ones, B0 * ones)
+    np.testing.assert_allclose(fx, E0x + uy / g * (B0 + 0.25), rtol=0, atol=1e-14)
+    np.testing.assert_allclose(fy, E0y - ux / g * (B0 + 0.25), rtol=0, atol=1e-14)
+    # beta = +x, B_z > 0: F_y = -beta B (q v x B with z-hat B)
+    fx1, fy1 = oracle.forces(nx, ny, h, h, fk, x[:1], y[:1], [1e6], [0.0], 0.0, 0 * ones, 0 * ones, ones)
+    assert abs(fx1[0]) < 1e-12 and abs(fy1[0] + 1.0) < 1e-9
+    # E_x = a + b * u_node on the rotated mesh: exact at the particle's own u
+    U = np.arange(nx)[None, :] * h * np.ones((ny, 1))
+    z = np.zeros((ny, nx))
+    fx, fy = oracle.forces(nx, ny, h, h, fk, x, y, np.zeros(50), np.zeros(50), 0.0, 0.4 + 1.3 * U, z, z)
+    np.testing.assert_allclose(fx, 0.4 + 1.3 * u, rtol=0, atol=1e-13)
+    assert np.all(fy == 0)
+
+
+def test_particle_forces_are_the_first_order_boris_kick():
+    """The push's momentum change over a small step is q/mc dt times the force (first order in
+    q/mc dt): ties orc_forces to orc_push through an independent route."""
+    nx = ny = 8
+    rng = np.random.default_rng(5)
+    ex, ey, bz = (rng.normal(0, 1, (ny, nx)) for _ in range(3))
+    x, y = rng.uniform(2, 5, 20), rng.uniform(2, 5, 20)
+    ux, uy = rng.normal(0, 1, 20), rng.normal(0, 1, 20)
+    fk = (0.0, 0.0, 1.0, 0.0)
+    fx, fy = oracle.forces(nx, ny, 1.0, 1.0, fk, x, y, ux, uy, 0.3, ex, ey, bz)
+    qmc, dt = 1e-6, 1e-3
+    _, _, ux2, uy2 = oracle.push(nx, ny, 1.0, 1.0, 1.0, dt, fk, x, y, ux, uy, qmc, 0.3, ex, ey, bz)
+    np.testing.assert_allclose((ux2 - ux) / (qmc * dt), fx, rtol=1e-6, atol=1e-7)
+    np.testing.assert_allclose((uy2 - uy) / (qmc * dt), fy, rtol=1e-6, atol=1e-7)
