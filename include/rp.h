@@ -222,15 +222,17 @@ int64_t rp_shard_capacity(const rp_ctx* ctx, int32_t world);
 int rp_shard_scatter(rp_ctx* ctx, const double* shards, int32_t world, int64_t cap,
                      double* phi, double* ax, double* ay, double* err, int32_t* nseg);
 
-/* Self-fields on mesh k (R-15): second-order central differences (one-sided at the
- * edges) in frame coordinates rotated to the lab;
- *   E = -grad phi - (1/c) dA/dt,  dA/dt = (A_k - A_{k-1})/dt - (V.grad) A_k,
- *   V = node velocity (P_k - P_{k-1})/dt;  B_z = d_x A_y - d_y A_x.
- * ax_prev / ay_prev (step k-1 on its own mesh) may both be NULL: dA/dt is then 0.
- * All arrays [ny*nx]. */
+/* Self-fields on mesh k (R-15, R-15b): second-order central differences (one-sided at
+ * the edges) in frame coordinates rotated to the lab;
+ *   E = -grad phi - (1/c) dA/dt,  B_z = d_x A_y - d_y A_x,
+ *   dA/dt = (1/dt) sum_j BD_j A_{k-j} - (V . grad) A_k,  V = (1/dt) sum_j BD_j P_{k-j},
+ * consistent order-m backward differences at t_k of the node values and of the node position
+ * on the frames of levels k .. k-m (exact for a field at rest in the lab, O(dt^m) for one
+ * co-moving with the mesh).  a_prev: DEVICE [n_prev][2][ny*nx], (A_x, A_y) of steps k-1, ...,
+ * k-n_prev (most recent first); n_prev = 0..4 (0: dA/dt omitted); m = n_prev, lowered when the
+ * ring holds fewer frames.  All other arrays [ny*nx].  EINVAL on n_prev outside 0..4. */
 int rp_compute_fields(rp_ctx* ctx, const double* phi, const double* ax, const double* ay,
-                      const double* ax_prev, const double* ay_prev, double* ex, double* ey,
-                      double* bz);
+                      const double* a_prev, int32_t n_prev, double* ex, double* ey, double* bz);
 
 /* Relativistic Boris leap-frog push by dt (R-15) of n particles in place:
  * TSC gather of (E_x, E_y, B_z) on frame k (same weights as deposition), plus a uniform
@@ -247,10 +249,21 @@ int rp_particle_forces(rp_ctx* ctx, const double* x, const double* y, const doub
                        const double* uy, int64_t n, double bz_ext, const double* ex,
                        const double* ey, const double* bz, double* fx, double* fy);
 
+/* Time-centred momenta for the deposit's current (R-27): the leap-frog momenta u (at
+ * t_k - dt/2) advanced by frac * dt in the uniform external B_z = bz_ext (the Boris
+ * rotation of rp_push_particles with E = 0), written to ux_out / uy_out [n] (DEVICE; may alias
+ * the inputs).  The loop deposits with frac = 1/2 so the current of step k is rho v(t_k); a
+ * current half a step behind the bunch's motion is misaligned by half the step's bend angle,
+ * which swamps the CSR force (a 1e-4 residual of space-charge-sized terms). */
+int rp_kick_external(rp_ctx* ctx, const double* ux, const double* uy, int64_t n,
+                     double q_over_mc, double bz_ext, double frac, double* ux_out,
+                     double* uy_out);
+
 /* One whole step through HOST buffers (end-to-end path).  With an rp_dist the host arrays
  * hold this rank's particle shard and the mesh outputs are the full mesh.  Copies the particles
- * host->device, runs deposit_step, compute_potentials, compute_fields (with the previous
- * step's A kept by the context), push, and copies the pushed particles and the six mesh
+ * host->device, runs kick_external (frac 1/2) + deposit_step, compute_potentials,
+ * compute_fields (with the previous
+ * steps' A kept by the context, up to 4), push, and copies the pushed particles and the six mesh
  * outputs back.  x_host .. uy_host are updated in place; mesh_host is [6][ny*nx]
  * (phi, ax, ay, ex, ey, bz).  Pinned host memory gives full-bandwidth copies.  info
  * (nullable) receives the potentials' work counters.  Syncs. */

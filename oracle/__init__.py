@@ -111,7 +111,8 @@ def lib():
             "orc_inner_at": (i64, [P(Params), P(Hist), P(Source), d, d, i32, d, pd]),
             "orc_integrand_at": (None, [P(Params), P(Hist), P(Source), i32, d, d, d, pd]),
             "orc_gk15_at": (None, [P(Params), P(Hist), P(Source), d, d, i32, d, d, pd, pd, pd]),
-            "orc_fields": (None, [P(Params), P(Frame), P(Frame), pd, pd, pd, pd, pd, pd, pd, pd]),
+            "orc_fields": (None, [P(Params), P(Frame), i32, pd, pd, pd, pd, pd, pd, pd]),
+            "orc_kick_external": (None, [P(Params), i64, pd, pd, d, d, d, pd, pd]),
             "orc_forces": (None, [P(Params), P(Frame), i64, pd, pd, pd, pd, d, pd, pd, pd, pd, pd]),
             "orc_push": (None, [P(Params), P(Frame), i64, pd, pd, pd, pd, d, d, pd, pd, pd]),
         }
@@ -359,16 +360,22 @@ def arcs_disk(cu, cv, r, x0, y0, a):
     return n, out[: 2 * max(n, 0)].reshape(-1, 2)
 
 
-def fields(nx, ny, hx, hy, c, dt, fk, fkm1, phi, ax, ay, ax_prev=None, ay_prev=None):
+def fields(nx, ny, hx, hy, c, dt, frames, phi, ax, ay, a_prev=()):
+    """frames: of levels k, k-1, ..., k-m; a_prev: the m previous (A_x, A_y) pairs, most recent
+    first (m <= 4; order-m backward differences, R-15b).  m = 0: no dA/dt term."""
     P = Params(nx, ny, hx, hy, c, dt, 1.0, 64, 30, 2, 1, 0)
     phi, ax, ay = (np.ascontiguousarray(a, dtype=np.float64) for a in (phi, ax, ay))
-    if ax_prev is not None:
-        ax_prev = np.ascontiguousarray(ax_prev, dtype=np.float64)
-        ay_prev = np.ascontiguousarray(ay_prev, dtype=np.float64)
+    m = len(a_prev)
+    fr = np.asarray(frames, dtype=np.float64).reshape(-1, 4)
+    assert m <= 4 and len(fr) >= m + 1
+    fa = (Frame * len(fr))(*[frame(f) for f in fr])
+    prev = None
+    if m:
+        prev = np.ascontiguousarray(np.stack([np.stack([np.ravel(a), np.ravel(b)]) for a, b in a_prev]),
+                                    dtype=np.float64)
     ex, ey, bz = np.zeros_like(phi), np.zeros_like(phi), np.zeros_like(phi)
-    fm = C.byref(frame(fkm1)) if fkm1 is not None else None
-    lib().orc_fields(C.byref(P), C.byref(frame(fk)), fm, _pd(phi), _pd(ax), _pd(ay),
-                     _pd(ax_prev), _pd(ay_prev), _pd(ex), _pd(ey), _pd(bz))
+    lib().orc_fields(C.byref(P), fa, m, _pd(phi), _pd(ax), _pd(ay), _pd(prev), _pd(ex), _pd(ey),
+                     _pd(bz))
     return ex, ey, bz
 
 
@@ -391,3 +398,13 @@ def forces(nx, ny, hx, hy, fk, x, y, ux, uy, bz_ext, ex, ey, bz):
     lib().orc_forces(C.byref(P), C.byref(frame(fk)), len(x), _pd(x), _pd(y), _pd(ux), _pd(uy),
                      bz_ext, _pd(ex), _pd(ey), _pd(bz), _pd(fx), _pd(fy))
     return fx, fy
+
+
+def kick_external(dt, ux, uy, q_over_mc, bz_ext, frac=0.5):
+    """Momenta advanced by frac * dt in the uniform external B_z (R-27): (ux, uy)."""
+    P = Params(4, 4, 1.0, 1.0, 1.0, dt, 1.0, 64, 30, 2, 1, 0)
+    ux, uy = (np.ascontiguousarray(a, dtype=np.float64) for a in (ux, uy))
+    ox, oy = np.zeros(len(ux)), np.zeros(len(ux))
+    lib().orc_kick_external(C.byref(P), len(ux), _pd(ux), _pd(uy), q_over_mc, bz_ext, frac,
+                            _pd(ox), _pd(oy))
+    return ox, oy

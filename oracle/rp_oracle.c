@@ -925,13 +925,29 @@ static double d_dir(const double* f, int32_t nx, int32_t ny, int32_t ix, int32_t
 #undef AT
 }
 
-/* E = -grad(phi) - (1/c) dA/dt ,  B_z = d_x A_y - d_y A_x  on mesh k.
- * dA/dt|lab = (A_k - A_{k-1})/dt - (V . grad) A_k with V the node velocity
- * (P_k - P_{k-1})/dt; omitted when ax_prev/ay_prev are NULL. */
-void orc_fields(const orc_params* P, const orc_frame* Fk, const orc_frame* Fkm1,
-                const double* phi, const double* ax, const double* ay, const double* ax_prev,
-                const double* ay_prev, double* ex, double* ey, double* bz) {
+/* Backward-difference weights of order m = 1..4 for f'(t_k) from f(t_k), ..., f(t_{k-m}),
+ * in units of 1/dt (exact for polynomials of degree m; R-15b). */
+static const double BD[5][5] = {{0, 0, 0, 0, 0},
+                                {1.0, -1.0, 0, 0, 0},
+                                {1.5, -2.0, 0.5, 0, 0},
+                                {11.0 / 6.0, -3.0, 1.5, -1.0 / 3.0, 0},
+                                {25.0 / 12.0, -4.0, 3.0, -4.0 / 3.0, 0.25}};
+
+/* E = -grad(phi) - (1/c) dA/dt ,  B_z = d_x A_y - d_y A_x  on mesh k (R-15b).
+ * The mesh moves with its frame, so the lab time derivative at a node is the derivative
+ * following the node minus the convective term:
+ *   dA/dt|lab = (1/dt) sum_j BD[m][j] A_{k-j}(node)  -  (V . grad) A_k,
+ *   V = (1/dt) sum_j BD[m][j] P_{k-j}(node),
+ * both order-m backward differences at t_k (j = 0..m) on the same nodes, so a field at rest in
+ * the lab cancels exactly and one co-moving with the mesh is exact to O(dt^m).
+ * fr[0..m]: frames of levels k, k-1, ..., k-m; a_prev [m][2][ny*nx]: (A_x, A_y) of steps
+ * k-1, ..., k-m (most recent first); m = 0 omits the dA/dt term. */
+void orc_fields(const orc_params* P, const orc_frame* fr, int32_t m, const double* phi,
+                const double* ax, const double* ay, const double* a_prev, double* ex, double* ey,
+                double* bz) {
   const int32_t nx = P->nx, ny = P->ny;
+  const int64_t npts = (int64_t)nx * ny;
+  const orc_frame* Fk = fr;
   for (int32_t iy = 0; iy < ny; ++iy)
     for (int32_t ix = 0; ix < nx; ++ix) {
       int64_t id = (int64_t)iy * nx + ix;
@@ -943,13 +959,20 @@ void orc_fields(const orc_params* P, const orc_frame* Fk, const orc_frame* Fkm1,
       double axx = c * xu - s * xv, axy = s * xu + c * xv; /* d_x A_x, d_y A_x */
       double ayx = c * yu - s * yv, ayy = s * yu + c * yv; /* d_x A_y, d_y A_y */
       double dax = 0.0, day = 0.0;
-      if (ax_prev && ay_prev && Fkm1) {
-        double pxk, pyk, pxm, pym;
-        orc_mesh_point(P, Fk, ix, iy, &pxk, &pyk);
-        orc_mesh_point(P, Fkm1, ix, iy, &pxm, &pym);
-        double vx = (pxk - pxm) / P->dt, vy = (pyk - pym) / P->dt;
-        dax = (ax[id] - ax_prev[id]) / P->dt - (vx * axx + vy * axy);
-        day = (ay[id] - ay_prev[id]) / P->dt - (vx * ayx + vy * ayy);
+      if (a_prev && m >= 1) {
+        double vx = 0.0, vy = 0.0, nax = BD[m][0] * ax[id], nay = BD[m][0] * ay[id];
+        for (int32_t j = 0; j <= m; ++j) {
+          double px, py;
+          orc_mesh_point(P, fr + j, ix, iy, &px, &py);
+          vx += BD[m][j] * px;
+          vy += BD[m][j] * py;
+          if (j >= 1) {
+            nax += BD[m][j] * a_prev[(int64_t)(j - 1) * 2 * npts + id];
+            nay += BD[m][j] * a_prev[(int64_t)(j - 1) * 2 * npts + npts + id];
+          }
+        }
+        dax = (nax - (vx * axx + vy * axy)) / P->dt;
+        day = (nay - (vx * ayx + vy * ayy)) / P->dt;
       }
       ex[id] = -phx - dax / P->c;
       ey[id] = -phy - day / P->c;
@@ -1007,6 +1030,25 @@ void orc_push(const orc_params* P, const orc_frame* Fk, int64_t n, double* x, do
     uy[i] = nuy;
     x[i] += P->c * P->dt * nux / g;
     y[i] += P->c * P->dt * nuy / g;
+  }
+}
+
+/* Time-centred momenta for the current (R-27): the leap-frog momenta live at t_k - dt/2 (P:60,
+ * R-21), the current of step k at t_k, so the loop deposits u advanced by frac * dt in the
+ * uniform external B_z -- the Boris rotation of orc_push with E = 0 and step frac * dt (the
+ * self-field part of that half step is below 1e-6 relative in the bend and the previous step's
+ * fields live on the previous mesh, which the bunch has left; it is not included). */
+void orc_kick_external(const orc_params* P, int64_t n, const double* ux, const double* uy,
+                       double q_over_mc, double bz_ext, double frac, double* ux_out,
+                       double* uy_out) {
+  for (int64_t i = 0; i < n; ++i) {
+    double h = 0.5 * q_over_mc * (frac * P->dt);
+    double gm = sqrt(1.0 + ux[i] * ux[i] + uy[i] * uy[i]);
+    double t = h * bz_ext / gm;
+    double sr = 2.0 * t / (1.0 + t * t);
+    double upx = ux[i] + uy[i] * t, upy = uy[i] - ux[i] * t;
+    ux_out[i] = ux[i] + upy * sr;
+    uy_out[i] = uy[i] - upx * sr;
   }
 }
 

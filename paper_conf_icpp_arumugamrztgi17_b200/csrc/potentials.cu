@@ -46,6 +46,7 @@ enum : int { C_ITEMS = 0, C_NEXT = 1, C_EVALS = 2, C_SEGS = 3, C_LEAVES = 4, C_C
              C_TIES = 6, C_MAXLEV = 7, C_NODES = 8, C_NOUT = 9, C_SKIP = 10, C_UNITS = 11,
              C_NEXT_U = 12, C_COUNT = 16 };
 constexpr int kUnitShift = 20;  // unit key = item << 20 | index of the subtree root at its level
+constexpr int kGridVar = 4;  // grid evaluation loop: software-pipelined rounds (6 = Lagrange-3)
 constexpr int kUnitBudget = 64;  // subtree units per near-field item (DFS order)
 constexpr uint32_t kEmptyKey = 0xFFFFFFFFu;  // schedule key of an item without support
 
@@ -312,6 +313,9 @@ __constant__ double c_pio2[3] = {0.63661977236758134308, 1.5707963267948965580,
                                  6.1232339957367658e-17};  // 2/pi, pi/2 = hi + lo
 
 __device__ __forceinline__ void sincos_b(double x, double* s, double* c) {
+#ifdef RP_EXP_CHEAPSINCOS  // development timing experiment: wrong results
+  { const double z = x * x; *s = x * (1.0 - z * 0.16666); *c = 1.0 - 0.5 * z; return; }
+#endif
   const double k = rint(x * c_pio2[0]);
   double r = fma(-k, c_pio2[1], x);
   r = fma(-k, c_pio2[2], r);
@@ -519,9 +523,10 @@ __device__ __forceinline__ Geo geom_point(const Params& P, const WarpSmem& S, do
   const double fx = floor(tx + 0.5), fy = floor(ty + 0.5);
   const int ix = min(max(__double2int_rz(fx), -2), P.nx + 1);
   const int iy = min(max(__double2int_rz(fy), -2), P.ny + 1);
+  // a slot the node does not have evaluates slot 0's (finite) point with weight 0 and no refill
   Geo g;
-  g.dx = valid ? tx - fx : 0.0;
-  g.dy = valid ? ty - fy : 0.0;
+  g.dx = tx - fx;
+  g.dy = ty - fy;
   g.w = valid ? (LAG ? w : 0.25 * w) : 0.0;  // 0.25 undoes the 2 x 2 scaling of the TSC weights
   g.cell = valid ? (iy - 1) * P.PX + (ix - 1) : kNoCell;
   return g;
@@ -584,7 +589,8 @@ __device__ __forceinline__ void pipelined_round(const Item& it, const Params& P,
                                                 int nn, int N, double wfull, double third,
                                                 double (&st)[3][9][3], int& ccell, double& k0,
                                                 double& k1, double& k2, double& g0, double& g1,
-                                                double& g2, unsigned fullmask) {
+                                                double& g2, unsigned fullmask,
+                                                unsigned gmask) {
   const size_t rs = (size_t)4 * P.PX;
   const float inv_n1 = 1.0f / (float)(N - 1);  // arc slots per arc (R-24, R-25b)
   const double2 trf = __ldg(trig_full + (e < N ? e : 0));
@@ -592,7 +598,11 @@ __device__ __forceinline__ void pipelined_round(const Item& it, const Params& P,
                         : geom_point<false, LAG>(P, S, trf, e, 0, N, wfull, third, inv_n1);
 #pragma unroll 1
   for (int n = 0; n < nn; ++n) {
+#ifdef RP_EXP_NOREFILL  // development timing experiment: wrong results
+    if (cur.cell != kNoCell && ccell == kNoCell) {
+#else
     if (cur.cell != kNoCell && cur.cell != ccell) {
+#endif
       ccell = cur.cell;
       refill(it, rs, cur.cell, st);
     }
@@ -611,7 +621,7 @@ __device__ __forceinline__ void pipelined_round(const Item& it, const Params& P,
     }
     const double wk = cur.w * nd.wk;
     k0 += wk * f0; k1 += wk * f1; k2 += wk * f2;
-    if ((n & 1) || P.rule == RP_RULE_SIMPSON) {  // G7: Gauss nodes only (warp-uniform n)
+    if ((gmask >> n) & 1) {  // G7: Gauss nodes only (warp-uniform n)
       const double wg = cur.w * nd.wg;
       g0 += wg * f0; g1 += wg * f1; g2 += wg * f2;
     }
@@ -643,8 +653,9 @@ __global__ void __launch_bounds__(32 * kWarps) k_integrate(
     const double2* __restrict__ trig_full, double4* __restrict__ item_val,
     int4* __restrict__ item_cnt, uint2* __restrict__ item_aux,
     unsigned long long* __restrict__ counters) {
-  extern __shared__ __align__(16) unsigned char smem_raw[];
-  WarpSmem* smem = reinterpret_cast<WarpSmem*>(smem_raw);
+  // one warp per CTA: its per-item block is a static shared variable (a fixed shared address,
+  // no per-access window arithmetic)
+  __shared__ WarpSmem smem[kWarps];
   const int lane = threadIdx.x & 31;
   WarpSmem& S = smem[kWarps == 1 ? 0 : (threadIdx.x >> 5)];
   const unsigned long long n_items = counters[UNIT ? C_UNITS : C_ITEMS];
@@ -769,14 +780,16 @@ __global__ void __launch_bounds__(32 * kWarps) k_integrate(
       // (radially adjacent) segment.  Grid path: whole rounds (arc end nodes skipped, R-24: at
       // most 2 idle slots per arc); analytic sources: full rounds, then the leftover slots of
       // 65-node arcs as (slot, node) units.
+      // r' nodes that carry a G7 (or Simpson) weight: all five Simpson nodes, else the odd GK15
+      // nodes (the Gauss nodes; warp-uniform, kept in a register instead of re-reading P.rule)
+      const unsigned gmask = P.rule == RP_RULE_SIMPSON ? 0x1Fu : 0x2AAAu;
       const int rounds = (KIND == RP_SRC_GRID && VAR >= 4) ? (emax + 31) >> 5 : emax >> 5;
       const int left = (KIND == RP_SRC_GRID && VAR >= 4) ? 0 : emax - 32 * rounds;
       if (KIND == RP_SRC_GRID && VAR >= 4) {
         for (int rr = 0; rr < rounds; ++rr) {
           const int r = (nseg & 1) ? rounds - 1 - rr : rr;
-          pipelined_round<VAR == 6>(it, P, S, trig_full, 32 * r + lane, nn, N,
-                                                   wfull, third, st, ccell, k0, k1, k2, g0, g1,
-                                                   g2, fullmask);
+          pipelined_round<VAR == 6>(it, P, S, trig_full, 32 * r + lane, nn, N, wfull, third, st,
+                                    ccell, k0, k1, k2, g0, g1, g2, fullmask, gmask);
         }
       } else {
         for (int rr = 0; rr < rounds; ++rr) {
@@ -1071,7 +1084,7 @@ static int launch_integrate_one(rp_ctx* ctx, const Params& P) {
   // persistent grid: resident warps per SM x SMs (occupancy queried once per instantiation)
   static int occ_of_dev[64] = {0};
   int& occ = occ_of_dev[ctx->cfg.device & 63];
-  const size_t smem = sizeof(WarpSmem) * kWarps;
+  const size_t smem = 0;  // the warp's block is a static __shared__ variable
   if (occ == 0) {
     RP_CUDA(cudaFuncSetAttribute(k_integrate<KIND, VAR, UNIT>,
                                  cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
@@ -1196,8 +1209,8 @@ static int run_potentials(rp_ctx* ctx, Params P, int32_t rank, int32_t world,
     P.unit_cnt = ctx->unit_cnt;
     P.unit_aux = ctx->unit_aux;
     int rc2 = KIND != RP_SRC_GRID ? launch_integrate<KIND, 0>(ctx, P)
-              : var == 6 ? launch_integrate<KIND, 6>(ctx, P)
-                         : launch_integrate<KIND, 4>(ctx, P);
+              : var == 6 ? launch_integrate<KIND, kGridVar + 2>(ctx, P)
+                         : launch_integrate<KIND, kGridVar>(ctx, P);
     if (rc2) return rc2;
   }
   ProfScope ps_red(ctx, PK_REDUCE);

@@ -57,8 +57,8 @@ void free_all(rp_ctx* c) {
                   c->sched_key, c->sched_key_sorted, c->sched_idx, c->sched_order, c->cost_prev,
                   c->item_val, c->item_cnt, c->item_aux, c->counters, c->amp_dev, c->trig_full,
                   c->point_key, c->point_key_sorted, c->point_idx, c->point_order,
-                  c->point_owner, c->nseg_prev_pt, c->point_cnt, c->hx_d, c->hy_d, c->hux_d, c->huy_d,
-                  c->mesh_d, c->leaves_prev, c->cluster_dev, c->bp_off_dev, c->bp_dev,
+                  c->point_owner, c->nseg_prev_pt, c->point_cnt, c->hx_d, c->hy_d, c->hux_d, c->huy_d, c->cux_d, c->cuy_d,
+                  c->mesh_d, c->aprev_d, c->leaves_prev, c->cluster_dev, c->bp_off_dev, c->bp_dev,
                   c->unit_key, c->unit_okey, c->unit_okey_sorted, c->unit_iota, c->unit_perm, c->unit_val,
                   c->unit_ndef, c->partials_all, c->shard_buf, c->shards_all,
                   c->unit_cnt, c->unit_aux};
@@ -408,10 +408,9 @@ int rp_shard_scatter(rp_ctx* ctx, const double* shards, int32_t world, int64_t c
 }
 
 int rp_compute_fields(rp_ctx* ctx, const double* phi, const double* ax, const double* ay,
-                      const double* ax_prev, const double* ay_prev, double* ex, double* ey,
-                      double* bz) {
+                      const double* a_prev, int32_t n_prev, double* ex, double* ey, double* bz) {
   RP_ENTER(ctx);
-  return rp_fields_impl(ctx, phi, ax, ay, ax_prev, ay_prev, ex, ey, bz);
+  return rp_fields_impl(ctx, phi, ax, ay, a_prev, n_prev, ex, ey, bz);
 }
 
 int rp_push_particles(rp_ctx* ctx, double* x, double* y, double* ux, double* uy, int64_t n,
@@ -428,6 +427,13 @@ int rp_particle_forces(rp_ctx* ctx, const double* x, const double* y, const doub
   return rp_forces_impl(ctx, x, y, ux, uy, n, bz_ext, ex, ey, bz, fx, fy);
 }
 
+int rp_kick_external(rp_ctx* ctx, const double* ux, const double* uy, int64_t n,
+                     double q_over_mc, double bz_ext, double frac, double* ux_out,
+                     double* uy_out) {
+  RP_ENTER(ctx);
+  return rp_kick_impl(ctx, ux, uy, n, q_over_mc, bz_ext, frac, ux_out, uy_out);
+}
+
 int rp_step_host(rp_ctx* ctx, double* xh, double* yh, double* uxh, double* uyh, int64_t n,
                  double q, const rp_frame* frame_k, double q_over_mc, double bz_ext,
                  double* mesh_host, rp_potential_info* info) {
@@ -437,15 +443,19 @@ int rp_step_host(rp_ctx* ctx, double* xh, double* yh, double* uxh, double* uyh, 
   const size_t npts = (size_t)ctx->cfg.nx * ctx->cfg.ny;
   if (n > ctx->host_cap) {
     cudaFree(ctx->hx_d); cudaFree(ctx->hy_d); cudaFree(ctx->hux_d); cudaFree(ctx->huy_d);
-    ctx->hx_d = ctx->hy_d = ctx->hux_d = ctx->huy_d = nullptr;
+    cudaFree(ctx->cux_d); cudaFree(ctx->cuy_d);
+    ctx->hx_d = ctx->hy_d = ctx->hux_d = ctx->huy_d = ctx->cux_d = ctx->cuy_d = nullptr;
     ctx->host_cap = 0;
     RP_CUDA(cudaMalloc(&ctx->hx_d, n * sizeof(double)));
     RP_CUDA(cudaMalloc(&ctx->hy_d, n * sizeof(double)));
     RP_CUDA(cudaMalloc(&ctx->hux_d, n * sizeof(double)));
     RP_CUDA(cudaMalloc(&ctx->huy_d, n * sizeof(double)));
+    RP_CUDA(cudaMalloc(&ctx->cux_d, n * sizeof(double)));
+    RP_CUDA(cudaMalloc(&ctx->cuy_d, n * sizeof(double)));
     ctx->host_cap = n;
   }
-  if (!ctx->mesh_d) RP_CUDA(cudaMalloc(&ctx->mesh_d, 8 * npts * sizeof(double)));
+  if (!ctx->mesh_d) RP_CUDA(cudaMalloc(&ctx->mesh_d, 6 * npts * sizeof(double)));
+  if (!ctx->aprev_d) RP_CUDA(cudaMalloc(&ctx->aprev_d, 4 * 2 * npts * sizeof(double)));
   cudaStream_t st = ctx->stream;
   size_t nb = (size_t)n * sizeof(double);
   if (n > 0) {
@@ -456,18 +466,28 @@ int rp_step_host(rp_ctx* ctx, double* xh, double* yh, double* uxh, double* uyh, 
   }
   double* m = ctx->mesh_d;
   double *phi = m, *ax = m + npts, *ay = m + 2 * npts, *ex = m + 3 * npts, *ey = m + 4 * npts,
-         *bz = m + 5 * npts, *axp = m + 6 * npts, *ayp = m + 7 * npts;
+         *bz = m + 5 * npts;
   {
     ProfScope ps(ctx, PK_STEP);  // the device part of the step, between the copies
-    int rc = deposit_step(ctx, ctx->hx_d, ctx->hy_d, ctx->hux_d, ctx->huy_d, q, n, frame_k, nullptr);
+    // the current of step k with the momenta of t_k (R-27): the leap-frog momenta advanced by
+    // half a step in the external field
+    int rc = rp_kick_impl(ctx, ctx->hux_d, ctx->huy_d, n, q_over_mc, bz_ext, 0.5, ctx->cux_d,
+                          ctx->cuy_d);
+    if (rc) return rc;
+    rc = deposit_step(ctx, ctx->hx_d, ctx->hy_d, ctx->cux_d, ctx->cuy_d, q, n, frame_k, nullptr);
     if (rc) return rc;
     rc = potentials_full(ctx, phi, ax, ay, nullptr, nullptr, info);
     if (rc) return rc;
-    rc = rp_fields_impl(ctx, phi, ax, ay, ctx->have_prev_A ? axp : nullptr,
-                        ctx->have_prev_A ? ayp : nullptr, ex, ey, bz);
+    rc = rp_fields_impl(ctx, phi, ax, ay, ctx->aprev_d, ctx->n_prev_A, ex, ey, bz);
     if (rc) return rc;
-    RP_CUDA(cudaMemcpyAsync(axp, ax, 2 * npts * sizeof(double), cudaMemcpyDeviceToDevice, st));
-    ctx->have_prev_A = 1;
+    // A history for the next step's dA/dt (R-15b): shift, then this step's (A_x, A_y) first
+    const size_t pair = 2 * npts * sizeof(double);
+    for (int j = 3; j >= 1; --j)
+      RP_CUDA(cudaMemcpyAsync(ctx->aprev_d + (size_t)j * 2 * npts,
+                              ctx->aprev_d + (size_t)(j - 1) * 2 * npts, pair,
+                              cudaMemcpyDeviceToDevice, st));
+    RP_CUDA(cudaMemcpyAsync(ctx->aprev_d, ax, pair, cudaMemcpyDeviceToDevice, st));
+    ctx->n_prev_A = ctx->n_prev_A < 4 ? ctx->n_prev_A + 1 : 4;
     rc = rp_push_impl(ctx, ctx->hx_d, ctx->hy_d, ctx->hux_d, ctx->huy_d, n, q_over_mc, bz_ext, ex,
                       ey, bz);
     if (rc) return rc;
@@ -504,7 +524,7 @@ int rp_load_state(rp_ctx* ctx, int32_t k, int32_t n_pre, const rp_frame* frames_
   ctx->rigid_pending = 0;
   ctx->prehist_set = 1;
   ctx->has_forecast = 0;
-  ctx->have_prev_A = 0;
+  ctx->n_prev_A = 0;
   return RP_OK;
 }
 

@@ -137,8 +137,10 @@ struct rp_ctx {
   // end-to-end (host buffer) path scratch
   int64_t host_cap = 0;
   double* hx_d = nullptr; double* hy_d = nullptr; double* hux_d = nullptr; double* huy_d = nullptr;
-  double* mesh_d = nullptr;         // [8][npts]: phi ax ay ex ey bz ax_prev ay_prev
-  int have_prev_A = 0;
+  double* cux_d = nullptr; double* cuy_d = nullptr;  // time-centred momenta of the deposit (R-27)
+  double* mesh_d = nullptr;         // [6][npts]: phi ax ay ex ey bz of the last rp_step_host
+  double* aprev_d = nullptr;        // [4][2][npts]: A of the 4 steps before (most recent first)
+  int n_prev_A = 0;                 // how many of them are valid
 
   int64_t launches = 0;
   std::string err;
@@ -233,13 +235,15 @@ int rp_potentials_impl(rp_ctx* ctx, int src_kind, const double src[6], int32_t r
                        int32_t* nseg, double* shard_out, int64_t cap, int64_t* n_out,
                        rp_potential_info* info);
 int rp_fields_impl(rp_ctx* ctx, const double* phi, const double* ax, const double* ay,
-                   const double* axp, const double* ayp, double* ex, double* ey, double* bz);
+                   const double* a_prev, int n_prev, double* ex, double* ey, double* bz);
 int rp_push_impl(rp_ctx* ctx, double* x, double* y, double* ux, double* uy, int64_t n,
                  double qmc, double bz_ext, const double* ex, const double* ey,
                  const double* bz);
 int rp_forces_impl(rp_ctx* ctx, const double* x, const double* y, const double* ux,
                    const double* uy, int64_t n, double bz_ext, const double* ex, const double* ey,
                    const double* bz, double* fx, double* fy);
+int rp_kick_impl(rp_ctx* ctx, const double* ux, const double* uy, int64_t n, double qmc,
+                 double bz_ext, double frac, double* ox, double* oy);
 int rp_scatter_impl(rp_ctx* ctx, const double* shards, int32_t world, int64_t cap,
                     double* phi, double* ax, double* ay, double* err, int32_t* nseg);
 int rp_alloc_potential_scratch(rp_ctx* ctx);

@@ -118,9 +118,10 @@ _SIG = {
                                               _P(rp_potential_info)]),
     "rp_shard_capacity": (_i64, [_vp, _i32]),
     "rp_shard_scatter": (C.c_int, [_vp, _vp, _i32, _i64, _vp, _vp, _vp, _vp, _vp]),
-    "rp_compute_fields": (C.c_int, [_vp, _vp, _vp, _vp, _vp, _vp, _vp, _vp, _vp]),
+    "rp_compute_fields": (C.c_int, [_vp, _vp, _vp, _vp, _vp, _i32, _vp, _vp, _vp]),
     "rp_push_particles": (C.c_int, [_vp, _vp, _vp, _vp, _vp, _i64, _d, _d, _vp, _vp, _vp]),
     "rp_particle_forces": (C.c_int, [_vp, _vp, _vp, _vp, _vp, _i64, _d, _vp, _vp, _vp, _vp, _vp]),
+    "rp_kick_external": (C.c_int, [_vp, _vp, _vp, _i64, _d, _d, _d, _vp, _vp]),
     "rp_step_host": (C.c_int, [_vp, _vp, _vp, _vp, _vp, _i64, _d, _P(rp_frame), _d, _d, _vp,
                                _P(rp_potential_info)]),
     "rp_load_state": (C.c_int, [_vp, _i32, _i32, _P(rp_frame), _vp]),
@@ -347,10 +348,15 @@ def rp_shard_scatter(ctx, shards, world, phi, ax, ay, err=None, nseg=None) -> No
                                  _i32t(nseg, "nseg")), ctx, "rp_shard_scatter")
 
 
-def rp_compute_fields(ctx, phi, ax, ay, ax_prev, ay_prev, ex, ey, bz) -> None:
-    _check(_lib.rp_compute_fields(ctx, _f64(phi), _f64(ax), _f64(ay), _f64(ax_prev),
-                                  _f64(ay_prev), _f64(ex), _f64(ey), _f64(bz)), ctx,
-           "rp_compute_fields")
+def rp_compute_fields(ctx, phi, ax, ay, a_prev, ex, ey, bz, n_prev=None) -> None:
+    """a_prev: None, or a float64 CUDA tensor [n_prev][2][npts] of (A_x, A_y) at steps k-1, ...
+    (most recent first); n_prev defaults to its first dimension (0..4)."""
+    if a_prev is None:
+        n = 0
+    else:
+        n = a_prev.shape[0] if n_prev is None else int(n_prev)
+    _check(_lib.rp_compute_fields(ctx, _f64(phi), _f64(ax), _f64(ay), _f64(a_prev, "a_prev"), n,
+                                  _f64(ex), _f64(ey), _f64(bz)), ctx, "rp_compute_fields")
 
 
 def rp_push_particles(ctx, x, y, ux, uy, q_over_mc, bz_ext, ex, ey, bz) -> None:
@@ -364,6 +370,12 @@ def rp_particle_forces(ctx, x, y, ux, uy, bz_ext, ex, ey, bz, fx, fy) -> None:
                                    x.numel(), float(bz_ext), _f64(ex, "ex"), _f64(ey, "ey"),
                                    _f64(bz, "bz"), _f64(fx, "fx"), _f64(fy, "fy")), ctx,
            "rp_particle_forces")
+
+
+def rp_kick_external(ctx, ux, uy, q_over_mc, bz_ext, frac, ux_out, uy_out) -> None:
+    _check(_lib.rp_kick_external(ctx, _f64(ux, "ux"), _f64(uy, "uy"), ux.numel(), float(q_over_mc),
+                                 float(bz_ext), float(frac), _f64(ux_out, "ux_out"),
+                                 _f64(uy_out, "uy_out")), ctx, "rp_kick_external")
 
 
 def rp_step_host(ctx, x, y, ux, uy, q, frame_k, q_over_mc, bz_ext, mesh_out, info=False):

@@ -143,17 +143,23 @@ class OracleOps:
                     nseg[p] = int(rec[5])
         ctx.nseg_prev = ns
 
-    def rp_compute_fields(self, ctx, phi, ax, ay, axp, ayp, ex, ey, bz):
-        fk = ctx.frames[ctx.k % ctx.H]
-        fm = ctx.frames[(ctx.k - 1) % ctx.H]
+    def rp_compute_fields(self, ctx, phi, ax, ay, a_prev, ex, ey, bz):
         sh = (ctx.ny, ctx.nx)
-        a, b, c = oracle.fields(ctx.nx, ctx.ny, ctx.hx, ctx.hy, ctx.c, ctx.dt, fk, fm,
+        m = 0 if a_prev is None else a_prev.shape[0]
+        m = min(m, ctx.H - 1, ctx.k + ctx.n_pre)  # the frames the ring holds (rp.h)
+        frames = [ctx.frames[(ctx.k - j) % ctx.H] for j in range(m + 1)]
+        prev = [(a_prev[j, 0].numpy().reshape(sh), a_prev[j, 1].numpy().reshape(sh)) for j in range(m)]
+        a, b, c = oracle.fields(ctx.nx, ctx.ny, ctx.hx, ctx.hy, ctx.c, ctx.dt, frames,
                                 phi.numpy().reshape(sh), ax.numpy().reshape(sh), ay.numpy().reshape(sh),
-                                None if axp is None else axp.numpy().reshape(sh),
-                                None if ayp is None else ayp.numpy().reshape(sh))
+                                prev)
         ex.copy_(torch.from_numpy(a.ravel()))
         ey.copy_(torch.from_numpy(b.ravel()))
         bz.copy_(torch.from_numpy(c.ravel()))
+
+    def rp_kick_external(self, ctx, ux, uy, qmc, bz_ext, frac, ox, oy):
+        a, b = oracle.kick_external(ctx.dt, ux.numpy(), uy.numpy(), qmc, bz_ext, frac)
+        ox.copy_(torch.from_numpy(a))
+        oy.copy_(torch.from_numpy(b))
 
     def rp_push_particles(self, ctx, x, y, ux, uy, qmc, bz_ext, ex, ey, bz):
         fk = ctx.frames[ctx.k % ctx.H]

@@ -106,22 +106,8 @@ def test_nccl_one_rank_communicator_matches_single_gpu(torch):
     from paper_conf_icpp_arumugamrztgi17_b200.sim import Simulation
     cfg = W.config(1)
     a = Simulation(cfg)
-    dev = torch.device("cuda", 0)
-    nid = rp.rp_nccl_unique_id()
-    # a Simulation whose context holds a one-rank communicator (the N > 1 product path)
-    b = Simulation.__new__(Simulation)
-    b.__dict__.update({k: v for k, v in a.__dict__.items() if k not in ("ctx",)})
-    b.ctx = rp.rp_create(cfg.nx, cfg.ny, cfg.hx, cfg.hy, cfg.kappa_max, cfg.c, cfg.dt, cfg.tau,
-                         cfg.n_theta, cfg.max_depth, cfg.n_root, 0, cfg.rule, cfg.interp,
-                         dist=(0, 1, nid))
+    b = Simulation(cfg, transport="nccl", nccl_id=rp.rp_nccl_unique_id())
     try:
-        rp.rp_set_stream(b.ctx, torch.cuda.current_stream(dev))
-        rp.rp_history_init(b.ctx, cfg.n_pre, W.frames(cfg, range(-cfg.n_pre, 0)), None, True)
-        f64 = dict(dtype=torch.float64, device=dev)
-        for name in ("x", "y", "ux", "uy", "phi", "err", "ex", "ey", "bz"):
-            setattr(b, name, getattr(a, name).clone())
-        b.A = [(torch.zeros(a.npts, **f64), torch.zeros(a.npts, **f64)) for _ in range(2)]
-        b.nseg = a.nseg.clone()
         for _ in range(3):
             a.step()
             inf = b.step(info=True)

@@ -409,32 +409,31 @@ def test_analytic_sources_closed_form_on_gpu(torch, kind):
 
 # ------------------------------------------------------------------ fields and push
 def test_fields_parity(torch):
+    """k_fields vs orc_fields from common inputs (R-15b: order-m backward differences of the node
+    values and positions, m = 0..4), 1e-11 relative."""
     from paper_conf_icpp_arumugamrztgi17_b200 import rp
-    cfg = _bend_small(n=17, kap=4)
+    cfg = _bend_small(n=17, kap=6)
     rng = np.random.default_rng(21)
     npts = cfg.nx * cfg.ny
-    phi, ax, ay, axp, ayp = (rng.standard_normal(npts) for _ in range(5))
-    fk, fm = W.frame(cfg, 1), W.frame(cfg, 0)
-    ex, ey, bz = oracle.fields(cfg.nx, cfg.ny, cfg.hx, cfg.hy, cfg.c, cfg.dt, fk, fm,
-                               phi.reshape(cfg.ny, cfg.nx), ax.reshape(cfg.ny, cfg.nx),
-                               ay.reshape(cfg.ny, cfg.nx), axp.reshape(cfg.ny, cfg.nx),
-                               ayp.reshape(cfg.ny, cfg.nx))
+    sh = (cfg.ny, cfg.nx)
+    phi, ax, ay = (rng.standard_normal(npts) for _ in range(3))
+    prev = rng.standard_normal((4, 2, npts))
+    k = 5
     ctx = G.make_ctx(cfg)
     try:
         ring = np.zeros((cfg.H, cfg.ny, cfg.nx, 4))
-        G.load_state(ctx, cfg, 1, 0, ring, W.ring_frames(cfg, 1))
-        d = _dev_arrays(torch, phi, ax, ay, axp, ayp)
+        G.load_state(ctx, cfg, k, 0, ring, W.ring_frames(cfg, k))
+        d = _dev_arrays(torch, phi, ax, ay, prev)
         out = [torch.zeros(npts, dtype=torch.float64, device="cuda") for _ in range(3)]
-        rp.rp_compute_fields(ctx, *d, *out)
-        for got, want in zip(out, (ex, ey, bz)):
-            g = got.cpu().numpy().reshape(cfg.ny, cfg.nx)
-            assert np.abs(g - want).max() <= 1e-11 * np.abs(want).max()
-        # without the previous step: dA/dt = 0
-        rp.rp_compute_fields(ctx, d[0], d[1], d[2], None, None, *out)
-        ex0, ey0, bz0 = oracle.fields(cfg.nx, cfg.ny, cfg.hx, cfg.hy, cfg.c, cfg.dt, fk, None,
-                                      phi.reshape(cfg.ny, cfg.nx), ax.reshape(cfg.ny, cfg.nx),
-                                      ay.reshape(cfg.ny, cfg.nx))
-        assert np.abs(out[0].cpu().numpy().reshape(cfg.ny, cfg.nx) - ex0).max() <= 1e-11 * np.abs(ex0).max()
+        for m in range(5):
+            frames = [W.frame(cfg, k - j) for j in range(m + 1)]
+            want = oracle.fields(cfg.nx, cfg.ny, cfg.hx, cfg.hy, cfg.c, cfg.dt, frames,
+                                 phi.reshape(sh), ax.reshape(sh), ay.reshape(sh),
+                                 [(prev[j, 0].reshape(sh), prev[j, 1].reshape(sh)) for j in range(m)])
+            rp.rp_compute_fields(ctx, d[0], d[1], d[2], d[3][:m].contiguous() if m else None, *out)
+            for got, w in zip(out, want):
+                g = got.cpu().numpy().reshape(sh)
+                assert np.abs(g - w).max() <= 1e-11 * np.abs(w).max(), m
     finally:
         rp.rp_destroy(ctx)
 
@@ -491,6 +490,27 @@ def test_particle_forces_parity(torch):
         rp.rp_destroy(ctx)
 
 
+def test_kick_external_parity(torch):
+    """rp_kick_external (the deposit's time-centred momenta, R-27) against orc_kick_external on
+    the bend bunch with its dipole field; 1e-13 relative."""
+    from paper_conf_icpp_arumugamrztgi17_b200 import rp
+    cfg = W.config(2)
+    _, _, ux, uy = W.particles(cfg, n=100_000, seed=3)
+    want = oracle.kick_external(cfg.dt, ux, uy, cfg.q_over_mc, cfg.bz_ext, 0.5)
+    ctx = G.make_ctx(cfg)
+    try:
+        uxd, uyd = _dev_arrays(torch, ux, uy)
+        ox, oy = torch.empty_like(uxd), torch.empty_like(uyd)
+        rp.rp_kick_external(ctx, uxd, uyd, cfg.q_over_mc, cfg.bz_ext, 0.5, ox, oy)
+        for g, w in zip((ox, oy), want):
+            assert np.abs(g.cpu().numpy() - w).max() <= 1e-13 * np.abs(want[0]).max()
+        # it turns the momenta from the tangent at -dt/2 onto the tangent at 0 (R-21, R-27)
+        ang = np.arctan2(oy.cpu().numpy(), ox.cpu().numpy())
+        assert abs(np.median(ang)) < 1e-6 < abs(np.median(np.arctan2(uy, ux)))
+    finally:
+        rp.rp_destroy(ctx)
+
+
 # ------------------------------------------------------------------ sharding, e2e, loop
 def test_shard_path_equals_full_mesh(torch):
     """Mesh-point sharding simulated on one GPU: ranks 0..W-1 each compute
@@ -536,14 +556,19 @@ def test_step_host_matches_device_path(torch):
         rp.rp_history_init(ctx2, cfg.n_pre, pre, None, True)
         xd, yd, uxd, uyd = _dev_arrays(torch, x, y, ux, uy)
         n = cfg.nx * cfg.ny
-        phi, ax, ay, ex, ey, bz, axp, ayp = (torch.zeros(n, dtype=torch.float64, device="cuda") for _ in range(8))
+        phi, ax, ay, ex, ey, bz = (torch.zeros(n, dtype=torch.float64, device="cuda") for _ in range(6))
+        ahist = torch.zeros((4, 2, n), dtype=torch.float64, device="cuda")
         hx, hy, hux, huy = (torch.tensor(a).pin_memory() for a in (x, y, ux, uy))
         mesh = torch.zeros((6, n), dtype=torch.float64).pin_memory()
-        for k in range(3):
-            rp.rp_deposit_step(ctx, xd, yd, uxd, uyd, q, W.frame(cfg, k))
+        for k in range(6):
+            cux, cuy = torch.empty_like(uxd), torch.empty_like(uyd)
+            rp.rp_kick_external(ctx, uxd, uyd, cfg.q_over_mc, 0.0, 0.5, cux, cuy)
+            rp.rp_deposit_step(ctx, xd, yd, cux, cuy, q, W.frame(cfg, k))
             rp.rp_compute_potentials(ctx, phi, ax, ay)
-            rp.rp_compute_fields(ctx, phi, ax, ay, axp if k else None, ayp if k else None, ex, ey, bz)
-            axp.copy_(ax); ayp.copy_(ay)
+            rp.rp_compute_fields(ctx, phi, ax, ay, ahist[:min(k, 4)].contiguous() if k else None,
+                                 ex, ey, bz)
+            ahist[1:] = ahist[:-1].clone()
+            ahist[0, 0].copy_(ax); ahist[0, 1].copy_(ay)
             rp.rp_push_particles(ctx, xd, yd, uxd, uyd, cfg.q_over_mc, 0.0, ex, ey, bz)
             rp.rp_step_host(ctx2, hx, hy, hux, huy, q, W.frame(cfg, k), cfg.q_over_mc, 0.0, mesh)
             torch.cuda.synchronize()

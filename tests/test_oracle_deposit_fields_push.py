@@ -75,7 +75,7 @@ def test_fields_exact_on_quadratics():
     phi = 1.5 * U * U - 0.7 * U * V + 0.2 * V * V + U - 3 * V
     ax = 0.3 * U * V + 2 * U
     ay = -0.5 * V * V + U
-    ex, ey, bz = oracle.fields(nx, ny, hx, hy, 1.0, 0.1, fk, None, phi, ax, ay)
+    ex, ey, bz = oracle.fields(nx, ny, hx, hy, 1.0, 0.1, [fk], phi, ax, ay)
     pu, pv = 3 * U - 0.7 * V + 1, -0.7 * U + 0.4 * V - 3
     c, s = fk[2], fk[3]
     np.testing.assert_allclose(ex, -(c * pu - s * pv), atol=1e-12)
@@ -97,13 +97,89 @@ def test_fields_dA_dt_translating_mesh():
     ax = fk[0] + U
     ax_prev = fkm1[0] + U
     z = np.zeros_like(U)
-    ex, ey, bz = oracle.fields(nx, ny, h, h, 2.0, dt, fk, fkm1, z, ax, z, ax_prev, z)
+    ex, ey, bz = oracle.fields(nx, ny, h, h, 2.0, dt, [fk, fkm1], z, ax, z, [(ax_prev, z)])
     np.testing.assert_allclose(ex, 0.0, atol=1e-13)
     np.testing.assert_allclose(ey, 0.0, atol=1e-13)
     # a purely time-dependent A_x (no gradient): E_x = -(1/c) dA_x/dt
     ax2 = np.full_like(U, 3.0)
-    ex, ey, bz = oracle.fields(nx, ny, h, h, 2.0, dt, fk, fk, z, ax2, z, ax2 - 0.4, z)
+    ex, ey, bz = oracle.fields(nx, ny, h, h, 2.0, dt, [fk, fk], z, ax2, z, [(ax2 - 0.4, z)])
     np.testing.assert_allclose(ex, -(0.4 / dt) / 2.0, atol=1e-13)
+
+
+def _rot(a):
+    return np.array([[math.cos(a), -math.sin(a)], [math.sin(a), math.cos(a)]])
+
+
+@pytest.mark.parametrize("m", [1, 2, 3, 4])
+def test_fields_dA_dt_on_a_rotating_mesh(m):
+    """R-15b pin: a mesh rotating rigidly about C (the bend's frames) and a vector potential
+    rotating with it, A(x, t) = R(wt) (G R(-wt) (x - C) + a0), linear in x so the mesh
+    differences are exact.  The exact dA/dt|lab comes from A itself (central difference in t at
+    fixed x).  The scheme's consistent order-m backward differences (node values and node
+    velocity at t_k) must converge as (w dt)^m: the physics needs it, because E_s in the bend
+    is a 1e-4 residual of space-charge-sized terms (so a (w dt)^1 or ^2 error of 1e-5..1e-6
+    relative is not small there)."""
+    nx, ny, h = 7, 6, 0.01
+    R0, w, dt, k = 25.0, 0.04, 0.05, 5
+    C = np.array([0.0, R0])
+    G = np.array([[0.7, -1.3], [2.1, 0.4]])
+    a0 = np.array([0.2, -0.5])
+
+    def A(x, t):
+        return _rot(w * t) @ (G @ (_rot(-w * t) @ (x - C)) + a0)
+
+    def frame(t):  # lower-left node on the circle, u along the tangent
+        ang = w * t
+        O = C + _rot(ang) @ (np.array([0.0, 0.0]) - C)
+        return (O[0], O[1], math.cos(ang), math.sin(ang))
+
+    def nodes(f):
+        U, V = np.meshgrid(np.arange(nx) * h, np.arange(ny) * h)
+        return (f[0] + U * f[2] - V * f[3], f[1] + U * f[3] + V * f[2])
+
+    def grid(t):
+        X, Y = nodes(frame(t))
+        out = np.zeros((2, ny, nx))
+        for iy in range(ny):
+            for ix in range(nx):
+                out[:, iy, ix] = A(np.array([X[iy, ix], Y[iy, ix]]), t)
+        return out
+
+    tk = k * dt
+    Ak = grid(tk)
+    prev = [tuple(grid(tk - j * dt)) for j in range(1, m + 1)]
+    frs = [frame(tk - j * dt) for j in range(m + 1)]
+    z = np.zeros((ny, nx))
+    ex, ey, _ = oracle.fields(nx, ny, h, h, 1.0, dt, frs, z, Ak[0], Ak[1], prev)
+    X, Y = nodes(frame(tk))
+    want = np.zeros((2, ny, nx))
+    d = 1e-4
+    for iy in range(ny):
+        for ix in range(nx):
+            p = np.array([X[iy, ix], Y[iy, ix]])
+            want[:, iy, ix] = -(A(p, tk + d) - A(p, tk - d)) / (2 * d)
+    err = max(np.abs(ex - want[0]).max(), np.abs(ey - want[1]).max())
+    scale = np.abs(want).max()
+    eps = w * dt
+    # order m: error ~ eps^m (relative); the m = 1 scheme's error is measured at 1.9e-5 here
+    assert err <= 10 * eps ** m * scale + 1e-10, (m, err)
+    if m >= 3:
+        assert err < 1e-9 * scale
+
+
+def test_fields_dA_dt_time_polynomial_exact():
+    """A purely time-dependent A_x on a static mesh: the order-m backward difference is exact
+    for polynomials in t of degree <= m."""
+    nx, ny, h, dt = 5, 4, 0.5, 0.3
+    f = (0.0, 0.0, 1.0, 0.0)
+    z = np.zeros((ny, nx))
+    for m in range(1, 5):
+        p = lambda t: sum(c * t ** i for i, c in enumerate([1.0, 0.3, -0.2, 0.05, 0.01][:m + 1]))
+        dp = lambda t: sum(i * c * t ** (i - 1) for i, c in enumerate([1.0, 0.3, -0.2, 0.05, 0.01][:m + 1]) if i)
+        tk = 2.0
+        prev = [(np.full((ny, nx), p(tk - j * dt)), z) for j in range(1, m + 1)]
+        ex, _, _ = oracle.fields(nx, ny, h, h, 1.0, dt, [f] * (m + 1), z, np.full((ny, nx), p(tk)), z, prev)
+        np.testing.assert_allclose(ex, -dp(tk), rtol=0, atol=1e-11)
 
 
 def test_boris_gyration():
@@ -186,3 +262,27 @@ def test_particle_forces_are_the_first_order_boris_kick():
     _, _, ux2, uy2 = oracle.push(nx, ny, 1.0, 1.0, 1.0, dt, fk, x, y, ux, uy, qmc, 0.3, ex, ey, bz)
     np.testing.assert_allclose((ux2 - ux) / (qmc * dt), fx, rtol=1e-6, atol=1e-7)
     np.testing.assert_allclose((uy2 - uy) / (qmc * dt), fy, rtol=1e-6, atol=1e-7)
+
+
+def test_kick_external_centres_the_leap_frog_momenta():
+    """R-27: the current of step k uses the momenta of t_k, the leap-frog ones advanced by dt/2
+    in the external dipole.  Pins: |u| conserved; the rotation angle is the cyclotron angle
+    q/mc B (dt/2) / gamma to its O(angle^3) Boris error; two half kicks rotate like one full
+    push of a particle at rest in E (orc_push, E = 0) to O(angle^3); the sense: B_z < 0 with
+    q > 0 turns u counter-clockwise (the bend, workloads R-20)."""
+    ux, uy = np.array([3.0, 1e4, -2.0]), np.array([0.0, 15.0, 0.5])
+    qmc, B, dt = 1.0, -2.0, 0.01
+    kx, ky = oracle.kick_external(dt, ux, uy, qmc, B, 0.5)
+    np.testing.assert_allclose(np.hypot(kx, ky), np.hypot(ux, uy), rtol=1e-15)
+    g = np.sqrt(1 + ux ** 2 + uy ** 2)
+    ang = np.arctan2(ky, kx) - np.arctan2(uy, ux)
+    want = -qmc * B * 0.5 * dt / g
+    assert np.all(np.abs(ang - want) <= np.abs(want) ** 3 / 6 + 1e-15)
+    assert ang[0] > 0
+    z = np.zeros((4, 4))
+    _, _, px, py = oracle.push(4, 4, 1.0, 1.0, 1.0, dt, (100, 100, 1, 0), np.zeros(3), np.zeros(3),
+                               ux, uy, qmc, B, z, z, z)
+    k2x, k2y = oracle.kick_external(dt, kx, ky, qmc, B, 0.5)
+    full = np.arctan2(py, px) - np.arctan2(uy, ux)
+    two = np.arctan2(k2y, k2x) - np.arctan2(uy, ux)
+    assert np.all(np.abs(full - two) <= np.abs(full) ** 3 / 4 + 1e-15)

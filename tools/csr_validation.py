@@ -72,16 +72,18 @@ def tsc_expected_nodes(cfg):
     return np.outer(axis(cfg.ny, cfg.hy), axis(cfg.nx, cfg.hx))
 
 
-def steady_ring(cfg, k, density=None):
+def steady_ring(cfg, k, density=None, psi_offset=0.0):
     """Ring at step k: every level holds the same comoving bunch `density` (default: node
-    samples of the Gaussian), current rho beta0 along the level's tangent (lab components)."""
+    samples of the Gaussian), current rho beta0 along the level's tangent turned by psi_offset
+    (lab components)."""
     g = gaussian_nodes(cfg) if density is None else density
     ring = np.zeros((cfg.H, cfg.ny, cfg.nx, 4))
+    co, so = math.cos(psi_offset), math.sin(psi_offset)
     for l in range(k - cfg.H + 1, k + 1):
         _, _, c, s = W.frame(cfg, l)
         ring[l % cfg.H, :, :, 0] = g
-        ring[l % cfg.H, :, :, 1] = g * cfg.beta0 * c
-        ring[l % cfg.H, :, :, 2] = g * cfg.beta0 * s
+        ring[l % cfg.H, :, :, 1] = g * cfg.beta0 * (c * co - s * so)
+        ring[l % cfg.H, :, :, 2] = g * cfg.beta0 * (s * co + c * so)
     return ring
 
 
@@ -166,21 +168,25 @@ def axis_points(cfg, k, offsets_sigma, v_sigma=0.0):
 
 
 # ------------------------------------------------------------------ GPU path
-def gpu_steady_fields(rp, torch, cfg, k, density=None):
-    """Potentials at steps k-1 and k of the steady-state ring, then the fields at step k."""
+def gpu_steady_fields(rp, torch, cfg, k, density=None, psi_offset=0.0, n_prev=4):
+    """Potentials at steps k-n_prev .. k of the steady-state ring, then the fields at step k
+    (dA/dt from the n_prev previous steps, R-15b)."""
     n = cfg.nx * cfg.ny
     dev = torch.device("cuda:0")
     ctx = rp.rp_create(cfg.nx, cfg.ny, cfg.hx, cfg.hy, cfg.kappa_max, cfg.c, cfg.dt, cfg.tau)
     try:
         pot = {}
-        for kk in (k - 1, k):
+        for kk in range(k - n_prev, k + 1):
             rp.rp_load_state(ctx, kk, cfg.n_pre, W.ring_frames(cfg, kk),
-                             torch.tensor(steady_ring(cfg, kk, density), device=dev))
+                             torch.tensor(steady_ring(cfg, kk, density, psi_offset), device=dev))
             t3 = [torch.zeros(n, dtype=torch.float64, device=dev) for _ in range(3)]
             rp.rp_compute_potentials(ctx, *t3)
             pot[kk] = t3
+        prev = None
+        if n_prev:
+            prev = torch.stack([torch.stack([pot[k - j][1], pot[k - j][2]]) for j in range(1, n_prev + 1)])
         out = [torch.zeros(n, dtype=torch.float64, device=dev) for _ in range(3)]
-        rp.rp_compute_fields(ctx, *pot[k], pot[k - 1][1], pot[k - 1][2], *out)
+        rp.rp_compute_fields(ctx, *pot[k], prev, *out)
         torch.cuda.synchronize()
         return ctx, out
     except Exception:
@@ -248,12 +254,14 @@ def _bunch_particles(cfg, n, seed, k):
     return X, Y, cd * ux - sd * uy, sd * ux + cd * uy
 
 
-def mse_study(ns=(10_000, 100_000, 1_000_000, 10_000_000), n=129, k=1, seed=17_129):
+def mse_study(ns=(10_000, 100_000, 1_000_000, 10_000_000), n=129, k=4, seed=17_129):
     """Fig. 3: mean-square error of the longitudinal force on the particles vs N on a fixed
-    129^2 grid.  Each run: rigid pre-history + GPU deposit of the bunch at steps 0 and 1
-    (the particles carried rigidly), potentials at both steps, fields, forces at the step-1
-    particles.  The exact force of each particle: the same path fed the noise-free expected
-    deposit (Gaussian x TSC kernel), gathered at the same positions."""
+    129^2 grid.  Each run: rigid pre-history + GPU deposit of the bunch at steps 0..k (the
+    particles carried rigidly along the orbit), potentials at every step, fields at step k from
+    the k previous potentials (R-15b), forces at the step-k particles.  The exact force of each
+    particle: the same path fed the noise-free expected deposit (the Gaussian convolved with the
+    TSC kernel) with the particles' mean current -- along the tangent half a step back, where
+    the leap-frog momenta live (R-21) -- gathered at the same positions."""
     import torch
     from paper_conf_icpp_arumugamrztgi17_b200 import rp
     cfg = csr_config(n)
@@ -261,23 +269,27 @@ def mse_study(ns=(10_000, 100_000, 1_000_000, 10_000_000), n=129, k=1, seed=17_1
     npts = n * n
     t = lambda a: torch.tensor(np.ascontiguousarray(a, dtype=np.float64), device=dev)
     ref_ctx, ref_fields = gpu_steady_fields(rp, torch, cfg, k, tsc_expected_nodes(cfg))
-    out = {"mesh": n, "ns": list(ns), "mse_Fs": [], "mse_Fn": [], "mean_Fs2": [], "n_ppc": []}
+    out = {"mesh": n, "step": k, "ns": list(ns), "mse_Fs": [], "mse_Fn": [], "mean_Fs2": [],
+           "mean_Fn2": [], "n_ppc": []}
     try:
         for N in ns:
             ctx = rp.rp_create(cfg.nx, cfg.ny, cfg.hx, cfg.hy, cfg.kappa_max, cfg.c, cfg.dt, cfg.tau)
             try:
                 rp.rp_history_init(ctx, cfg.n_pre, W.frames(cfg, range(-cfg.n_pre, 0)), None, True)
                 pot = []
-                for kk in (0, 1):
+                for kk in range(k + 1):
                     X, Y, UX, UY = _bunch_particles(cfg, N, seed, kk)
-                    q = 1.0 / N
-                    rp.rp_deposit_step(ctx, t(X), t(Y), t(UX), t(UY), q, W.frame(cfg, kk))
+                    # the current with the momenta of t_k (R-27), as the simulation loop does
+                    cu = [torch.empty(N, dtype=torch.float64, device=dev) for _ in range(2)]
+                    rp.rp_kick_external(ctx, t(UX), t(UY), cfg.q_over_mc, cfg.bz_ext, 0.5, *cu)
+                    rp.rp_deposit_step(ctx, t(X), t(Y), *cu, 1.0 / N, W.frame(cfg, kk))
                     p3 = [torch.zeros(npts, dtype=torch.float64, device=dev) for _ in range(3)]
                     rp.rp_compute_potentials(ctx, *p3)
                     pot.append(p3)
+                prev = torch.stack([torch.stack([pot[k - j][1], pot[k - j][2]]) for j in range(1, k + 1)])
                 fld = [torch.zeros(npts, dtype=torch.float64, device=dev) for _ in range(3)]
-                rp.rp_compute_fields(ctx, *pot[1], pot[0][1], pot[0][2], *fld)
-                xs, ys, uxs, uys = (t(a) for a in (X, Y, UX, UY))
+                rp.rp_compute_fields(ctx, *pot[k], prev, *fld)
+                xs, ys, uxs, uys = t(X), t(Y), cu[0], cu[1]
                 f = [torch.zeros(N, dtype=torch.float64, device=dev) for _ in range(4)]
                 rp.rp_particle_forces(ctx, xs, ys, uxs, uys, 0.0, *fld, f[0], f[1])
                 rp.rp_particle_forces(ref_ctx, xs, ys, uxs, uys, 0.0, *ref_fields, f[2], f[3])
@@ -291,11 +303,30 @@ def mse_study(ns=(10_000, 100_000, 1_000_000, 10_000_000), n=129, k=1, seed=17_1
             out["mse_Fs"].append(float(np.mean((fs - rs) ** 2)))
             out["mse_Fn"].append(float(np.mean((fn - rn) ** 2)))
             out["mean_Fs2"].append(float(np.mean(rs ** 2)))
+            out["mean_Fn2"].append(float(np.mean(rn ** 2)))
             out["n_ppc"].append(N / npts)
+            if N == max(ns):  # absolute forces on a sample of particles vs the exact solution
+                # particles in the bunch core (|u|, |v| <= 3 sigma of the centre): the mesh ends at
+                # 5 sigma, where the zero-padded stencils and one-sided differences take over
+                fk = W.frame(cfg, k)
+                du = (X - fk[0]) * fk[2] + (Y - fk[1]) * fk[3] - 0.5 * cfg.extent
+                dv = (Y - fk[1]) * fk[2] - (X - fk[0]) * fk[3] - 0.5 * cfg.extent
+                core = np.nonzero((np.abs(du) <= 3 * cfg.sigma) & (np.abs(dv) <= 3 * cfg.sigma))[0]
+                rng = np.random.default_rng(5)
+                idx = rng.choice(core, 60, replace=False)
+                ex_ = np.array([semi_analytic_forces(cfg, (X[i], Y[i]), k * cfg.dt) for i in idx])
+                peak = np.abs(ex_[:, 0]).max()
+                out["sample_particles"] = 60
+                out["exact_Fs_peak_in_sample"] = float(peak)
+                out["ref_vs_exact_Fs_max_over_peak"] = float(np.abs(rs[idx] - ex_[:, 0]).max() / peak)
+                out["ref_vs_exact_Fn_max_over_peak"] = float(
+                    np.abs(rn[idx] - ex_[:, 1]).max() / np.abs(ex_[:, 1]).max())
+                out["noisy_vs_exact_Fs_rms_over_peak"] = float(
+                    np.sqrt(np.mean((fs[idx] - ex_[:, 0]) ** 2)) / peak)
     finally:
         rp.rp_destroy(ref_ctx)
-    ln, lm = np.log(np.array(ns, dtype=float)), np.log(np.array(out["mse_Fs"]))
-    out["slope_Fs"] = float(np.polyfit(ln, lm, 1)[0])
+    ln = np.log(np.array(ns, dtype=float))
+    out["slope_Fs"] = float(np.polyfit(ln, np.log(np.array(out["mse_Fs"])), 1)[0])
     out["slope_Fn"] = float(np.polyfit(ln, np.log(np.array(out["mse_Fn"])), 1)[0])
     return out
 
