@@ -77,6 +77,8 @@ typedef struct {
   int64_t evals;                /* integrand evaluations (flop census)                */
   int64_t nodes;                /* r' nodes evaluated (15 per segment)                */
   double min_margin;            /* min |err - tol| / tol over all decisions           */
+  int64_t chase_segs;           /* diagnostics: segments whose subtree ends in a */
+  int64_t chase_evals;          /* capped leaf, and their integrand evaluations          */
 } orc_result;
 
 /* ------------------------------------------------------------------ */
@@ -557,10 +559,12 @@ static void tree(subctx* X, double A, double B, double R, int32_t lev, int64_t i
   double fa = ldexp((double)idx, -lev), fb = ldexp((double)(idx + 1), -lev);
   double a = A + (B - A) * fa, b = A + (B - A) * fb;
   double K[3], G[3], err;
+  const int64_t e0 = X->evals;
   if (P->rule == 1)
     simpson5(X, a, b, K, G, &err);
   else
     gk15(X, a, b, K, G, &err);
+  const int64_t de = X->evals - e0;
   res->nseg++;
   res->nodes += P->rule == 1 ? 5 : 15;
   double tol = P->tau * ldexp(B - A, -lev) / R;
@@ -569,7 +573,11 @@ static void tree(subctx* X, double A, double B, double R, int32_t lev, int64_t i
   if (margin < 1e-9) res->ties++;
   if (lev > res->max_level) res->max_level = lev;
   if (err <= tol || lev >= P->max_depth) {
-    if (!(err <= tol)) res->capped++;
+    if (!(err <= tol)) {
+      res->capped++;
+      res->chase_segs++;
+      res->chase_evals += de;
+    }
     res->nleaf++;
     res->phi += K[0];
     res->ax += K[1];
@@ -577,8 +585,13 @@ static void tree(subctx* X, double A, double B, double R, int32_t lev, int64_t i
     res->err += err;
     return;
   }
+  const int32_t capped0 = res->capped;
   tree(X, A, B, R, lev + 1, 2 * idx, res);
   tree(X, A, B, R, lev + 1, 2 * idx + 1, res);
+  if (res->capped > capped0) {  /* this segment split on the way to a capped leaf */
+    res->chase_segs++;
+    res->chase_evals += de;
+  }
 }
 
 /* ------------------------------------------------------------------ */

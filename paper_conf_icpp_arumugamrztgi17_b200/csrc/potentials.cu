@@ -313,9 +313,6 @@ __constant__ double c_pio2[3] = {0.63661977236758134308, 1.5707963267948965580,
                                  6.1232339957367658e-17};  // 2/pi, pi/2 = hi + lo
 
 __device__ __forceinline__ void sincos_b(double x, double* s, double* c) {
-#ifdef RP_EXP_CHEAPSINCOS  // development timing experiment: wrong results
-  { const double z = x * x; *s = x * (1.0 - z * 0.16666); *c = 1.0 - 0.5 * z; return; }
-#endif
   const double k = rint(x * c_pio2[0]);
   double r = fma(-k, c_pio2[1], x);
   r = fma(-k, c_pio2[2], r);
@@ -598,11 +595,7 @@ __device__ __forceinline__ void pipelined_round(const Item& it, const Params& P,
                         : geom_point<false, LAG>(P, S, trf, e, 0, N, wfull, third, inv_n1);
 #pragma unroll 1
   for (int n = 0; n < nn; ++n) {
-#ifdef RP_EXP_NOREFILL  // development timing experiment: wrong results
-    if (cur.cell != kNoCell && ccell == kNoCell) {
-#else
     if (cur.cell != kNoCell && cur.cell != ccell) {
-#endif
       ccell = cur.cell;
       refill(it, rs, cur.cell, st);
     }
