@@ -52,14 +52,8 @@ constexpr uint32_t kEmptyKey = 0xFFFFFFFFu;  // schedule key of an item without 
 
 constexpr double kTwoPi = 6.283185307179586476925286766559;
 constexpr int kMaxArcs = 8;
-#ifdef RP_CTA_CHUNK
-constexpr int kWarps = 8;       // warps per CTA: one CTA per SM works a window of kChunk items
-constexpr int kChunk = 64;      // consecutive items in the schedule order (same subregion, points
-                                // in raster order within a cost class: overlapping circles, L1 reuse)
-#else
 constexpr int kWarps = 1;  // warps per CTA of k_integrate (1: the warp's shared block sits at
                             // a constant address, no per-iteration warp-index arithmetic)
-#endif
 
 struct Params {
   int nx, ny, PX, npts, kmax, kap, k, H, n_theta, max_depth, n_root, rule, variant, interp;
@@ -662,33 +656,9 @@ __global__ void __launch_bounds__(32 * kWarps) k_integrate(
   const double Nd = (double)N;
   const double wfull = kTwoPi / Nd;
   const double third = 1.0 / 3.0;
-#ifdef RP_CTA_CHUNK
-  // CTA work window: state = chunk << 32 | next; the warp that draws next == kChunk fetches the
-  // next chunk from the global counter, warps that draw beyond it wait for the new chunk
-  __shared__ unsigned long long s_state;
-  if (threadIdx.x == 0)
-    s_state = atomicAdd(&counters[UNIT ? C_NEXT_U : C_NEXT], 1ULL) << 32;
-  __syncthreads();
-#endif
   for (;;) {
     unsigned long long idx = 0;
-#ifdef RP_CTA_CHUNK
-    if (lane == 0) {
-      for (;;) {
-        const unsigned long long st0 = atomicAdd(&s_state, 1ULL);
-        const unsigned long long chunk = st0 >> 32, nxt = st0 & 0xffffffffULL;
-        if (nxt < (unsigned long long)kChunk) { idx = chunk * kChunk + nxt; break; }
-        if (nxt == (unsigned long long)kChunk) {
-          const unsigned long long c2 = atomicAdd(&counters[UNIT ? C_NEXT_U : C_NEXT], 1ULL);
-          atomicExch(&s_state, c2 << 32);
-        } else {
-          while ((*(volatile unsigned long long*)&s_state >> 32) == chunk) {}
-        }
-      }
-    }
-#else
     if (lane == 0) idx = atomicAdd(&counters[UNIT ? C_NEXT_U : C_NEXT], 1ULL);
-#endif
     idx = __shfl_sync(0xffffffffu, idx, 0);
     if (idx >= n_items) break;
     const int uidx = UNIT ? P.unit_order[idx] : 0;

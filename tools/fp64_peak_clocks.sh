@@ -4,7 +4,7 @@ set -e
 nvcc -gencode arch=compute_100a,code=sm_100a -O3 -o /tmp/mix_peak tools/mix_peak.cu
 nvidia-smi --query-gpu=clocks.sm,clocks.max.sm,clocks_event_reasons.active,power.draw --format=csv,noheader,nounits -lms 50 > /tmp/clk.csv &
 SMI=$!
-for i in $(seq 1 60); do /tmp/mix_peak; done > /tmp/mix.jsonl
+/tmp/mix_peak 1500 > /tmp/mix.jsonl
 kill $SMI
 python - <<'PY'
 import json, statistics
@@ -18,8 +18,8 @@ for l in open("/tmp/clk.csv"):
         clk.append((float(p[0]), float(p[1]), p[2], float(p[3])))
     except Exception:
         pass
-busy = [c for c in clk if c[3] > 400]  # samples under load
-out = {"tool": "tools/mix_peak.cu (8 interleaved DFMA chains / 8 DMMA per iteration, 148 SMs), 60 repeats",
+busy = [c for c in clk if c[3] > 250]  # samples under load (idle ~ 140 W)
+out = {"tool": "tools/mix_peak.cu 1500 (8 interleaved DFMA chains / 8 DMMA per iteration, 148 SMs; the pure DFMA and DMMA runs repeated 1500 times, ~8 s of load)",
        "dfma_tf_median": statistics.median(dfma), "dfma_tf_max": max(dfma),
        "dmma_tf_median": statistics.median(dmma), "dmma_tf_max": max(dmma),
        "clock_samples_under_load": len(busy),

@@ -1,3 +1,4 @@
+#include <cstdlib>
 // Do DMMA (tensor) and DFMA (FP64 pipe) run concurrently on sm_100a?  Mixed-loop throughput.
 #include <cstdio>
 #include <cuda_runtime.h>
@@ -39,9 +40,11 @@ void run(int sms, double* out) {
          NM, NF, ms, mma_fl / (ms * 1e-3) / 1e12, fma_fl / (ms * 1e-3) / 1e12,
          (mma_fl + fma_fl) / (ms * 1e-3) / 1e12);
 }
-int main() {
+int main(int argc, char** argv) {
   int sms = 0; cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, 0);
   double* out; cudaMalloc(&out, 8);
+  const int reps = argc > 1 ? atoi(argv[1]) : 1;  // repeat the pure DFMA / DMMA runs (clock logs)
+  for (int r = 1; r < reps; ++r) { run<0, 8>(sms, out); run<8, 0>(sms, out); }
   run<8, 0>(sms, out);
   run<0, 8>(sms, out);
   run<8, 8>(sms, out);

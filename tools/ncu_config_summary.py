@@ -76,10 +76,15 @@ def main():
              "is in the profiler range. Integrator = `k_integrate` item launch + unit launch. "
              "Algorithmic TF/s = the census (evals - skipped) x 210 + r' nodes x 100 + segments x 60 "
              f"over the ncu durations of the two integrator launches; peak {peak} TF/s (DFMA, "
-             "measured). ncu durations are serialised replays (`--clock-control none`).",
+             "measured). ncu durations are serialised replays (`--clock-control none`). DRAM GB/call: "
+             "read + write of the integrator launches of one whole-mesh call; ring GB: the whole "
+             "history ring (the levels with support are read once with the subregion-major order; the "
+             "rest of the traffic is the dense (point, subregion) item arrays). Config 5: the counters "
+             "of rank 0's shard of an 8-way split (`tools/ncu_cfg5.sh`; a full call is ~55 s per ncu "
+             "replay pass) and the DRAM bytes of its whole call.",
              "",
              "| config | integrator ms (ncu) | share of call | alg. TF/s | frac | FP64 pipe % | "
-             "executed FP64 TF/s | DRAM GB/call | alg. DRAM GB | L2 hit % | L1 hit % | branch uniform % | "
+             "executed FP64 TF/s | DRAM GB/call | ring GB | L2 hit % | L1 hit % | branch uniform % | "
              "sectors/req | threads/instr | warps active % | issue % | regs |",
              "|" + "---|" * 17]
     for n in range(1, 6):
