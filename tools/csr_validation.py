@@ -314,7 +314,16 @@ def mse_study(ns=(10_000, 100_000, 1_000_000, 10_000_000), n=129, k=4, seed=17_1
                 core = np.nonzero((np.abs(du) <= 3 * cfg.sigma) & (np.abs(dv) <= 3 * cfg.sigma))[0]
                 rng = np.random.default_rng(5)
                 idx = rng.choice(core, 60, replace=False)
-                ex_ = np.array([semi_analytic_forces(cfg, (X[i], Y[i]), k * cfg.dt) for i in idx])
+                # the exact force on each sampled particle with its own velocity (its transverse
+                # beta ~ 2e-5 times the space-charge B_z is of the size of the CSR force)
+                cux, cuy = cu[0].cpu().numpy(), cu[1].cpu().numpy()
+                ex_ = []
+                for i in idx:
+                    exf, eyf, bzf = semi_analytic_fields(cfg, (X[i], Y[i]), k * cfg.dt)
+                    g = math.sqrt(1.0 + cux[i] ** 2 + cuy[i] ** 2)
+                    fx_, fy_ = exf + cuy[i] / g * bzf, eyf - cux[i] / g * bzf
+                    ex_.append((fx_ * c + fy_ * s, -fx_ * s + fy_ * c))
+                ex_ = np.array(ex_)
                 peak = np.abs(ex_[:, 0]).max()
                 out["sample_particles"] = 60
                 out["exact_Fs_peak_in_sample"] = float(peak)
