@@ -544,33 +544,6 @@ __device__ __forceinline__ void refill(const Item& it, size_t rs, int cell,
     }
 }
 
-#ifdef RP_LATE_REFILL
-// predicated refill: the 27 loads of the next node's cell are issued in the same basic block as
-// the current contraction; each load only has to wait for the last read of its registers, so the
-// refill latency overlaps the rest of the contraction (lanes with on == false load nothing)
-__device__ __forceinline__ void refill_pred(const Item& it, size_t rs, int cell, bool on,
-                                            double (&st)[3][9][3]) {
-  const size_t base = (size_t)4 * (ptrdiff_t)cell;
-  const double* g[3] = {it.g0 + base, it.g1 + base, it.g2 + base};
-  const unsigned pr = on ? 1u : 0u;
-#pragma unroll
-  for (int l = 0; l < 3; ++l)
-#pragma unroll
-    for (int b = 0; b < 3; ++b) {
-      const double* row = g[l] + b * rs;
-#pragma unroll
-      for (int a = 0; a < 3; ++a) {
-        double d = 0.0;
-        asm("{\n\t.reg .pred q;\n\tsetp.ne.u32 q, %4, 0;\n\t"
-            "@q ld.global.nc.v4.f64 {%0,%1,%2,%3}, [%5];\n\t}"
-            : "+d"(st[l][3 * b + a][0]), "+d"(st[l][3 * b + a][1]), "+d"(st[l][3 * b + a][2]),
-              "+d"(d)
-            : "r"(pr), "l"(row + 4 * a));
-      }
-    }
-}
-#endif
-
 // 27-node x 3-component contraction at one point -> (f0, f1, f2)
 template <bool LAG>
 __device__ __forceinline__ void contract_point(const Geo& g, const NodeRec& nd,
@@ -620,24 +593,12 @@ __device__ __forceinline__ void pipelined_round(const Item& it, const Params& P,
   const double2 trf = __ldg(trig_full + (e < N ? e : 0));
   Geo cur = (fullmask & 1) ? geom_point<true, LAG>(P, S, trf, e, 0, N, wfull, third, inv_n1)
                         : geom_point<false, LAG>(P, S, trf, e, 0, N, wfull, third, inv_n1);
-#ifdef RP_LATE_REFILL
-  if (cur.cell != kNoCell && cur.cell != ccell) {  // the round's first node
-    ccell = cur.cell;
-    refill(it, rs, cur.cell, st);
-  }
-#endif
-#ifdef RP_UNROLL2
-#pragma unroll 2
-#else
 #pragma unroll 1
-#endif
   for (int n = 0; n < nn; ++n) {
-#ifndef RP_LATE_REFILL
     if (cur.cell != kNoCell && cur.cell != ccell) {
       ccell = cur.cell;
       refill(it, rs, cur.cell, st);
     }
-#endif
     const NodeRec& nd = S.node[n];
     double f0, f1, f2;
     Geo nxt;
@@ -651,13 +612,6 @@ __device__ __forceinline__ void pipelined_round(const Item& it, const Params& P,
       nxt = cur;
       contract_point<LAG>(cur, nd, st, f0, f1, f2);
     }
-#ifdef RP_LATE_REFILL
-    {
-      const bool need = n + 1 < nn && nxt.cell != kNoCell && nxt.cell != ccell;
-      refill_pred(it, rs, need ? nxt.cell : 0, need, st);
-      if (need) ccell = nxt.cell;
-    }
-#endif
     const double wk = cur.w * nd.wk;
     k0 += wk * f0; k1 += wk * f1; k2 += wk * f2;
     if ((gmask >> n) & 1) {  // G7: Gauss nodes only (warp-uniform n)
