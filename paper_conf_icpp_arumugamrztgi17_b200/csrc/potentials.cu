@@ -312,8 +312,15 @@ __constant__ double c_cosp[6] = {-1.13596475577881948265e-11, 2.0875723212981748
 __constant__ double c_pio2[3] = {0.63661977236758134308, 1.5707963267948965580,
                                  6.1232339957367658e-17};  // 2/pi, pi/2 = hi + lo
 
+// Round-to-integer through the FP64 adder: for |y| < 2^51, y + 1.5 * 2^52 rounds y to an
+// integer in the unit of the last place (IEEE mode of the add), the low word of the sum is that
+// integer (two's complement) and the sum minus the constant is it as a double -- exact, and on
+// the FP64 pipe instead of the variable-latency FRND / F2I conversions.
+constexpr double kRoundMagic = 6755399441055744.0;  // 1.5 * 2^52
+
 __device__ __forceinline__ void sincos_b(double x, double* s, double* c) {
-  const double k = rint(x * c_pio2[0]);
+  const double kk = __dadd_rn(__dmul_rn(x, c_pio2[0]), kRoundMagic);  // rint(x * 2/pi) + magic
+  const double k = __dsub_rn(kk, kRoundMagic);
   double r = fma(-k, c_pio2[1], x);
   r = fma(-k, c_pio2[2], r);
   const double z = r * r;
@@ -329,7 +336,7 @@ __device__ __forceinline__ void sincos_b(double x, double* s, double* c) {
   pc = fma(z, pc, c_cosp[4]);
   pc = fma(z, pc, c_cosp[5]);
   const double cr = fma(z * z, pc, fma(-0.5, z, 1.0));
-  const int q = (int)k & 3;
+  const int q = __double2loint(kk) & 3;
   const double ss = (q & 1) ? cr : sr, cc = (q & 1) ? sr : cr;
   *s = (q & 2) ? -ss : ss;
   *c = ((q + 1) & 2) ? -cc : cc;
@@ -507,23 +514,30 @@ __device__ __forceinline__ Geo geom_point(const Params& P, const WarpSmem& S, do
     // lie on the support boundary, where the zero-padded TSC stencil vanishes (R-24) and the
     // Lagrange-3 integrand takes its limit from outside, 0 (R-25b)
     const int ec = valid ? e : 0;
-    const int q = __float2int_rz(((float)ec + 0.5f) * inv_n1);  // arc index, exact for e < 2^20
+    // arc index trunc((ec + 1/2) / (N - 1)), exact for e < 2^20 (the quotient stays >= 1/(2N)
+    // from an integer); truncated by an FP32 add in round-toward-zero (no F2I)
+    const float qf = __fadd_rz(fmaf((float)ec, inv_n1, 0.5f * inv_n1), 12582912.0f);
+    const int q = __float_as_int(qf) - 0x4B400000;
     const int mm = ec - q * (N - 1) + 1;
     const double d = S.dth[n][q];
-    sincos_b(S.th1[n][q] + (double)mm * d, &sn, &cs);
+    const double mmd = __dsub_rn(__hiloint2double(0x43300000, mm), 4503599627370496.0);  // (double)mm
+    sincos_b(S.th1[n][q] + mmd * d, &sn, &cs);
     const double coef = (mm & 1) ? 4.0 : 2.0;
     w = coef * d * third;
   }
   const NodeRec& nd = S.node[n];
   const double u = nd.cu + nd.r * cs, v = nd.cv + nd.r * sn;
-  const double tx = u * P.inv_hx, ty = v * P.inv_hy;
-  const double fx = floor(tx + 0.5), fy = floor(ty + 0.5);
-  const int ix = min(max(__double2int_rz(fx), -2), P.nx + 1);
-  const int iy = min(max(__double2int_rz(fy), -2), P.ny + 1);
+  // nearest node (ix, iy) = floor(t + 1/2) and the offset t - floor(t + 1/2), t = u / h: the
+  // floor as a round-down add of the magic constant (see sincos_b; no FRND / F2I)
+  const double sx = __dadd_rd(fma(u, P.inv_hx, 0.5), kRoundMagic);
+  const double sy = __dadd_rd(fma(v, P.inv_hy, 0.5), kRoundMagic);
+  const double fx = __dsub_rn(sx, kRoundMagic), fy = __dsub_rn(sy, kRoundMagic);
+  const int ix = min(max(__double2loint(sx), -2), P.nx + 1);
+  const int iy = min(max(__double2loint(sy), -2), P.ny + 1);
   // a slot the node does not have evaluates slot 0's (finite) point with weight 0 and no refill
   Geo g;
-  g.dx = tx - fx;
-  g.dy = ty - fy;
+  g.dx = fma(u, P.inv_hx, -fx);
+  g.dy = fma(v, P.inv_hy, -fy);
   g.w = valid ? (LAG ? w : 0.25 * w) : 0.0;  // 0.25 undoes the 2 x 2 scaling of the TSC weights
   g.cell = valid ? (iy - 1) * P.PX + (ix - 1) : kNoCell;
   return g;
