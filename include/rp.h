@@ -134,11 +134,13 @@ int rp_create(const rp_config* cfg, const rp_dist* dist, rp_ctx** out);
 
 /* Subtree work units: in the near-field subregion S_0 a segment at level
  * level-1 that splits hands its two children to a second, persistent launch instead of
- * descending (at most 64 per item, in DFS order), so one deep tree does not bound the step
- * on one warp.  The tree, every decision and the counts are unchanged; only the summation
- * groups the subtrees (results within rounding, bit-identical across ranks).  level = 0
- * turns it off; default 12.  EINVAL unless level == 0 or 2 <= level <= max_depth. */
-int rp_set_work_split(rp_ctx* ctx, int32_t level);
+ * descending (at most `budget` per item, the first in DFS order; a segment that would exceed
+ * the budget descends in place), so one deep tree does not bound the step on one warp.  The
+ * tree, every decision and the counts are unchanged; only the summation groups the subtrees
+ * (results within rounding, bit-identical across ranks).  level = 0 turns it off; default
+ * level 12, budget 64.  budget = 0 keeps the default.  EINVAL unless level == 0 or
+ * 2 <= level <= max_depth, and budget == 0 or an even number in 2..64. */
+int rp_set_work_split(rp_ctx* ctx, int32_t level, int32_t budget);
 
 /* Destroy a context (NULL is ignored).  Synchronises its stream first. */
 void rp_destroy(rp_ctx* ctx);

@@ -1209,7 +1209,7 @@ static int run_potentials(rp_ctx* ctx, Params P, int32_t rank, int32_t world,
     }
     P.split_level = (KIND == RP_SRC_GRID && var >= 4 && P.bp_off == nullptr) ? ctx->split_level : 0;
     P.split_j = ctx->split_j;
-    P.unit_budget = kUnitBudget;
+    P.unit_budget = ctx->unit_budget;  // <= kUnitBudget, the slots allocated per item
     P.unit_ndef = ctx->unit_ndef;
     P.unit_key = ctx->unit_key;
     P.unit_val = ctx->unit_val;

@@ -159,11 +159,14 @@ int rp_set_schedule(rp_ctx* ctx, int32_t policy, int32_t k) {
   return RP_OK;
 }
 
-int rp_set_work_split(rp_ctx* ctx, int32_t level) {
+int rp_set_work_split(rp_ctx* ctx, int32_t level, int32_t budget) {
   if (!ctx) return RP_EINVAL;
   if (level != 0 && (level < 2 || level > ctx->cfg.max_depth))
     return rp_fail(ctx, RP_EINVAL, "set_work_split: level must be 0 or 2..max_depth");
+  if (budget != 0 && (budget < 2 || budget > 64 || (budget & 1)))
+    return rp_fail(ctx, RP_EINVAL, "set_work_split: budget must be 0 or even in 2..64");
   ctx->split_level = level;
+  ctx->unit_budget = budget ? budget : 64;
   return RP_OK;
 }
 

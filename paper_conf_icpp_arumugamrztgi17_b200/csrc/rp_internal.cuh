@@ -113,6 +113,7 @@ struct rp_ctx {
 
   // subtree work units of the deep trees (k_integrate split_level; rp_set_work_split)
   int split_level = 12;             // 0 = off
+  int unit_budget = 64;             // units per near-field item (<= the slots allocated, 64)
   int split_j = 1;                  // split the trees of subregions j < split_j (the near field)
   long long unit_slots = 0;         // npts * split_j * unit budget
   int32_t* unit_ndef = nullptr;     // [npts * split_j] units deferred per near-field item

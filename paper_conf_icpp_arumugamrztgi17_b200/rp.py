@@ -103,7 +103,7 @@ _SIG = {
     "rp_profile_read": (C.c_int, [_vp, _P(rp_profile)]),
     "rp_create": (C.c_int, [_P(rp_config), _P(rp_dist), _P(_vp)]),
     "rp_nccl_unique_id": (C.c_int, [_vp]),
-    "rp_set_work_split": (C.c_int, [_vp, _i32]),
+    "rp_set_work_split": (C.c_int, [_vp, _i32, _i32]),
     "rp_destroy": (None, [_vp]),
     "rp_set_stream": (C.c_int, [_vp, _vp]),
     "rp_history_init": (C.c_int, [_vp, _i32, _P(rp_frame), _vp, _i32]),
@@ -267,8 +267,8 @@ def rp_create(nx, ny, hx, hy, history_depth, c, dt, tau, n_theta=64, max_depth=3
     return out
 
 
-def rp_set_work_split(ctx, level) -> None:
-    _check(_lib.rp_set_work_split(ctx, int(level)), ctx, "rp_set_work_split")
+def rp_set_work_split(ctx, level, budget=0) -> None:
+    _check(_lib.rp_set_work_split(ctx, int(level), int(budget)), ctx, "rp_set_work_split")
 
 
 def rp_destroy(ctx) -> None:

@@ -61,6 +61,8 @@ def test_host_side_calls_without_gpu():
     # setters reject bad arguments on a NULL context before touching it
     with pytest.raises(rp.RpError):
         rp.rp_set_work_split(None, 5)
+    with pytest.raises(rp.RpError):
+        rp.rp_set_work_split(None, 5, 3)
 
 
 def test_nccl_unique_id_loads_nccl_at_run_time():

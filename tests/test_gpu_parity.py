@@ -183,10 +183,11 @@ def test_potentials_bend_cfg2_full_size_sampled(torch):
     from paper_conf_icpp_arumugamrztgi17_b200 import rp
     cfg = W.config(2)
     ring, (x, y, ux, uy, q) = _deposit_rigid_ring(cfg)
-    pts = W.sample_points(cfg.nx, cfg.ny, 40, seed=5)
+    pts = W.sample_points(cfg.nx, cfg.ny, 128, seed=5)
     orc = G.oracle_problem(cfg, ring, W.ring_frames(cfg, 0), 0, cfg.n_pre).potentials(pts)
     ctx = G.make_ctx(cfg)
     try:
+        rp.rp_set_schedule(ctx, rp.RP_SCHED_SUBREGION, 1)  # bench.py's launch configuration
         pre = W.frames(cfg, range(-cfg.n_pre, 0))
         rp.rp_history_init(ctx, cfg.n_pre, pre, None, True)
         xd, yd, uxd, uyd = _dev_arrays(torch, x, y, ux, uy)
@@ -238,29 +239,37 @@ def test_potentials_bend_small_full_mesh_two_steps(torch, rule, interp):
 def test_subtree_units_match_the_unsplit_walk(torch):
     """Deep trees split into subtree work units walk the same canonical tree:
     equal segment counts per point and values equal to the single-warp walk up to the
-    summation grouping (config 2 at full size, the bench workload)."""
+    summation grouping (config 2 at full size, the bench workload).  With a per-item budget
+    of 2 units every further level-11 split of a near-field item descends in place (the
+    budget-full path): same tree, fewer units."""
     from paper_conf_icpp_arumugamrztgi17_b200 import rp
     cfg = W.config(2)
     ring, _ = _deposit_rigid_ring(cfg)
     frames = W.ring_frames(cfg, 0)
     out = {}
-    for split in ("12", "0"):
+    for split, budget in ((12, 0), (12, 2), (0, 0)):
         ctx = G.make_ctx(cfg)
         try:
-            rp.rp_set_work_split(ctx, int(split))
+            rp.rp_set_work_split(ctx, split, budget)
             G.load_state(ctx, cfg, 0, cfg.n_pre, ring, frames)
-            out[split] = G.gpu_potentials(ctx, cfg.nx * cfg.ny)
+            out[(split, budget)] = G.gpu_potentials(ctx, cfg.nx * cfg.ny)
         finally:
             rp.rp_destroy(ctx)
-    (a, ia), (b, ib) = out["12"], out["0"]
-    assert ia.units > 1000 and ib.units == 0
-    for k in ("nseg", "nleaf", "capped"):
-        np.testing.assert_array_equal(a[k], b[k])
-    assert ia.evals == ib.evals and ia.leaves == ib.leaves and ia.capped == ib.capped
-    scale = max(np.abs(b["phi"]).max(), np.abs(b["ax"]).max(), np.abs(b["ay"]).max())
-    # the leaf error estimate eps is merged from the units like the values (ADVICE r01)
-    for k in ("phi", "ax", "ay", "err"):
-        assert np.abs(a[k] - b[k]).max() <= 1e-13 * scale, k
+    b, ib = out[(0, 0)]
+    assert ib.units == 0
+    for key in ((12, 0), (12, 2)):
+        a, ia = out[key]
+        assert ia.units > 1000
+        for k in ("nseg", "nleaf", "capped"):
+            np.testing.assert_array_equal(a[k], b[k])
+        assert ia.evals == ib.evals and ia.leaves == ib.leaves and ia.capped == ib.capped
+        scale = max(np.abs(b["phi"]).max(), np.abs(b["ax"]).max(), np.abs(b["ay"]).max())
+        # the leaf error estimate eps is merged from the units like the values (ADVICE r01)
+        for k in ("phi", "ax", "ay", "err"):
+            assert np.abs(a[k] - b[k]).max() <= 1e-13 * scale, (key, k)
+    # the budget binds: at most 2 units per near-field item, fewer than the default budget's
+    assert out[(12, 2)][1].units < out[(12, 0)][1].units
+    assert out[(12, 2)][1].units <= 2 * cfg.nx * cfg.ny
 
 
 @pytest.mark.parametrize("which", ["bend_small", "cfg2_sampled"])
@@ -630,15 +639,16 @@ def test_history_init_explicit_grids_and_empty_deposit(torch):
 @pytest.mark.slow
 def test_potentials_bend_cfg3_full_size_sampled(torch):
     """Config 3 (128x128, 1e7 particles, full history kappa = 500) through the product path;
-    the oracle computes a stratified sample of 24 points from its own deposit."""
+    the oracle computes a stratified sample of 128 points from its own deposit."""
     from paper_conf_icpp_arumugamrztgi17_b200 import rp
     cfg = W.config(3)
     ring, (x, y, ux, uy, q) = _deposit_rigid_ring(cfg)
-    pts = W.sample_points(cfg.nx, cfg.ny, 24, seed=9)
+    pts = W.sample_points(cfg.nx, cfg.ny, 128, seed=9)
     orc = G.oracle_problem(cfg, ring, W.ring_frames(cfg, 0), 0, cfg.n_pre).potentials(pts)
     del ring
     ctx = G.make_ctx(cfg)
     try:
+        rp.rp_set_schedule(ctx, rp.RP_SCHED_SUBREGION, 1)  # bench.py's launch configuration
         rp.rp_history_init(ctx, cfg.n_pre, W.frames(cfg, range(-cfg.n_pre, 0)), None, True)
         xd, yd, uxd, uyd = _dev_arrays(torch, x, y, ux, uy)
         rp.rp_deposit_step(ctx, xd, yd, uxd, uyd, q, W.frame(cfg, 0))
@@ -654,16 +664,17 @@ def test_potentials_bend_cfg3_full_size_sampled(torch):
 @pytest.mark.slow
 def test_potentials_bend_cfg4_full_size_sampled(torch):
     """Config 4 (256x256, 1e8 particles, full history kappa = 1000: BASELINE.json configs[3])
-    through the product path on one GPU; the oracle computes 16 stratified points from its own
+    through the product path on one GPU; the oracle computes 64 stratified points from its own
     deposit of the same 1e8 particles (2.1 GB ring on the host)."""
     from paper_conf_icpp_arumugamrztgi17_b200 import rp
     cfg = W.config(4)
     ring, (x, y, ux, uy, q) = _deposit_rigid_ring(cfg)
-    pts = W.sample_points(cfg.nx, cfg.ny, 16, seed=13)
+    pts = W.sample_points(cfg.nx, cfg.ny, 64, seed=13)
     orc = G.oracle_problem(cfg, ring, W.ring_frames(cfg, 0), 0, cfg.n_pre).potentials(pts)
     del ring
     ctx = G.make_ctx(cfg)
     try:
+        rp.rp_set_schedule(ctx, rp.RP_SCHED_SUBREGION, 1)  # bench.py's launch configuration
         rp.rp_history_init(ctx, cfg.n_pre, W.frames(cfg, range(-cfg.n_pre, 0)), None, True)
         xd, yd, uxd, uyd = _dev_arrays(torch, x, y, ux, uy)
         del x, y, ux, uy
@@ -681,15 +692,16 @@ def test_potentials_bend_cfg4_full_size_sampled(torch):
 @pytest.mark.slow
 def test_potentials_bend_cfg5_full_size_sampled(torch):
     """Config 5 (512x512, 1e8 particles, kappa = 2000: BASELINE.json configs[4]) on one GPU
-    (76 GB of HBM), the oracle on 12 stratified points with a 16.8 GB host ring."""
+    (76 GB of HBM), the oracle on 48 stratified points with a 16.8 GB host ring."""
     from paper_conf_icpp_arumugamrztgi17_b200 import rp
     cfg = W.config(5)
     ring, (x, y, ux, uy, q) = _deposit_rigid_ring(cfg)
-    pts = W.sample_points(cfg.nx, cfg.ny, 12, seed=17)
+    pts = W.sample_points(cfg.nx, cfg.ny, 48, seed=17)
     orc = G.oracle_problem(cfg, ring, W.ring_frames(cfg, 0), 0, cfg.n_pre).potentials(pts)
     del ring
     ctx = G.make_ctx(cfg)
     try:
+        rp.rp_set_schedule(ctx, rp.RP_SCHED_SUBREGION, 1)  # bench.py's launch configuration
         rp.rp_history_init(ctx, cfg.n_pre, W.frames(cfg, range(-cfg.n_pre, 0)), None, True)
         xd, yd, uxd, uyd = _dev_arrays(torch, x, y, ux, uy)
         del x, y, ux, uy
@@ -704,7 +716,7 @@ def test_potentials_bend_cfg5_full_size_sampled(torch):
         rp.rp_destroy(ctx)
 
 
-@pytest.mark.parametrize("policy,k", [(0, 1), (2, 9), (2, 25), (2, 5)])
+@pytest.mark.parametrize("policy,k", [(0, 1), (2, 9), (2, 25), (2, 5), (3, 1)])
 def test_schedule_policies_bit_identical(torch, policy, k):
     """The forecast (paper's predictor g) only orders the work: every policy gives
     bit-identical results to the default persistence forecast over several steps."""
