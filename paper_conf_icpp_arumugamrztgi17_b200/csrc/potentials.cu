@@ -58,6 +58,7 @@ constexpr int kWarps = 1;  // warps per CTA of k_integrate (1: the warp's shared
 struct Params {
   int nx, ny, PX, npts, kmax, kap, k, H, n_theta, max_depth, n_root, rule, variant, interp;
   double hx, hy, inv_hx, inv_hy, cdt, tau, R;
+  double inv_n_theta;        // 1/N when N is a power of two (x/N = x * (1/N) exactly), else 0
   size_t slot_doubles;
   const double* ring;        // padded ring, slot 0 node (-PAD, -PAD)
   const rp_frame* frames;    // [H]
@@ -418,7 +419,7 @@ __device__ int arcs(const Item& it, const Params& P, double cu, double cv, doubl
     sincos_b(0.5 * (prev + cur), &sm, &cm);
     if (in_rect(cu + r * cm, cv + r * sm, it)) {
       th1[na] = prev;
-      dth[na] = (cur - prev) / N;
+      dth[na] = P.inv_n_theta != 0.0 ? (cur - prev) * P.inv_n_theta : (cur - prev) / N;
       ++na;
     }
     prev = cur;
@@ -701,10 +702,17 @@ __global__ void __launch_bounds__(32 * kWarps) k_integrate(
     }
     const bool pred = rt < rt_end;
     double A = ab.x, BA = __dsub_rn(ab.y, ab.x);
+    // R-10's tolerance (tau ((B - A) 2^-l)) / R = ((tau (B - A)) / R) 2^-l exactly (power-of-two
+    // scalings commute with rounding; tol stays far above the subnormals): one division per root
+    double tol0 = __ddiv_rn(__dmul_rn(P.tau, BA), P.R);
     if (pred) {  // first non-empty cut interval (one exists: the list covers S_j, [A, B] in S_j)
       for (; rt < rt_end; ++rt) {
         const double a = fmax(P.bp[rt], ab.x), b = fmin(P.bp[rt + 1], ab.y);
-        if (a < b) { A = a; BA = __dsub_rn(b, a); ++rt; break; }
+        if (a < b) {
+          A = a; BA = __dsub_rn(b, a); ++rt;
+          tol0 = __ddiv_rn(__dmul_rn(P.tau, BA), P.R);
+          break;
+        }
       }
     }
     __syncwarp();
@@ -727,7 +735,8 @@ __global__ void __launch_bounds__(32 * kWarps) k_integrate(
     const int rlev = UNIT ? P.split_level : 0;  // the walk ends when it climbs back here
     long long ix = UNIT ? (long long)(ukey & ((1ULL << kUnitShift) - 1)) : 0;
     for (;;) {
-      const double fa = ldexp((double)ix, -lev), fb = ldexp((double)(ix + 1), -lev);
+      const double p2 = __hiloint2double((1023 - lev) << 20, 0);  // 2^-lev, exact
+      const double fa = (double)ix * p2, fb = (double)(ix + 1) * p2;
       const double a = __dadd_rn(A, __dmul_rn(BA, fa)), b = __dadd_rn(A, __dmul_rn(BA, fb));
       const double m = __dmul_rn(0.5, __dadd_rn(a, b)), hw = __dmul_rn(0.5, __dsub_rn(b, a));
       // ---- node phase: lanes 0..14 build the r' nodes of the GK15 rule
@@ -820,8 +829,8 @@ __global__ void __launch_bounds__(32 * kWarps) k_integrate(
       double err = fabs(k0 - g0);
       err = fmax(err, fabs(k1 - g1));
       err = fmax(err, fabs(k2 - g2));
-      const double tol = __ddiv_rn(__dmul_rn(P.tau, ldexp(BA, -lev)), P.R);
-      if (fabs(err - tol) / tol < 1e-9) ++ties;
+      const double tol = tol0 * p2;
+      if (fabs(err - tol) < 1e-9 * tol) ++ties;
       bool finished = false;
       if (err <= tol || lev >= P.max_depth) {
         if (!(err <= tol)) ++capped;
@@ -849,7 +858,11 @@ __global__ void __launch_bounds__(32 * kWarps) k_integrate(
           bool more = false;
           for (; rt < rt_end && P.bp[rt] < ab.y; ++rt) {
             const double a = fmax(P.bp[rt], ab.x), b = fmin(P.bp[rt + 1], ab.y);
-            if (a < b) { A = a; BA = __dsub_rn(b, a); ++rt; more = true; break; }
+            if (a < b) {
+              A = a; BA = __dsub_rn(b, a); ++rt; more = true;
+              tol0 = __ddiv_rn(__dmul_rn(P.tau, BA), P.R);
+              break;
+            }
           }
           if (!more) break;
           ix = 0;
@@ -1241,6 +1254,7 @@ int rp_potentials_impl(rp_ctx* ctx, int kind, const double src[6], int32_t rank,
   P.nx = c.nx; P.ny = c.ny; P.PX = ctx->PX; P.npts = c.nx * c.ny; P.kmax = c.history_depth;
   P.kap = kappa_of(ctx); P.k = ctx->k; P.H = ctx->H; P.n_theta = c.n_theta;
   P.max_depth = c.max_depth; P.n_root = c.n_root; P.rule = c.outer_rule;
+  P.inv_n_theta = (c.n_theta & (c.n_theta - 1)) == 0 ? 1.0 / (double)c.n_theta : 0.0;
   P.variant = 0;
   P.interp = c.interp;
   P.hx = c.hx; P.hy = c.hy; P.inv_hx = 1.0 / c.hx; P.inv_hy = 1.0 / c.hy;
