@@ -157,7 +157,8 @@ int rp_predictive_setup(rp_ctx* ctx, int kap) {
   std::vector<double> bp((size_t)std::max<int64_t>(tot, 1));
   for (size_t i = 0; i < lists.size(); ++i)
     std::copy(lists[i].begin(), lists[i].end(), bp.begin() + off[i]);
-  // upload (the stream is idle: synchronous copies keep the host vectors' lifetime simple)
+  // upload on the context's stream (a non-blocking stream is not ordered after copies on the
+  // legacy default stream), then wait, so the host vectors may go out of scope
   if ((int64_t)off.size() > ctx->off_cap) {
     if (ctx->bp_off_dev) cudaFree(ctx->bp_off_dev);
     ctx->bp_off_dev = nullptr;
@@ -170,9 +171,13 @@ int rp_predictive_setup(rp_ctx* ctx, int kap) {
     RP_CUDA(cudaMalloc(&ctx->bp_dev, bp.size() * sizeof(double)));
     ctx->bp_cap = (int64_t)bp.size();
   }
-  RP_CUDA(cudaMemcpy(ctx->bp_off_dev, off.data(), off.size() * sizeof(int64_t), cudaMemcpyHostToDevice));
-  RP_CUDA(cudaMemcpy(ctx->bp_dev, bp.data(), bp.size() * sizeof(double), cudaMemcpyHostToDevice));
-  RP_CUDA(cudaMemcpy(ctx->cluster_dev, lab.data(), n * sizeof(int32_t), cudaMemcpyHostToDevice));
+  RP_CUDA(cudaMemcpyAsync(ctx->bp_off_dev, off.data(), off.size() * sizeof(int64_t),
+                          cudaMemcpyHostToDevice, ctx->stream));
+  RP_CUDA(cudaMemcpyAsync(ctx->bp_dev, bp.data(), bp.size() * sizeof(double),
+                          cudaMemcpyHostToDevice, ctx->stream));
+  RP_CUDA(cudaMemcpyAsync(ctx->cluster_dev, lab.data(), n * sizeof(int32_t),
+                          cudaMemcpyHostToDevice, ctx->stream));
+  RP_CUDA(cudaStreamSynchronize(ctx->stream));
   ctx->pred_info.active = 1;
   ctx->pred_info.clusters = m;
   ctx->pred_info.kmeans_passes = passes;

@@ -311,6 +311,9 @@ int rp_create(const rp_config* cfg, const rp_dist* dist, rp_ctx** out) {
       ctx->own_comm = 1;
     }
   }
+  // the setup copies, memsets and k_iota above ran on the legacy default stream, which a
+  // non-blocking caller stream (rp_set_stream) is not ordered after: finish them here
+  if (cudaDeviceSynchronize() != cudaSuccess) return fail(RP_ECUDA);
   *out = ctx;
   return RP_OK;
 }
