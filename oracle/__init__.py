@@ -60,9 +60,9 @@ class Source(C.Structure):
 class Result(C.Structure):
     _fields_ = [("phi", C.c_double), ("ax", C.c_double), ("ay", C.c_double), ("err", C.c_double),
                 ("nseg", C.c_int32), ("nleaf", C.c_int32), ("capped", C.c_int32),
-                ("ties", C.c_int32), ("max_level", C.c_int32), ("pad", C.c_int32),
+                ("ties", C.c_int32), ("max_level", C.c_int32), ("noise_ties", C.c_int32),
                 ("evals", C.c_int64), ("nodes", C.c_int64), ("min_margin", C.c_double),
-                ("chase_segs", C.c_int64), ("chase_evals", C.c_int64)]
+                ("chase_segs", C.c_int64), ("chase_evals", C.c_int64), ("min_noise", C.c_double)]
 
 
 _lib = None

@@ -26,10 +26,14 @@
  * stationarity in the bend.
  * "parity unpinned": none of the exported functions.
  */
+#include <float.h>
 #include <math.h>
 #include <stdint.h>
 #include <stdlib.h>
 #include <string.h>
+
+/* R-28: a decision within this many ulp of |K_rho| + |G_rho| is flagged (noise_ties) */
+#define ORC_NOISE_TIE 4.0
 
 #ifndef M_PI
 #define M_PI 3.14159265358979323846
@@ -73,12 +77,14 @@ typedef struct {
 
 typedef struct {
   double phi, ax, ay, err;      /* I_rho, I_{rho bx}, I_{rho by}, sum of leaf errors */
-  int32_t nseg, nleaf, capped, ties, max_level, pad;
+  int32_t nseg, nleaf, capped, ties, max_level;
+  int32_t noise_ties;           /* decisions inside the rounding noise of err (R-28)  */
   int64_t evals;                /* integrand evaluations (flop census)                */
   int64_t nodes;                /* r' nodes evaluated (15 per segment)                */
   double min_margin;            /* min |err - tol| / tol over all decisions           */
   int64_t chase_segs;           /* diagnostics: segments whose subtree ends in a */
   int64_t chase_evals;          /* capped leaf, and their integrand evaluations          */
+  double min_noise;             /* min |err - tol| / (eps (|K_rho| + |G_rho|)) (R-28)   */
 } orc_result;
 
 /* ------------------------------------------------------------------ */
@@ -571,6 +577,14 @@ static void tree(subctx* X, double A, double B, double R, int32_t lev, int64_t i
   double margin = fabs(err - tol) / tol;
   if (margin < res->min_margin) res->min_margin = margin;
   if (margin < 1e-9) res->ties++;
+  /* R-28: err = max_c |K_c - G_c| is a difference of two nearly equal sums; a different
+   * (equally valid) summation order moves it by a few ulp of |K| + |G| (rho component: it
+   * bounds the current components, |J| <= rho), so a decision whose margin lies within that
+   * noise is decided by rounding, not by R-10.  Diagnostic only: the tree is unchanged. */
+  const double scale = DBL_EPSILON * (fabs(K[0]) + fabs(G[0]));
+  const double noise = scale > 0.0 ? fabs(err - tol) / scale : INFINITY;
+  if (noise < res->min_noise) res->min_noise = noise;
+  if (noise < ORC_NOISE_TIE) res->noise_ties++;
   if (lev > res->max_level) res->max_level = lev;
   if (err <= tol || lev >= P->max_depth) {
     if (!(err <= tol)) {
@@ -647,6 +661,7 @@ static void point_lab_ex(const orc_params* P, const orc_hist* Hh, const orc_sour
                          orc_result* res) {
   memset(res, 0, sizeof(*res));
   res->min_margin = INFINITY;
+  res->min_noise = INFINITY;
   int32_t kap = orc_kappa(P, Hh);
   if (kap == 0) return;
   double cdt = P->c * P->dt;

@@ -165,7 +165,7 @@ def test_potentials_static_cfg1_full_mesh(torch):
     try:
         G.load_state(ctx, cfg, 0, cfg.n_pre, ring, frames)
         gpu, info = G.gpu_potentials(ctx, len(pts))
-        fail, worst, nties = G.compare_potentials(gpu, orc, pts)
+        fail, worst, nties = G.compare_potentials(gpu, orc, pts, tau=cfg.tau)
         assert not fail.any(), (np.nonzero(fail)[0][:10], worst)
         assert worst < G.REL
         assert info.segments == int(orc["nseg"].sum())
@@ -193,7 +193,7 @@ def test_potentials_bend_cfg2_full_size_sampled(torch):
         xd, yd, uxd, uyd = _dev_arrays(torch, x, y, ux, uy)
         rp.rp_deposit_step(ctx, xd, yd, uxd, uyd, q, W.frame(cfg, 0))
         gpu, info = G.gpu_potentials(ctx, cfg.nx * cfg.ny)
-        fail, worst, nties = G.compare_potentials(gpu, orc, pts)
+        fail, worst, nties = G.compare_potentials(gpu, orc, pts, tau=cfg.tau)
         assert not fail.any(), (pts[fail][:10], worst)
         assert np.isfinite(gpu["phi"]).all()
     finally:
@@ -230,7 +230,7 @@ def test_potentials_bend_small_full_mesh_two_steps(torch, rule, interp):
             orc = G.oracle_problem(cfg, ring, frames, k, cfg.n_pre).potentials(pts)
             G.load_state(ctx, cfg, k, cfg.n_pre, ring, frames)
             gpu, info = G.gpu_potentials(ctx, len(pts))
-            fail, worst, nties = G.compare_potentials(gpu, orc, pts)
+            fail, worst, nties = G.compare_potentials(gpu, orc, pts, tau=cfg.tau)
             assert not fail.any(), (np.nonzero(fail)[0][:10], worst)
     finally:
         rp.rp_destroy(ctx)
@@ -330,7 +330,7 @@ def test_potentials_variants(torch, variant):
     try:
         G.load_state(ctx, cfg, 3, 0, ring, frames)
         gpu, info = G.gpu_potentials(ctx, len(pts))
-        fail, worst, _ = G.compare_potentials(gpu, orc, pts)
+        fail, worst, _ = G.compare_potentials(gpu, orc, pts, tau=cfg.tau)
         assert not fail.any(), (np.nonzero(fail)[0][:10], worst)
         if "max_depth" in variant:
             assert info.capped > 0 and info.capped == int(orc["capped"].sum())
@@ -357,7 +357,7 @@ def test_potentials_degenerate_kappa_zero_and_min_grid(torch):
         for l in range(3):
             ring[l % cfg.H] = M
         orc = G.oracle_problem(cfg, ring, W.ring_frames(cfg, 2), 2, 0).potentials(np.arange(16))
-        fail, worst, _ = G.compare_potentials(gpu, orc, np.arange(16))
+        fail, worst, _ = G.compare_potentials(gpu, orc, np.arange(16), tau=cfg.tau)
         assert not fail.any(), worst
     finally:
         rp.rp_destroy(ctx)
@@ -398,7 +398,7 @@ def test_analytic_sources_closed_form_on_gpu(torch, kind):
                              tau=1e-6 * sq if kind == "gauss" else 1e-6)
         pts = np.arange(81)
         orc = P.potentials(pts)
-        fail, worst, _ = G.compare_potentials(gpu, orc, pts)
+        fail, worst, _ = G.compare_potentials(gpu, orc, pts, tau=P.params.tau)
         assert not fail.any(), worst
         for p in pts:
             px, py = P.mesh_point(p % 9, p // 9)
@@ -630,7 +630,7 @@ def test_history_init_explicit_grids_and_empty_deposit(torch):
         full[0 % cfg.H] = 0.0  # step 0 grid is empty
         pts = np.arange(cfg.nx * cfg.ny)
         orc = G.oracle_problem(cfg, full, W.ring_frames(cfg, 0), 0, n_pre).potentials(pts)
-        fail, worst, _ = G.compare_potentials(gpu, orc, pts)
+        fail, worst, _ = G.compare_potentials(gpu, orc, pts, tau=cfg.tau)
         assert not fail.any(), worst
     finally:
         rp.rp_destroy(ctx)
@@ -653,7 +653,7 @@ def test_potentials_bend_cfg3_full_size_sampled(torch):
         xd, yd, uxd, uyd = _dev_arrays(torch, x, y, ux, uy)
         rp.rp_deposit_step(ctx, xd, yd, uxd, uyd, q, W.frame(cfg, 0))
         gpu, info = G.gpu_potentials(ctx, cfg.nx * cfg.ny)
-        fail, worst, _ = G.compare_potentials(gpu, orc, pts)
+        fail, worst, _ = G.compare_potentials(gpu, orc, pts, tau=cfg.tau)
         assert not fail.any(), (pts[fail][:10], worst)
         assert info.kappa == cfg.kappa_max
         assert info.units > 0
@@ -681,7 +681,7 @@ def test_potentials_bend_cfg4_full_size_sampled(torch):
         rp.rp_deposit_step(ctx, xd, yd, uxd, uyd, q, W.frame(cfg, 0))
         del xd, yd, uxd, uyd
         gpu, info = G.gpu_potentials(ctx, cfg.nx * cfg.ny)
-        fail, worst, _ = G.compare_potentials(gpu, orc, pts)
+        fail, worst, _ = G.compare_potentials(gpu, orc, pts, tau=cfg.tau)
         assert not fail.any(), (pts[fail][:10], worst)
         assert info.kappa == cfg.kappa_max
         assert info.units > 0
@@ -708,7 +708,7 @@ def test_potentials_bend_cfg5_full_size_sampled(torch):
         rp.rp_deposit_step(ctx, xd, yd, uxd, uyd, q, W.frame(cfg, 0))
         del xd, yd, uxd, uyd
         gpu, info = G.gpu_potentials(ctx, cfg.nx * cfg.ny)
-        fail, worst, _ = G.compare_potentials(gpu, orc, pts)
+        fail, worst, _ = G.compare_potentials(gpu, orc, pts, tau=cfg.tau)
         assert not fail.any(), (pts[fail][:10], worst)
         assert info.kappa == cfg.kappa_max
         assert info.units > 0

@@ -33,7 +33,7 @@ def _two_steps(cfg, rings, n_pre, knn, m, pts=None):
         G.load_state(ctx, cfg, k0, n_pre, ring0, fr0)
         gpu0, _ = G.gpu_potentials(ctx, npts)  # no previous pattern yet: canonical tree
         assert rp.rp_predictive_info_read(ctx).active == 0
-        fail, worst, _ = G.compare_potentials(gpu0, canon0, allp)
+        fail, worst, _ = G.compare_potentials(gpu0, canon0, allp, tau=cfg.tau)
         assert not fail.any(), worst
         G.load_state(ctx, cfg, k1, n_pre, ring1, fr1)
         gpu1, info = G.gpu_potentials(ctx, npts)
@@ -42,7 +42,7 @@ def _two_steps(cfg, rings, n_pre, knn, m, pts=None):
         rp.rp_destroy(ctx)
     assert pinfo.active == 1 and pinfo.kmeans_passes == passes
     np.testing.assert_array_equal(clusters, clusters1)
-    fail, worst, nties = G.compare_potentials(gpu1, pred1, pts)
+    fail, worst, nties = G.compare_potentials(gpu1, pred1, pts, tau=cfg.tau)
     assert not fail.any(), (np.nonzero(fail)[0][:10], worst)
     assert info.segments == int(pred1["nseg"].sum()) or len(pts) < npts
     # forecast-dependent, but within the tolerance of the canonical result
