@@ -106,6 +106,13 @@ def lib():
             "orc_knn_pattern": (i32, [pu16, i32, i32, i32, i32, i32, i32]),
             "orc_kmeans": (i32, [pu16, i32, i32, i32, i32, pi32]),
             "orc_merge_partitions": (i64, [P(Params), pu16, pi32, i32, i32, pi64, pd]),
+            "orc_merge_partitions_mode": (i64, [P(Params), pu16, pi32, i32, i32, i32, pi64, pi32,
+                                                pd, pi64, pd]),
+            "orc_potentials_parts": (None, [P(Params), P(Hist), P(Source), pi32, i32, pi64, pd,
+                                            P(Result)]),
+            "orc_potentials_predictive2": (i32, [P(Params), P(Hist), P(Source), pu16, i32, i32,
+                                                 i32, i32, pi64, pi32, pd, pi32, i32, pi32, pu16,
+                                                 P(Result)]),
             "orc_clip_at": (i32, [P(Params), P(Hist), P(Source), d, d, i32, pd, pd]),
             "orc_dists_at": (None, [P(Params), P(Hist), P(Source), d, d, i32, d, pd, pd]),
             "orc_centre_at": (None, [P(Params), P(Hist), P(Source), d, d, i32, d, pd, pd, pd]),
@@ -240,6 +247,62 @@ class Problem:
                                              _pi(pts), len(pts), _pi(clusters), _pu16(leaves), out)
         res = np.ctypeslib.as_array(out).copy()[:len(pts)]
         return res, clusters, leaves, it
+
+    def potentials_parts(self, pts):
+        """The accepted partition of every item (P:104's partition of an earlier step): for
+        point i and subregion j, the leaves' left ends in r' order and the last right end
+        (count + 1 doubles; none without leaves).  Returns (results, leaves [len(pts), kmax],
+        off [len(pts) * kmax] int64, plen [len(pts) * kmax] int32, parts float64)."""
+        pts = np.ascontiguousarray(pts, dtype=np.int32)
+        res, leaves = self.potentials_items(pts)
+        plen = np.where(leaves > 0, leaves.astype(np.int64) + 1, 0).reshape(-1)
+        off = np.zeros(plen.size, dtype=np.int64)
+        off[1:] = np.cumsum(plen)[:-1]
+        parts = np.zeros(max(int(plen.sum()), 1))
+        out = (Result * max(len(pts), 1))()
+        lib().orc_potentials_parts(C.byref(self.params), C.byref(self.hist), C.byref(self.source),
+                                   _pi(pts), len(pts), off.ctypes.data_as(C.POINTER(C.c_int64)),
+                                   _pd(parts), out)
+        return res, leaves, off, plen.astype(np.int32), parts
+
+    def potentials_predictive_adaptive(self, prev, prev_off, prev_len, prev_parts, pts, knn=9,
+                                       m=0, max_iters=20):
+        """Predictive-RP with adaptive partitioning (reading R-26b): line 4 refines the
+        earlier step's accepted partitions of all nx*ny points (potentials_parts over every
+        point, in point order) by the forecast.  Same returns as potentials_predictive."""
+        prev = np.ascontiguousarray(prev, dtype=np.uint16)
+        nall = self.params.nx * self.params.ny
+        assert prev.shape == (nall, self.params.kappa_max)
+        prev_off = np.ascontiguousarray(prev_off, dtype=np.int64)
+        prev_len = np.ascontiguousarray(prev_len, dtype=np.int32)
+        prev_parts = np.ascontiguousarray(prev_parts, dtype=np.float64)
+        assert prev_off.size == nall * self.params.kappa_max == prev_len.size
+        pts = np.ascontiguousarray(pts, dtype=np.int32)
+        out = (Result * max(len(pts), 1))()
+        clusters = np.zeros(nall, dtype=np.int32)
+        leaves = np.zeros((len(pts), self.params.kappa_max), dtype=np.uint16)
+        it = lib().orc_potentials_predictive2(
+            C.byref(self.params), C.byref(self.hist), C.byref(self.source), _pu16(prev), knn, m,
+            max_iters, 1, prev_off.ctypes.data_as(C.POINTER(C.c_int64)), _pi(prev_len),
+            _pd(prev_parts), _pi(pts), len(pts), _pi(clusters), _pu16(leaves), out)
+        res = np.ctypeslib.as_array(out).copy()[:len(pts)]
+        return res, clusters, leaves, it
+
+    def merge_partitions_adaptive(self, pattern, assign, m, prev_off, prev_len, prev_parts):
+        """Per-cluster merged adaptive partitions (R-26b; lines 4, 9-12)."""
+        pattern = np.ascontiguousarray(pattern, dtype=np.uint16)
+        assign = np.ascontiguousarray(assign, dtype=np.int32)
+        prev_off = np.ascontiguousarray(prev_off, dtype=np.int64)
+        prev_len = np.ascontiguousarray(prev_len, dtype=np.int32)
+        prev_parts = np.ascontiguousarray(prev_parts, dtype=np.float64)
+        off = np.zeros(m * self.params.kappa_max + 1, dtype=np.int64)
+        args = (C.byref(self.params), _pu16(pattern), _pi(assign), len(assign), m, 1,
+                prev_off.ctypes.data_as(C.POINTER(C.c_int64)), _pi(prev_len), _pd(prev_parts),
+                off.ctypes.data_as(C.POINTER(C.c_int64)))
+        n = lib().orc_merge_partitions_mode(*args, None)
+        bp = np.zeros(max(n, 1))
+        lib().orc_merge_partitions_mode(*args, _pd(bp))
+        return off, bp[:n]
 
     def merge_partitions(self, pattern, assign, m):
         """Per-cluster merged uniform partitions of S_j (lines 4, 9-12): (off, breakpoints)."""

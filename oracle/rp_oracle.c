@@ -241,6 +241,8 @@ typedef struct {
   double amp[3];          /* analytic amplitudes of the 3 levels               */
   double U0, U1, V0, V1;  /* support rectangle (frame-local)                   */
   int64_t evals;
+  double* ends;           /* nullable: accepted leaves' left ends, then the last  */
+  int64_t nends;          /* right end (the item's partition; R-26b)       */
 } subctx;
 
 /* tau_t(r') = (j+1) - r'/(c dt) in [0,1] on S_j (t' = k dt - r'/c). */
@@ -593,6 +595,7 @@ static void tree(subctx* X, double A, double B, double R, int32_t lev, int64_t i
       res->chase_evals += de;
     }
     res->nleaf++;
+    if (X->ends) X->ends[X->nends++] = a;  /* DFS order = ascending r' */
     res->phi += K[0];
     res->ax += K[1];
     res->ay += K[2];
@@ -656,9 +659,12 @@ typedef struct {
   int32_t kappa_max;
 } orc_roots;
 
+/* parts (nullable): the item partitions -- for each j with accepted leaves, the leaves' left
+ * ends in r' order followed by the last leaf's right end, written at parts + parts_off[j]
+ * (parts_off [kappa_max], from a first call's leaf counts: count + 1 doubles per item). */
 static void point_lab_ex(const orc_params* P, const orc_hist* Hh, const orc_source* S,
                          double px, double py, const orc_roots* RT, uint16_t* leaves_row,
-                         orc_result* res) {
+                         const int64_t* parts_off, double* parts, orc_result* res) {
   memset(res, 0, sizeof(*res));
   res->min_margin = INFINITY;
   res->min_noise = INFINITY;
@@ -672,6 +678,8 @@ static void point_lab_ex(const orc_params* P, const orc_hist* Hh, const orc_sour
     double A, B;
     if (!orc_clip(&X, j * cdt, (j + 1) * cdt, &A, &B)) continue;
     int32_t leaves0 = res->nleaf;
+    if (parts) X.ends = parts + parts_off[j];
+    double last_b = A;
     int64_t lo = 0, hi = 0;
     if (RT) {
       int64_t i = (int64_t)RT->cluster * RT->kappa_max + j;
@@ -685,14 +693,17 @@ static void point_lab_ex(const orc_params* P, const orc_hist* Hh, const orc_sour
       for (int64_t t = lo; t + 1 < hi; ++t) {
         double a = RT->bp[t] > A ? RT->bp[t] : A;
         double b = RT->bp[t + 1] < B ? RT->bp[t + 1] : B;
-        if (a < b) tree(&X, a, b, R, 0, 0, res);
+        if (a < b) { tree(&X, a, b, R, 0, 0, res); last_b = b; }
       }
     } else if (P->n_root == 1) {
       tree(&X, A, B, R, 0, 0, res);
+      last_b = B;
     } else {
       tree(&X, A, B, R, 1, 0, res);
       tree(&X, A, B, R, 1, 1, res);
+      last_b = B;
     }
+    if (X.ends && X.nends > 0) X.ends[X.nends++] = last_b;
     if (leaves_row) {
       int32_t nl = res->nleaf - leaves0;
       leaves_row[j] = (uint16_t)(nl < 0xFFFF ? nl : 0xFFFF);
@@ -703,7 +714,7 @@ static void point_lab_ex(const orc_params* P, const orc_hist* Hh, const orc_sour
 
 void orc_point_lab(const orc_params* P, const orc_hist* Hh, const orc_source* S, double px,
                    double py, orc_result* res) {
-  point_lab_ex(P, Hh, S, px, py, NULL, NULL, res);
+  point_lab_ex(P, Hh, S, px, py, NULL, NULL, NULL, NULL, res);
 }
 
 /* Potentials at a list of mesh points (flattened iy*nx+ix) of frame k.  leaves (nullable):
@@ -719,7 +730,24 @@ void orc_potentials_ex(const orc_params* P, const orc_hist* Hh, const orc_source
     orc_mesh_point(P, Fk, p % P->nx, p / P->nx, &px, &py);
     uint16_t* row = leaves ? leaves + (int64_t)i * P->kappa_max : NULL;
     if (row) memset(row, 0, sizeof(uint16_t) * P->kappa_max);
-    point_lab_ex(P, Hh, S, px, py, NULL, row, out + i);
+    point_lab_ex(P, Hh, S, px, py, NULL, row, NULL, NULL, out + i);
+  }
+}
+
+/* The accepted partitions of every item (P:104's "partition generated at an earlier time
+ * step"): off [npts * kappa_max], point i's item j written at parts + off[i * kappa_max + j]
+ * (leaf left ends in r' order, then the last right end; nothing for an item without leaves).
+ * The offsets come from the leaf counts of orc_potentials_ex on the same state. */
+void orc_potentials_parts(const orc_params* P, const orc_hist* Hh, const orc_source* S,
+                          const int32_t* pts, int32_t npts, const int64_t* off, double* parts,
+                          orc_result* out) {
+  const orc_frame* Fk = Hh->frames + slot_of(Hh->k, Hh->H);
+#pragma omp parallel for schedule(dynamic, 1)
+  for (int32_t i = 0; i < npts; ++i) {
+    int32_t p = pts[i];
+    double px, py;
+    orc_mesh_point(P, Fk, p % P->nx, p / P->nx, &px, &py);
+    point_lab_ex(P, Hh, S, px, py, NULL, NULL, off + (int64_t)i * P->kappa_max, parts, out + i);
   }
 }
 
@@ -810,8 +838,75 @@ int32_t orc_kmeans(const uint16_t* pat, int32_t npts, int32_t kmax, int32_t m, i
  * the members of each cluster (sorted, duplicate values removed).  off has
  * m * kmax + 1 entries; bp (nullable: count only) receives the lists.  A point with
  * n_j(p) = 0 contributes nothing; an empty list means "no forecast" (canonical roots). */
+/* Line 4 by adaptive partitioning (reading R-26b): a member p whose item (p, j) had an
+ * accepted partition x_0 < ... < x_d at the earlier step (prev_parts + prev_off[p * kmax + j],
+ * prev_len[...] = d + 1 doubles) divides each of its d pieces into q = max(1, round(n/d))
+ * equal pieces, n = n_j(p) the forecast (q = (2n + d) / (2d) in integers: half up), with
+ * breakpoints x_{i-1} + (x_i - x_{i-1}) * (t / q), the last one x_i itself; a_j and b_j are
+ * added so the list covers S_j (pieces outside the earlier support stay whole).  A member
+ * without an earlier partition of S_j uses uniform partitioning.  MERGE-LISTS as above. */
+static int64_t adaptive_list(const orc_params* P, const uint16_t* pat, const int32_t* assign,
+                             int32_t npts, int32_t c, int32_t j, const int64_t* prev_off,
+                             const int32_t* prev_len, const double* prev_parts, double** buf,
+                             int64_t* cap) {
+  const int32_t kmax = P->kappa_max;
+  const double cdt = P->c * P->dt;
+  const double aj = j * cdt, bj = (j + 1) * cdt;
+  int64_t need = 0;
+  for (int32_t p = 0; p < npts; ++p) {
+    int32_t n = pat[(int64_t)p * kmax + j];
+    if (assign[p] != c || n == 0) continue;
+    int32_t len = prev_len[(int64_t)p * kmax + j];
+    if (len >= 2) {
+      int32_t d = len - 1, q = (2 * n + d) / (2 * d);
+      if (q < 1) q = 1;
+      need += (int64_t)d * q + 1 + 2;
+    } else {
+      need += n + 1;
+    }
+  }
+  if (need > *cap) {
+    *cap = need;
+    *buf = (double*)realloc(*buf, sizeof(double) * (size_t)need);
+  }
+  double* L = *buf;
+  int64_t u = 0;
+  for (int32_t p = 0; p < npts; ++p) {
+    int32_t n = pat[(int64_t)p * kmax + j];
+    if (assign[p] != c || n == 0) continue;
+    int32_t len = prev_len[(int64_t)p * kmax + j];
+    if (len >= 2) {
+      const double* x = prev_parts + prev_off[(int64_t)p * kmax + j];
+      int32_t d = len - 1, q = (2 * n + d) / (2 * d);
+      if (q < 1) q = 1;
+      L[u++] = aj;
+      L[u++] = bj;
+      for (int32_t i = 1; i <= d; ++i)
+        for (int32_t t = 0; t < q; ++t) L[u++] = x[i - 1] + (x[i] - x[i - 1]) * ((double)t / (double)q);
+      L[u++] = x[d];
+    } else {
+      for (int32_t t = 0; t <= n; ++t) L[u++] = t == n ? bj : aj + (bj - aj) * ((double)t / (double)n);
+    }
+  }
+  return u;
+}
+
+int64_t orc_merge_partitions_mode(const orc_params* P, const uint16_t* pat, const int32_t* assign,
+                                  int32_t npts, int32_t m, int32_t mode, const int64_t* prev_off,
+                                  const int32_t* prev_len, const double* prev_parts, int64_t* off,
+                                  double* bp);
+
 int64_t orc_merge_partitions(const orc_params* P, const uint16_t* pat, const int32_t* assign,
                              int32_t npts, int32_t m, int64_t* off, double* bp) {
+  return orc_merge_partitions_mode(P, pat, assign, npts, m, 0, NULL, NULL, NULL, off, bp);
+}
+
+/* mode 0: uniform partitioning; 1: adaptive partitioning (needs the earlier
+ * partitions prev_off / prev_len / prev_parts of all npts points). */
+int64_t orc_merge_partitions_mode(const orc_params* P, const uint16_t* pat, const int32_t* assign,
+                                  int32_t npts, int32_t m, int32_t mode, const int64_t* prev_off,
+                                  const int32_t* prev_len, const double* prev_parts, int64_t* off,
+                                  double* bp) {
   const int32_t kmax = P->kappa_max;
   const double cdt = P->c * P->dt;
   int64_t total = 0;
@@ -821,6 +916,17 @@ int64_t orc_merge_partitions(const orc_params* P, const uint16_t* pat, const int
   for (int32_t c = 0; c < m; ++c)
     for (int32_t j = 0; j < kmax; ++j) {
       off[(int64_t)c * kmax + j] = total;
+      if (mode == 1) {
+        int64_t q = adaptive_list(P, pat, assign, npts, c, j, prev_off, prev_len, prev_parts,
+                                  &buf, &cap);
+        if (q) qsort(buf, (size_t)q, sizeof(double), cmp_double);
+        int64_t u = 0;
+        for (int64_t i = 0; i < q; ++i)
+          if (u == 0 || buf[i] != buf[u - 1]) buf[u++] = buf[i];
+        if (bp) memcpy(bp + total, buf, sizeof(double) * (size_t)u);
+        total += u;
+        continue;
+      }
       memset(seen, 0, 65536);
       int64_t n_all = 0;
       for (int32_t p = 0; p < npts; ++p) {
@@ -856,10 +962,30 @@ int64_t orc_merge_partitions(const orc_params* P, const uint16_t* pat, const int
  * pattern [nx*ny][kmax] (e.g. from orc_potentials_ex); m = number of clusters (0: max(nx,
  * ny)).  Writes the clusters (nullable) and the results at pts; leaves (nullable) as
  * in orc_potentials_ex.  Returns the number of k-means assignment passes. */
+int32_t orc_potentials_predictive2(const orc_params* P, const orc_hist* Hh, const orc_source* S,
+                                   const uint16_t* prev, int32_t knn, int32_t m,
+                                   int32_t max_iters, int32_t mode, const int64_t* prev_off,
+                                   const int32_t* prev_len, const double* prev_parts,
+                                   const int32_t* pts, int32_t npts, int32_t* cluster_out,
+                                   uint16_t* leaves, orc_result* out);
+
 int32_t orc_potentials_predictive(const orc_params* P, const orc_hist* Hh, const orc_source* S,
                                   const uint16_t* prev, int32_t knn, int32_t m,
                                   int32_t max_iters, const int32_t* pts, int32_t npts,
                                   int32_t* cluster_out, uint16_t* leaves, orc_result* out) {
+  return orc_potentials_predictive2(P, Hh, S, prev, knn, m, max_iters, 0, NULL, NULL, NULL, pts,
+                                    npts, cluster_out, leaves, out);
+}
+
+/* mode 0: uniform partitioning; mode 1: adaptive partitioning from the earlier
+ * step's accepted partitions of all nx*ny points (prev_off / prev_len [nx*ny * kmax], as
+ * written by orc_potentials_parts). */
+int32_t orc_potentials_predictive2(const orc_params* P, const orc_hist* Hh, const orc_source* S,
+                                   const uint16_t* prev, int32_t knn, int32_t m,
+                                   int32_t max_iters, int32_t mode, const int64_t* prev_off,
+                                   const int32_t* prev_len, const double* prev_parts,
+                                   const int32_t* pts, int32_t npts, int32_t* cluster_out,
+                                   uint16_t* leaves, orc_result* out) {
   const int32_t nx = P->nx, ny = P->ny, kmax = P->kappa_max, nall = nx * ny;
   const int32_t kap = orc_kappa(P, Hh);
   if (m <= 0) m = nx > ny ? nx : ny;
@@ -871,9 +997,11 @@ int32_t orc_potentials_predictive(const orc_params* P, const orc_hist* Hh, const
   int32_t* assign = (int32_t*)malloc(sizeof(int32_t) * nall);
   int32_t iters = orc_kmeans(pat, nall, kmax, m, max_iters, assign);
   int64_t* off = (int64_t*)malloc(sizeof(int64_t) * ((size_t)m * kmax + 1));
-  int64_t nbp = orc_merge_partitions(P, pat, assign, nall, m, off, NULL);
+  int64_t nbp = orc_merge_partitions_mode(P, pat, assign, nall, m, mode, prev_off, prev_len,
+                                          prev_parts, off, NULL);
   double* bp = (double*)malloc(sizeof(double) * (size_t)(nbp > 0 ? nbp : 1));
-  orc_merge_partitions(P, pat, assign, nall, m, off, bp);
+  orc_merge_partitions_mode(P, pat, assign, nall, m, mode, prev_off, prev_len, prev_parts, off,
+                            bp);
   const orc_frame* Fk = Hh->frames + slot_of(Hh->k, Hh->H);
 #pragma omp parallel for schedule(dynamic, 1)
   for (int32_t i = 0; i < npts; ++i) {
@@ -883,7 +1011,7 @@ int32_t orc_potentials_predictive(const orc_params* P, const orc_hist* Hh, const
     orc_roots RT = {bp, off, assign[p], kmax};
     uint16_t* row = leaves ? leaves + (int64_t)i * kmax : NULL;
     if (row) memset(row, 0, sizeof(uint16_t) * kmax);
-    point_lab_ex(P, Hh, S, px, py, &RT, row, out + i);
+    point_lab_ex(P, Hh, S, px, py, &RT, row, NULL, NULL, out + i);
   }
   if (cluster_out) memcpy(cluster_out, assign, sizeof(int32_t) * nall);
   free(pat); free(assign); free(off); free(bp);

@@ -114,3 +114,61 @@ def test_predictive_singleton_clusters_one_interval_is_the_single_root_tree():
     canon = P.potentials(pts)
     for key in ("phi", "ax", "ay", "err", "nseg", "nleaf", "evals"):
         np.testing.assert_array_equal(res[key], canon[key])
+
+
+# ---------------------------------------------------------------- adaptive partitioning
+def test_adaptive_partition_refines_the_earlier_partition_golden():
+    """P:104 / R-26b: each piece of the earlier partition of S_j is cut into round(n/d) equal
+    pieces (half up, at least 1), a_j and b_j close the list, a member without an earlier
+    partition partitions S_j uniformly, and the cluster's lists are merged (sorted, distinct).
+    Dyadic values, so every breakpoint is exact; expected lists written out by hand."""
+    P = oracle.Problem(nx=2, ny=1, hx=1.0, hy=1.0, c=1.0, dt=1.0, tau=1e-6, kappa_max=1, k=5,
+                       n_pre=0)
+    x = [0.25, 0.5, 0.625, 0.75]                      # d = 3 pieces inside S_0 = [0, 1]
+    prev_parts = np.array(x)
+    prev_off = np.array([0, 0], dtype=np.int64)
+    prev_len = np.array([4, 0], dtype=np.int32)       # point 1: no earlier partition
+    assign = np.array([0, 0], dtype=np.int32)
+    cases = {
+        # n = 6, d = 3 -> 2 pieces each; point 1, n = 2 -> uniform halves of [0, 1]
+        (6, 2): [0.0, 0.25, 0.375, 0.5, 0.5625, 0.625, 0.6875, 0.75, 1.0],
+        # n = 4 -> round(4/3) = 1: the earlier partition itself, plus a_j, b_j
+        (4, 1): [0.0, 0.25, 0.5, 0.625, 0.75, 1.0],
+        # n = 5 -> round(5/3) = 2 (half up from 1.67)
+        (5, 1): [0.0, 0.25, 0.375, 0.5, 0.5625, 0.625, 0.6875, 0.75, 1.0],
+        # n = 1 -> round(1/3) = 0 -> at least 1
+        (1, 4): [0.0, 0.25, 0.5, 0.625, 0.75, 1.0],
+        # n = 9 -> 3 pieces each (thirds of 0.25 / 0.125 / 0.125)
+        (9, 0): [0.0, 0.25, 0.25 + 0.25 / 3, 0.25 + 0.25 * 2 / 3, 0.5, 0.5 + 0.125 / 3,
+                 0.5 + 0.125 * 2 / 3, 0.625, 0.625 + 0.125 / 3, 0.625 + 0.125 * 2 / 3, 0.75, 1.0],
+    }
+    for (n0, n1), want in cases.items():
+        pat = np.array([[n0], [n1]], dtype=np.uint16)
+        off, bp = P.merge_partitions_adaptive(pat, assign, 1, prev_off, prev_len, prev_parts)
+        if n1 == 4:  # point 1 uniform in quarters on top
+            want = sorted(set(want) | {0.0, 0.25, 0.5, 0.75, 1.0})
+        np.testing.assert_allclose(bp[off[0]:off[1]], want, rtol=0, atol=1e-16)
+        assert bp[off[0]] == 0.0 and bp[off[1] - 1] == 1.0
+
+
+def test_adaptive_partition_with_unchanged_forecast_reproduces_the_canonical_leaves():
+    """A static history, a one-point mesh (one cluster, one member) and the forecast equal to
+    the earlier counts (k = 1): the merged list of every S_j is the earlier accepted partition
+    plus a_j, b_j, so every root is an earlier leaf and is accepted at once -- the result is
+    the canonical tree's, one segment per leaf (whatever k-means does on a larger mesh, where
+    identical patterns share a cluster and their partitions merge, as the golden case
+    above pins)."""
+    for x0, y0 in ((0.0, 0.0), (1.3, -0.4), (3.1, 2.2), (-5.0, 0.5)):
+        P = oracle.Problem(nx=1, ny=1, hx=1.0, hy=1.0, c=1.0, dt=1.6, tau=1e-6 * SQ,
+                           kappa_max=12, k=20, n_pre=0, source=oracle.SRC_GAUSS, x0=x0, y0=y0,
+                           width=1.0, q=1.0, bx=0.3, by=-0.2)
+        canon, leaves, off, plen, parts = P.potentials_parts([0])
+        for j in range(12):  # each partition tiles the item's support [A, B] in order
+            L = parts[off[j]:off[j] + plen[j]]
+            if len(L):
+                assert (L[0], L[-1]) == P.clip(0.0, 0.0, j) and np.all(np.diff(L) > 0)
+        res, _, _, _ = P.potentials_predictive_adaptive(leaves, off, plen, parts, [0], knn=1, m=1)
+        assert res["ties"][0] + res["noise_ties"][0] == 0
+        assert res["nseg"][0] == res["nleaf"][0] == canon["nleaf"][0]
+        for key in ("phi", "ax", "ay"):
+            assert abs(res[key][0] - canon[key][0]) <= 1e-14 * abs(canon["phi"][0])
