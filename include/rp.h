@@ -302,6 +302,10 @@ int rp_debug_clip(rp_ctx* ctx, double* ab_dev, int64_t n);
  * n = nx*ny entries (either may be NULL).  Points not owned by the last shard call keep
  * stale values.  EINVAL on a wrong n, ESTATE before the first potentials call. */
 int rp_debug_point_counts(rp_ctx* ctx, int32_t* nleaf_dev, int32_t* capped_dev, int64_t n);
+/* Accepted segments of every (point, subregion) item of the last rp_compute_potentials (the
+ * observed access pattern n_j(p) of P:83-95 that the forecast reads), uint16 (saturating)
+ * [nx * ny][history_depth] device array, n = nx * ny * history_depth.  Enqueue-only. */
+int rp_debug_item_leaves(rp_ctx* ctx, uint16_t* leaves_dev, int64_t n);
 
 /* Test hook: potentials with an analytic source in place of the grid:
  * kind = RP_SRC_GAUSS (centre (x0,y0) frame-local, width = sigma, q = Q) or RP_SRC_DISK
@@ -350,11 +354,26 @@ int rp_set_schedule(rp_ctx* ctx, int32_t policy, int32_t k);
 int rp_set_predictive(rp_ctx* ctx, int32_t enable, int32_t knn, int32_t n_clusters,
                       int32_t max_iters);
 
+/* Line 4 of the Predictive-RP variant: RP_PART_UNIFORM (default) cuts S_j into
+ * n_j(p) equal pieces; RP_PART_ADAPTIVE refines the partition accepted at the earlier
+ * step (DESIGN reading R-26b): each of the d_j pieces the item (p, j) was integrated on
+ * in the previous rp_compute_potentials is cut into max(1, round(n_j / d_j)) equal pieces,
+ * a_j and b_j close the list, an item without an earlier partition falls back to uniform
+ * partitioning; then MERGE-LISTS as before.  With ADAPTIVE every call records its accepted
+ * leaves on the device (one 32-B record per leaf, a buffer of max(2^22, 4 x nx x ny x
+ * history_depth) records, grown to twice the count on overflow; a call whose predecessor
+ * overflowed it uses uniform partitioning, reported as partition = -1).  EINVAL on another mode, ENOMEM when the buffer cannot be
+ * allocated.  Takes effect at the next rp_compute_potentials. */
+#define RP_PART_UNIFORM 0
+#define RP_PART_ADAPTIVE 1
+int rp_set_predictive_partition(rp_ctx* ctx, int32_t mode);
+
 typedef struct {
   int32_t active;          /* 1 if the last rp_compute_potentials used a forecast partition    */
   int32_t clusters;        /* k-means clusters m                                               */
   int32_t kmeans_passes;   /* assignment passes made                                           */
-  int32_t pad;
+  int32_t partition;       /* line 4 used: RP_PART_UNIFORM / RP_PART_ADAPTIVE, or -1 when
+                              adaptive was asked for but the earlier leaves overflowed        */
   int64_t breakpoints;     /* total length of the merged partition lists                      */
   double host_ms;          /* host time of lines 1-12 (download of n_j, forecast, clustering,  */
                            /* merge, upload), included in the call                             */
@@ -362,6 +381,10 @@ typedef struct {
 /* Statistics of the last rp_compute_potentials (host struct, no sync).  clusters_host
  * (nullable): the k-means cluster of every mesh point [nx * ny] (parity with the oracle). */
 int rp_predictive_info_read(rp_ctx* ctx, rp_predictive_info* out, int32_t* clusters_host);
+/* The merged partition lists of the last call that used a forecast (host copies; parity with
+ * the oracle's MERGE-LISTS): off_host [clusters * history_depth + 1] (nullable), bp_host
+ * [breakpoints] (nullable).  ESTATE when no call has used a forecast partition. */
+int rp_predictive_lists_read(rp_ctx* ctx, int64_t* off_host, double* bp_host);
 
 /* Per-kernel device time, measured with CUDA events recorded on the context's stream around
  * each launch while profiling is enabled (bench.py's live roofline numbers). */

@@ -243,6 +243,7 @@ typedef struct {
   int64_t evals;
   double* ends;           /* nullable: accepted leaves' left ends, then the last  */
   int64_t nends;          /* right end (the item's partition; R-26b)       */
+  double last_b;          /* right end of the last accepted leaf, as computed     */
 } subctx;
 
 /* tau_t(r') = (j+1) - r'/(c dt) in [0,1] on S_j (t' = k dt - r'/c). */
@@ -595,7 +596,7 @@ static void tree(subctx* X, double A, double B, double R, int32_t lev, int64_t i
       res->chase_evals += de;
     }
     res->nleaf++;
-    if (X->ends) X->ends[X->nends++] = a;  /* DFS order = ascending r' */
+    if (X->ends) { X->ends[X->nends++] = a; X->last_b = b; }  /* DFS order = ascending r' */
     res->phi += K[0];
     res->ax += K[1];
     res->ay += K[2];
@@ -679,7 +680,6 @@ static void point_lab_ex(const orc_params* P, const orc_hist* Hh, const orc_sour
     if (!orc_clip(&X, j * cdt, (j + 1) * cdt, &A, &B)) continue;
     int32_t leaves0 = res->nleaf;
     if (parts) X.ends = parts + parts_off[j];
-    double last_b = A;
     int64_t lo = 0, hi = 0;
     if (RT) {
       int64_t i = (int64_t)RT->cluster * RT->kappa_max + j;
@@ -693,17 +693,17 @@ static void point_lab_ex(const orc_params* P, const orc_hist* Hh, const orc_sour
       for (int64_t t = lo; t + 1 < hi; ++t) {
         double a = RT->bp[t] > A ? RT->bp[t] : A;
         double b = RT->bp[t + 1] < B ? RT->bp[t + 1] : B;
-        if (a < b) { tree(&X, a, b, R, 0, 0, res); last_b = b; }
+        if (a < b) tree(&X, a, b, R, 0, 0, res);
       }
     } else if (P->n_root == 1) {
       tree(&X, A, B, R, 0, 0, res);
-      last_b = B;
     } else {
       tree(&X, A, B, R, 1, 0, res);
       tree(&X, A, B, R, 1, 1, res);
-      last_b = B;
     }
-    if (X.ends && X.nends > 0) X.ends[X.nends++] = last_b;
+    /* the leaves tile [A, B]; the list closes with the last leaf's right end as the tree
+     * computed it (A + (B - A) * 1, which may differ from B in the last bit) */
+    if (X.ends && X.nends > 0) X.ends[X.nends++] = X.last_b;
     if (leaves_row) {
       int32_t nl = res->nleaf - leaves0;
       leaves_row[j] = (uint16_t)(nl < 0xFFFF ? nl : 0xFFFF);

@@ -46,7 +46,8 @@ enum : int { C_ITEMS = 0, C_NEXT = 1, C_EVALS = 2, C_SEGS = 3, C_LEAVES = 4, C_C
              C_TIES = 6, C_MAXLEV = 7, C_NODES = 8, C_NOUT = 9, C_SKIP = 10, C_UNITS = 11,
              C_NEXT_U = 12, C_COUNT = 16 };
 constexpr int kUnitShift = 20;  // unit key = item << 20 | index of the subtree root at its level
-constexpr int kGridVar = 4;  // grid evaluation loop: software-pipelined rounds (6 = Lagrange-3)
+constexpr int kGridVar = 4;  // grid evaluation loop: software-pipelined rounds (6 = Lagrange-3;
+                             // 5 / 7: the same recording the accepted leaves, R-26b)
 constexpr int kUnitBudget = 64;  // subtree units per near-field item (DFS order)
 constexpr uint32_t kEmptyKey = 0xFFFFFFFFu;  // schedule key of an item without support
 
@@ -68,6 +69,10 @@ struct Params {
   const double* bp;
   const int64_t* bp_off;
   const int32_t* cluster;
+  // adaptive partitioning (R-26b): every accepted leaf appended as (a, b, item, 0)
+  double4* leaf_rec;
+  unsigned long long* leaf_count;
+  long long leaf_cap;
   // subtree work units (deep trees split at a fixed level, see k_integrate)
   int split_level;                  // 0: off
   int split_j;                      // only subregions j < split_j are split (the near field)
@@ -376,7 +381,12 @@ __device__ int arcs(const Item& it, const Params& P, double cu, double cv, doubl
     t[2 * e] = t[2 * e + 1] = CUDART_INF;
     const bool vert = e < 2;
     const double edge = e == 0 ? it.U0 : e == 1 ? it.U1 : e == 2 ? it.V0 : it.V1;
-    const double d = (edge - (vert ? cu : cv)) * rinv;
+    const double de = __dsub_rn(edge, vert ? cu : cv);
+    double d = de * rinv;
+    // near a tangency (|d| -> 1) whether the circle crosses the edge -- full circle
+    // (trapezoid) or arc (Simpson), R-11 -- is decided by the last bit of d: there it is the
+    // one IEEE division (edge - c) / r of the oracle, so both sides decide alike (R-19)
+    if (fabs(d) > 0.9999) d = __ddiv_rn(de, r);
     if (!(fabs(d) < 1.0)) continue;
     const double h = r * sqrt(1.0 - d * d);  // r sin(acos d) = r cos(asin d)
     const double lo = vert ? it.V0 : it.U0, hi = vert ? it.V1 : it.U1;
@@ -804,7 +814,7 @@ __global__ void __launch_bounds__(32 * kWarps) k_integrate(
       if (KIND == RP_SRC_GRID && VAR >= 4) {
         for (int rr = 0; rr < rounds; ++rr) {
           const int r = (nseg & 1) ? rounds - 1 - rr : rr;
-          pipelined_round<VAR == 6>(it, P, S, trig_full, 32 * r + lane, nn, N, wfull, third, st,
+          pipelined_round<(VAR == 6 || VAR == 7)>(it, P, S, trig_full, 32 * r + lane, nn, N, wfull, third, st,
                                     ccell, k0, k1, k2, g0, g1, g2, fullmask, gmask);
         }
       } else {
@@ -835,6 +845,11 @@ __global__ void __launch_bounds__(32 * kWarps) k_integrate(
       if (err <= tol || lev >= P.max_depth) {
         if (!(err <= tol)) ++capped;
         ++nleaf;
+        if ((VAR == 5 || VAR == 7) && lane == 0) {  // the accepted partition, for P:104 next call
+          const unsigned long long pos = atomicAdd(P.leaf_count, 1ULL);
+          if (pos < (unsigned long long)P.leaf_cap)
+            P.leaf_rec[pos] = make_double4(a, b, (double)item, 0.0);
+        }
         s_phi += k0; s_ax += k1; s_ay += k2; s_err += err;
         finished = true;
       } else if (!UNIT && P.split_level > 0 && lev + 1 == P.split_level && j < P.split_j &&
@@ -1220,6 +1235,15 @@ static int run_potentials(rp_ctx* ctx, Params P, int32_t rank, int32_t world,
       P.bp_off = ctx->bp_off_dev;
       P.cluster = ctx->cluster_dev;
     }
+    const bool rec = KIND == RP_SRC_GRID && ctx->pred_on && ctx->pred_part == RP_PART_ADAPTIVE &&
+                     !shard_out && var != 0 && ctx->leaf_rec;
+    if (rec) {  // this call's accepted leaves, for the next call's adaptive partitioning
+      RP_CUDA(cudaMemsetAsync(ctx->leaf_count_dev, 0, sizeof(unsigned long long), st));
+      P.leaf_rec = ctx->leaf_rec;
+      P.leaf_count = ctx->leaf_count_dev;
+      P.leaf_cap = ctx->leaf_cap;
+    }
+    ctx->leaf_valid = rec ? 1 : 0;
     P.split_level = (KIND == RP_SRC_GRID && var >= 4 && P.bp_off == nullptr) ? ctx->split_level : 0;
     P.split_j = ctx->split_j;
     P.unit_budget = ctx->unit_budget;  // <= kUnitBudget, the slots allocated per item
@@ -1229,8 +1253,10 @@ static int run_potentials(rp_ctx* ctx, Params P, int32_t rank, int32_t world,
     P.unit_cnt = ctx->unit_cnt;
     P.unit_aux = ctx->unit_aux;
     int rc2 = KIND != RP_SRC_GRID ? launch_integrate<KIND, 0>(ctx, P)
-              : var == 6 ? launch_integrate<KIND, kGridVar + 2>(ctx, P)
-                         : launch_integrate<KIND, kGridVar>(ctx, P);
+              : var == 6 ? (P.leaf_rec ? launch_integrate<KIND, kGridVar + 3>(ctx, P)
+                                         : launch_integrate<KIND, kGridVar + 2>(ctx, P))
+              : P.leaf_rec ? launch_integrate<KIND, kGridVar + 1>(ctx, P)
+                           : launch_integrate<KIND, kGridVar>(ctx, P);
     if (rc2) return rc2;
   }
   ProfScope ps_red(ctx, PK_REDUCE);
@@ -1262,6 +1288,7 @@ int rp_potentials_impl(rp_ctx* ctx, int kind, const double src[6], int32_t rank,
   P.slot_doubles = ctx->slot_doubles; P.ring = ctx->ring; P.frames = ctx->frames_dev;
   P.amp = ctx->amp_dev;
   P.bp = nullptr; P.bp_off = nullptr; P.cluster = nullptr;
+  P.leaf_rec = nullptr; P.leaf_count = nullptr; P.leaf_cap = 0;
   P.split_level = 0; P.split_j = 0; P.unit_budget = 0; P.unit_ndef = nullptr;
   P.unit_order = nullptr; P.unit_key = nullptr; P.unit_val = nullptr;
   P.unit_cnt = nullptr; P.unit_aux = nullptr;

@@ -3,7 +3,10 @@
 // runs on the CPU.  From the previous call's observed access pattern n_j(p)
 // (accepted segments per point and subregion, written by k_reduce):
 //   line 3   forecast g(p): kNN regression over the comoving mesh;
-//   line 4   COMPUTE-PARTITION: uniform partitioning of S_j into n_j(p) pieces;
+//   line 4   COMPUTE-PARTITION: uniform partitioning of S_j into n_j(p) pieces, or
+//            adaptive partitioning (R-26b): the item's partition accepted at the
+//            previous call (recorded by k_integrate) with each piece cut into
+//            max(1, round(n_j / d_j)) equal pieces, a_j and b_j added;
 //   line 6   RP-CLUSTERING: k-means of the pattern vectors, m = max(nx, ny);
 //   9-12     MERGE-LISTS of the partitions of each cluster.
 // The merged lists and the point clusters go to the device; k_integrate (potentials.cu) runs
@@ -125,7 +128,58 @@ int rp_predictive_setup(rp_ctx* ctx, int kap) {
   m = std::min(m, n);
   std::vector<int32_t>& lab = ctx->cluster_host;
   const int passes = kmeans(pat, n, d, m, ctx->pred_iters, lab);
-  // lines 4, 9-12: per (cluster, j) the sorted union of the members' uniform grids of S_j
+  // line 4 by adaptive partitioning: the previous call's accepted partition of every
+  // item, from the leaf records (a, b, item): per item the left ends in r' order, then the
+  // last right end (the leaves tile the item's support)
+  int adaptive = ctx->pred_part == RP_PART_ADAPTIVE ? 1 : 0;
+  std::vector<int64_t> poff;
+  std::vector<int32_t> plen;
+  std::vector<double> parts;
+  if (adaptive) {
+    unsigned long long cnt = 0;
+    if (ctx->leaf_valid) {
+      RP_CUDA(cudaMemcpyAsync(&cnt, ctx->leaf_count_dev, sizeof(cnt), cudaMemcpyDeviceToHost,
+                              ctx->stream));
+      RP_CUDA(cudaStreamSynchronize(ctx->stream));
+    }
+    if (!ctx->leaf_valid || cnt > (unsigned long long)ctx->leaf_cap) {
+      adaptive = -1;  // no (complete) earlier partition: uniform partitioning this call
+      if (ctx->leaf_valid) {  // grow for the next call
+        cudaFree(ctx->leaf_rec);
+        ctx->leaf_rec = nullptr;
+        const long long cap = (long long)(2 * cnt);
+        RP_CUDA(cudaMalloc(&ctx->leaf_rec, (size_t)cap * sizeof(double4)));
+        ctx->leaf_cap = cap;
+      }
+    } else {
+      std::vector<double4> rec((size_t)cnt);
+      if (cnt) {
+        RP_CUDA(cudaMemcpyAsync(rec.data(), ctx->leaf_rec, cnt * sizeof(double4),
+                                cudaMemcpyDeviceToHost, ctx->stream));
+        RP_CUDA(cudaStreamSynchronize(ctx->stream));
+      }
+      std::sort(rec.begin(), rec.end(), [](const double4& x, const double4& y) {
+        return x.z < y.z || (x.z == y.z && x.x < y.x);
+      });
+      poff.assign((size_t)n * d, 0);
+      plen.assign((size_t)n * d, 0);
+      parts.reserve(rec.size() + rec.size() / 4 + 1);
+      for (size_t i = 0; i < rec.size();) {
+        size_t e = i;
+        while (e < rec.size() && rec[e].z == rec[i].z) ++e;
+        const size_t item = (size_t)rec[i].z;
+        poff[item] = (int64_t)parts.size();
+        for (size_t t = i; t < e; ++t) parts.push_back(rec[t].x);
+        parts.push_back(rec[e - 1].y);
+        plen[item] = (int32_t)(e - i + 1);
+        i = e;
+      }
+    }
+  }
+  // lines 4, 9-12: per (cluster, j) the sorted union of the members' partitions of S_j
+  std::vector<std::vector<int>> mem(adaptive == 1 ? m : 0);
+  if (adaptive == 1)
+    for (int p = 0; p < n; ++p) mem[lab[p]].push_back(p);
   std::vector<std::vector<int>> ns((size_t)m * d);
   for (int p = 0; p < n; ++p)
     for (int j = 0; j < kap; ++j) {
@@ -136,6 +190,31 @@ int rp_predictive_setup(rp_ctx* ctx, int kap) {
   std::vector<int64_t> off((size_t)m * d + 1);
   std::vector<std::vector<double>> lists((size_t)m * d);
   parallel_for(m * d, [&](int i) {
+    if (adaptive == 1) {
+      const int c = i / d, j = i % d;
+      const double aj = (double)j * cdt, bj = (double)(j + 1) * cdt;
+      std::vector<double>& L = lists[i];
+      for (int p : mem[c]) {
+        const int q0 = pat[(size_t)p * d + j];
+        if (q0 == 0) continue;
+        const size_t it = (size_t)p * d + j;
+        if (plen[it] >= 2) {  // each earlier piece into max(1, round(n / d)) pieces
+          const double* x = parts.data() + poff[it];
+          const int dd = plen[it] - 1;
+          const int q = std::max(1, (2 * q0 + dd) / (2 * dd));
+          L.push_back(aj);
+          L.push_back(bj);
+          for (int k = 1; k <= dd; ++k)
+            for (int t = 0; t < q; ++t) L.push_back(x[k - 1] + (x[k] - x[k - 1]) * ((double)t / (double)q));
+          L.push_back(x[dd]);
+        } else {  // no earlier partition of S_j: uniform
+          for (int t = 0; t <= q0; ++t) L.push_back(t == q0 ? bj : aj + (bj - aj) * ((double)t / (double)q0));
+        }
+      }
+      std::sort(L.begin(), L.end());
+      L.erase(std::unique(L.begin(), L.end()), L.end());
+      return;
+    }
     std::vector<int>& v = ns[i];
     std::sort(v.begin(), v.end());
     v.erase(std::unique(v.begin(), v.end()), v.end());
@@ -157,6 +236,8 @@ int rp_predictive_setup(rp_ctx* ctx, int kap) {
   std::vector<double> bp((size_t)std::max<int64_t>(tot, 1));
   for (size_t i = 0; i < lists.size(); ++i)
     std::copy(lists[i].begin(), lists[i].end(), bp.begin() + off[i]);
+  ctx->pred_off_host = off;  // kept for rp_predictive_lists_read (parity with the oracle)
+  ctx->pred_bp_host.assign(bp.begin(), bp.begin() + tot);
   // upload on the context's stream (a non-blocking stream is not ordered after copies on the
   // legacy default stream), then wait, so the host vectors may go out of scope
   if ((int64_t)off.size() > ctx->off_cap) {
@@ -179,6 +260,7 @@ int rp_predictive_setup(rp_ctx* ctx, int kap) {
                           cudaMemcpyHostToDevice, ctx->stream));
   RP_CUDA(cudaStreamSynchronize(ctx->stream));
   ctx->pred_info.active = 1;
+  ctx->pred_info.partition = adaptive == 1 ? RP_PART_ADAPTIVE : adaptive == -1 ? -1 : RP_PART_UNIFORM;
   ctx->pred_info.clusters = m;
   ctx->pred_info.kmeans_passes = passes;
   ctx->pred_info.breakpoints = tot;

@@ -2,6 +2,8 @@
 // the argument checking around the kernels of deposit.cu, potentials.cu, fields_push.cu.
 #include <new>
 
+#include <algorithm>
+
 #include "rp_internal.cuh"
 
 // every entry point: a context, and its device current for the call (restored on return)
@@ -61,7 +63,7 @@ void free_all(rp_ctx* c) {
                   c->mesh_d, c->aprev_d, c->leaves_prev, c->cluster_dev, c->bp_off_dev, c->bp_dev,
                   c->unit_key, c->unit_okey, c->unit_okey_sorted, c->unit_iota, c->unit_perm, c->unit_val,
                   c->unit_ndef, c->partials_all, c->shard_buf, c->shards_all,
-                  c->unit_cnt, c->unit_aux};
+                  c->unit_cnt, c->unit_aux, c->leaf_rec, c->leaf_count_dev};
   for (void* p : ptrs)
     if (p) cudaFree(p);
   for (auto& r : c->prof) {
@@ -167,6 +169,31 @@ int rp_set_work_split(rp_ctx* ctx, int32_t level, int32_t budget) {
     return rp_fail(ctx, RP_EINVAL, "set_work_split: budget must be 0 or even in 2..64");
   ctx->split_level = level;
   ctx->unit_budget = budget ? budget : 64;
+  return RP_OK;
+}
+
+int rp_set_predictive_partition(rp_ctx* ctx, int32_t mode) {
+  RP_ENTER(ctx);
+  if (mode != RP_PART_UNIFORM && mode != RP_PART_ADAPTIVE)
+    return rp_fail(ctx, RP_EINVAL, "set_predictive_partition: mode must be 0 or 1");
+  if (mode == RP_PART_ADAPTIVE && !ctx->leaf_rec) {
+    const long long cap =
+        std::max(1LL << 22, 4LL * ctx->cfg.nx * ctx->cfg.ny * ctx->cfg.history_depth);
+    RP_CUDA(cudaMalloc(&ctx->leaf_rec, (size_t)cap * sizeof(double4)));
+    RP_CUDA(cudaMalloc(&ctx->leaf_count_dev, sizeof(unsigned long long)));
+    RP_CUDA(cudaMemsetAsync(ctx->leaf_count_dev, 0, sizeof(unsigned long long), ctx->stream));
+    ctx->leaf_cap = cap;
+  }
+  ctx->pred_part = mode;
+  ctx->leaf_valid = 0;
+  return RP_OK;
+}
+
+int rp_predictive_lists_read(rp_ctx* ctx, int64_t* off_host, double* bp_host) {
+  if (!ctx) return RP_EINVAL;
+  if (ctx->pred_off_host.empty()) return rp_fail(ctx, RP_ESTATE, "predictive_lists: no forecast partition yet");
+  if (off_host) std::copy(ctx->pred_off_host.begin(), ctx->pred_off_host.end(), off_host);
+  if (bp_host) std::copy(ctx->pred_bp_host.begin(), ctx->pred_bp_host.end(), bp_host);
   return RP_OK;
 }
 
@@ -570,6 +597,16 @@ int rp_debug_point_counts(rp_ctx* ctx, int32_t* nleaf_dev, int32_t* capped_dev, 
   k_point_counts<<<(unsigned)((n + 255) / 256), 256, 0, ctx->stream>>>(n, ctx->point_cnt, nleaf_dev,
                                                                         capped_dev);
   RP_CHECK_LAUNCH();
+  return RP_OK;
+}
+
+int rp_debug_item_leaves(rp_ctx* ctx, uint16_t* leaves_dev, int64_t n) {
+  RP_ENTER(ctx);
+  const int64_t want = (int64_t)ctx->cfg.nx * ctx->cfg.ny * ctx->cfg.history_depth;
+  if (!leaves_dev || n != want) return rp_fail(ctx, RP_EINVAL, "debug_item_leaves: n must be nx*ny*history_depth");
+  if (!ctx->has_forecast) return rp_fail(ctx, RP_ESTATE, "debug_item_leaves: no potentials call yet");
+  RP_CUDA(cudaMemcpyAsync(leaves_dev, ctx->leaves_prev, (size_t)n * sizeof(uint16_t),
+                          cudaMemcpyDeviceToDevice, ctx->stream));
   return RP_OK;
 }
 

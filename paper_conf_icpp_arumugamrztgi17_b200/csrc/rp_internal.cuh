@@ -110,6 +110,16 @@ struct rp_ctx {
   int64_t bp_cap = 0, off_cap = 0;
   std::vector<int32_t> cluster_host;
   rp_predictive_info pred_info{};
+  // adaptive partitioning (rp_set_predictive_partition, R-26b): accepted leaves of the last
+  // call, (a, b, item, 0) per leaf, appended by k_integrate; the count lives apart from the
+  // per-call counters so the next call can read it before they are cleared
+  int pred_part = 0;
+  double4* leaf_rec = nullptr;
+  long long leaf_cap = 0;
+  unsigned long long* leaf_count_dev = nullptr;
+  int leaf_valid = 0;               // the last call recorded its leaves
+  std::vector<int64_t> pred_off_host;  // the last merged lists (rp_predictive_lists_read)
+  std::vector<double> pred_bp_host;
 
   // subtree work units of the deep trees (k_integrate split_level; rp_set_work_split)
   int split_level = 12;             // 0 = off

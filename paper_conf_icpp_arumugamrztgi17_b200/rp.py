@@ -78,10 +78,10 @@ class rp_dist(C.Structure):
 
 class rp_predictive_info(C.Structure):
     _fields_ = [("active", C.c_int32), ("clusters", C.c_int32), ("kmeans_passes", C.c_int32),
-                ("pad", C.c_int32), ("breakpoints", C.c_int64), ("host_ms", C.c_double)]
+                ("partition", C.c_int32), ("breakpoints", C.c_int64), ("host_ms", C.c_double)]
 
     def as_dict(self) -> dict:
-        return {k: getattr(self, k) for k, _ in self._fields_ if k != "pad"}
+        return {k: getattr(self, k) for k, _ in self._fields_}
 
 
 if not os.path.exists(LIB_PATH):
@@ -104,6 +104,8 @@ _SIG = {
     "rp_create": (C.c_int, [_P(rp_config), _P(rp_dist), _P(_vp)]),
     "rp_nccl_unique_id": (C.c_int, [_vp]),
     "rp_set_work_split": (C.c_int, [_vp, _i32, _i32]),
+    "rp_set_predictive_partition": (C.c_int, [_vp, _i32]),
+    "rp_predictive_lists_read": (C.c_int, [_vp, _vp, _vp]),
     "rp_destroy": (None, [_vp]),
     "rp_set_stream": (C.c_int, [_vp, _vp]),
     "rp_history_init": (C.c_int, [_vp, _i32, _P(rp_frame), _vp, _i32]),
@@ -129,6 +131,7 @@ _SIG = {
     "rp_debug_bins": (C.c_int, [_vp, _vp, _i64]),
     "rp_debug_clip": (C.c_int, [_vp, _vp, _i64]),
     "rp_debug_point_counts": (C.c_int, [_vp, _vp, _vp, _i64]),
+    "rp_debug_item_leaves": (C.c_int, [_vp, _vp, _i64]),
     "rp_debug_potentials_analytic": (C.c_int, [_vp, _i32, _d, _d, _d, _d, _d, _d, _vp, _vp, _vp,
                                                _vp, _vp, _vp, _P(rp_potential_info)]),
 }
@@ -218,6 +221,25 @@ def rp_set_schedule(ctx, policy, k=9) -> None:
 def rp_set_predictive(ctx, enable=True, knn=9, n_clusters=0, max_iters=20) -> None:
     _check(_lib.rp_set_predictive(ctx, int(bool(enable)), int(knn), int(n_clusters),
                                   int(max_iters)), ctx, "rp_set_predictive")
+
+
+RP_PART_UNIFORM, RP_PART_ADAPTIVE = 0, 1
+
+
+def rp_set_predictive_partition(ctx, mode) -> None:
+    """Line 4 of the Predictive-RP variant: RP_PART_UNIFORM or RP_PART_ADAPTIVE
+    (reading R-26b)."""
+    _check(_lib.rp_set_predictive_partition(ctx, int(mode)), ctx, "rp_set_predictive_partition")
+
+
+def rp_predictive_lists_read(ctx, n_lists, n_bp):
+    """The last merged partition lists: (off int64 [n_lists + 1], bp float64 [n_bp]) with
+    n_lists = clusters * history_depth and n_bp = rp_predictive_info.breakpoints."""
+    off = np.zeros(int(n_lists) + 1, dtype=np.int64)
+    bp = np.zeros(max(int(n_bp), 1), dtype=np.float64)
+    _check(_lib.rp_predictive_lists_read(ctx, off.ctypes.data_as(_vp), bp.ctypes.data_as(_vp)),
+           ctx, "rp_predictive_lists_read")
+    return off, bp[:int(n_bp)]
 
 
 def rp_predictive_info_read(ctx, npts=None):
@@ -407,6 +429,12 @@ def rp_save_state(ctx, ring=None, H=None):
 def rp_debug_clip(ctx, ab) -> None:
     """ab: float64 CUDA tensor of nx*ny*history_depth*2 elements ((A, B) per item)."""
     _check(_lib.rp_debug_clip(ctx, _f64(ab, "ab"), ab.numel() // 2), ctx, "rp_debug_clip")
+
+
+def rp_debug_item_leaves(ctx, out) -> None:
+    """out: torch.int16 tensor of nx * ny * history_depth elements (the uint16 counts)."""
+    _check(_lib.rp_debug_item_leaves(ctx, C.c_void_p(out.data_ptr()), out.numel()), ctx,
+           "rp_debug_item_leaves")
 
 
 def rp_debug_point_counts(ctx, nleaf=None, capped=None) -> None:

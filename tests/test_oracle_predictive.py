@@ -166,7 +166,9 @@ def test_adaptive_partition_with_unchanged_forecast_reproduces_the_canonical_lea
         for j in range(12):  # each partition tiles the item's support [A, B] in order
             L = parts[off[j]:off[j] + plen[j]]
             if len(L):
-                assert (L[0], L[-1]) == P.clip(0.0, 0.0, j) and np.all(np.diff(L) > 0)
+                A, B = P.clip(0.0, 0.0, j)
+                # the last right end is the one the tree computed: A + (B - A) * 1
+                assert L[0] == A and L[-1] == A + (B - A) and np.all(np.diff(L) > 0)
         res, _, _, _ = P.potentials_predictive_adaptive(leaves, off, plen, parts, [0], knn=1, m=1)
         assert res["ties"][0] + res["noise_ties"][0] == 0
         assert res["nseg"][0] == res["nleaf"][0] == canon["nleaf"][0]

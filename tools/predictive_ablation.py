@@ -6,7 +6,8 @@ canonical tree, identical results and states); from step 1 the second one foreca
 clusters and merges.  Step 1 starts from the same state in both, so its max |phi_pred -
 phi_canon| / tau measures the forecast dependence of the result; later steps
 drift apart by that much.  Per step: integrator time (CUDA events), host time of the
-forecast/cluster/merge pipeline, integrand evaluations and segments.  usage: python tools/predictive_ablation.py [config] [steps] [knn] [m]
+forecast/cluster/merge pipeline, integrand evaluations and segments.  usage: python tools/predictive_ablation.py [config] [steps] [knn] [m] [part]
+(part: 0 uniform partitioning; 1 adaptive partitioning, P:104 / R-26b)
 """
 import json
 import os
@@ -24,9 +25,11 @@ cfgn = int(sys.argv[1]) if len(sys.argv) > 1 else 2
 steps = int(sys.argv[2]) if len(sys.argv) > 2 else 4
 knn = int(sys.argv[3]) if len(sys.argv) > 3 else 9
 m = int(sys.argv[4]) if len(sys.argv) > 4 else 0
+part = int(sys.argv[5]) if len(sys.argv) > 5 else 0
 cfg = W.config(cfgn)
 a, b = Simulation(cfg), Simulation(cfg)
 rp.rp_set_predictive(b.ctx, True, knn, m, 20)
+rp.rp_set_predictive_partition(b.ctx, part)
 for s in (a, b):
     rp.rp_profile_enable(s.ctx, True)
 rows = []
@@ -40,7 +43,8 @@ for k in range(steps):
     d = float((a.phi - b.phi).abs().max()) / cfg.tau
     rows.append(dict(step=k, canon_ms=pa.integrate_ms - last[0], pred_ms=pb.integrate_ms - last[1],
                      pred_host_ms=pinfo.host_ms if pinfo.active else 0.0,
-                     active=pinfo.active, clusters=pinfo.clusters, passes=pinfo.kmeans_passes,
+                     active=pinfo.active, partition=pinfo.partition if pinfo.active else None,
+                     clusters=pinfo.clusters, passes=pinfo.kmeans_passes,
                      breakpoints=pinfo.breakpoints, canon_evals=ia.evals, pred_evals=ib.evals,
                      canon_segments=ia.segments, pred_segments=ib.segments,
                      max_dphi_over_tau=d))
@@ -48,7 +52,7 @@ for k in range(steps):
     print(json.dumps(rows[-1]), flush=True)
 act = [r for r in rows if r["active"]]
 if act:
-    print(json.dumps({"summary": True, "config": cfg.name, "knn": knn, "m": m,
+    print(json.dumps({"summary": True, "config": cfg.name, "knn": knn, "m": m, "part": part,
                       "canon_ms": float(np.mean([r["canon_ms"] for r in act])),
                       "pred_ms": float(np.mean([r["pred_ms"] for r in act])),
                       "pred_host_ms": float(np.mean([r["pred_host_ms"] for r in act])),
