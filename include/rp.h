@@ -361,8 +361,9 @@ int rp_set_predictive(rp_ctx* ctx, int32_t enable, int32_t knn, int32_t n_cluste
  * a_j and b_j close the list, an item without an earlier partition falls back to uniform
  * partitioning; then MERGE-LISTS as before.  With ADAPTIVE every call records its accepted
  * leaves on the device (one 32-B record per leaf, a buffer of max(2^22, 4 x nx x ny x
- * history_depth) records, grown to twice the count on overflow; a call whose predecessor
- * overflowed it uses uniform partitioning, reported as partition = -1).  EINVAL on another mode, ENOMEM when the buffer cannot be
+ * history_depth) records, grown to 4x the previous call's leaves when they fill half of it and to
+ * 2x the count after an overflow; a call whose predecessor overflowed it uses uniform
+ * partitioning, reported as partition = -1).  EINVAL on another mode, ENOMEM when the buffer cannot be
  * allocated.  Takes effect at the next rp_compute_potentials. */
 #define RP_PART_UNIFORM 0
 #define RP_PART_ADAPTIVE 1

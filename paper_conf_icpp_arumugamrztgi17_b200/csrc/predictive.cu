@@ -158,6 +158,13 @@ int rp_predictive_setup(rp_ctx* ctx, int kap) {
                                 cudaMemcpyDeviceToHost, ctx->stream));
         RP_CUDA(cudaStreamSynchronize(ctx->stream));
       }
+      if (2 * cnt > (unsigned long long)ctx->leaf_cap) {  // keep room for this call's leaves
+        cudaFree(ctx->leaf_rec);
+        ctx->leaf_rec = nullptr;
+        const long long cap = (long long)(4 * cnt);
+        RP_CUDA(cudaMalloc(&ctx->leaf_rec, (size_t)cap * sizeof(double4)));
+        ctx->leaf_cap = cap;
+      }
       std::sort(rec.begin(), rec.end(), [](const double4& x, const double4& y) {
         return x.z < y.z || (x.z == y.z && x.x < y.x);
       });
