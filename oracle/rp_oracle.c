@@ -51,7 +51,7 @@ typedef struct {
   double tau;        /* absolute tolerance per component (1e-6)      */
   int32_t n_theta;   /* inner panels per arc (R-11)                          */
   int32_t max_depth; /* bisection cap (R-12)                                 */
-  int32_t n_root;    /* 2: start from both halves of [A,B]; 1: from [A,B]   */
+  int32_t n_root;    /* 2: both halves of [A,B] (quarters in S_0); 1: [A,B]; 4: quarters */
   int32_t kappa_max; /* history depth (R-4)                                  */
   int32_t rule;      /* outer segment rule: 0 = GK15 (R-8), 1 = Simpson/Boole (R-22) */
   int32_t interp;    /* spatial weights: 0 = TSC (R-6), 1 = quadratic Lagrange (R-25)  */
@@ -697,6 +697,10 @@ static void point_lab_ex(const orc_params* P, const orc_hist* Hh, const orc_sour
       }
     } else if (P->n_root == 1) {
       tree(&X, A, B, R, 0, 0, res);
+    } else if (P->n_root == 4 || j == 0) {
+      /* R-12b: the four quarters of [A, B] (level 2) -- always for the near field S_0 (r' from
+       * 0, the widest range of structure: one estimate over half of it is not trusted) */
+      for (int64_t q = 0; q < 4; ++q) tree(&X, A, B, R, 2, q, res);
     } else {
       tree(&X, A, B, R, 1, 0, res);
       tree(&X, A, B, R, 1, 1, res);

@@ -185,3 +185,30 @@ def test_grid_cartesian_fine_cell_sum():
     phi = contrib.sum() + centre
     print("cartesian", phi, r["phi"], phi / r["phi"] - 1)
     assert abs(phi - r["phi"]) < 2e-3 * abs(r["phi"]), (phi, r["phi"])
+
+
+def test_canonical_roots_halves_and_near_field_quarters():
+    """R-12b: the canonical tree starts from the two halves of each item's support and from the
+    four quarters of the near field S_0 (n_root = 2), from [A, B] itself (n_root = 1) or from
+    quarters everywhere (n_root = 4).  With a tolerance no segment can miss, every root is a
+    leaf, so the per-item leaf counts are the root counts; and the near-field quarters are the
+    exact level-2 pieces of the halves' tree (a finer tolerance that splits both S_0 halves
+    gives the same leaves and values, two segments more)."""
+    pts = np.arange(64)
+    for n_root, want0, want in ((2, 4, 2), (1, 1, 1), (4, 4, 4)):
+        P = gauss_problem(tau=1e9, n_root=n_root)
+        res, leaves = P.potentials_items(pts)
+        has = leaves > 0
+        assert (leaves[:, 0][has[:, 0]] == want0).all()
+        assert (leaves[:, 1:][has[:, 1:]] == want).all()
+        assert (res["nseg"] == leaves.sum(axis=1)).all()
+    # the quarters are the exact level-2 pieces of the one-root tree: with a tolerance tight
+    # enough that [A, B] and both its halves always split (kappa = 1: the near field only),
+    # the near-field quarters (n_root = 2) give the one-root tree's leaves and values bit for
+    # bit with three segments fewer -- a wrong level, index or endpoint would not
+    P1 = gauss_problem(kap=1, k=5, cdt=8.0, n_root=1, tau=1e-13 * SQ)
+    P2 = gauss_problem(kap=1, k=5, cdt=8.0, n_root=2, tau=1e-13 * SQ)
+    r1, r2 = P1.potentials(pts), P2.potentials(pts)
+    for key in ("phi", "ax", "ay", "err", "nleaf"):
+        np.testing.assert_array_equal(r1[key], r2[key])
+    np.testing.assert_array_equal(r1["nseg"], r2["nseg"] + 3)
