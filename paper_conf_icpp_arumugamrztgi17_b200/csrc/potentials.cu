@@ -741,7 +741,12 @@ __global__ void __launch_bounds__(32 * kWarps) k_integrate(
     }
     int nseg = 0, nleaf = 0, capped = 0, ties = 0, maxlev = 0, ndef = 0;
     unsigned evals = 0, nskip = 0;
-    int lev = UNIT ? P.split_level : ((P.n_root == 2 && !pred) ? 1 : 0);
+    // canonical roots (R-12b): the n_root = 1, 2 or 4 equal pieces of [A, B] (levels 0, 1, 2);
+    // with n_root = 2 the near field S_0 starts from its quarters
+    const int lev0 = UNIT ? P.split_level
+                          : (pred ? 0 : (P.n_root == 4 || (P.n_root == 2 && j == 0)) ? 2
+                                      : P.n_root == 2 ? 1 : 0);
+    int lev = lev0;
     const int rlev = UNIT ? P.split_level : 0;  // the walk ends when it climbs back here
     long long ix = UNIT ? (long long)(ukey & ((1ULL << kUnitShift) - 1)) : 0;
     for (;;) {
@@ -884,6 +889,9 @@ __global__ void __launch_bounds__(32 * kWarps) k_integrate(
           continue;
         }
         ++ix;
+        // levels above the roots are never evaluated: from a sibling there, go down to the
+        // first root below it (quarters: after quarter 1, quarter 2)
+        while (lev < lev0) { ++lev; ix <<= 1; }
       } else {
         ++lev;
         ix <<= 1;

@@ -21,7 +21,7 @@ int validate(const rp_config* c) {
   if ((int64_t)c->nx * c->ny * c->history_depth > 0x7fffffffLL) return RP_EINVAL;
   if (c->n_theta < 2 || (c->n_theta & 1) || c->n_theta > 4096) return RP_EINVAL;
   if (c->max_depth < 1 || c->max_depth > 60) return RP_EINVAL;
-  if (c->n_root != 1 && c->n_root != 2) return RP_EINVAL;
+  if (c->n_root != 1 && c->n_root != 2 && c->n_root != 4) return RP_EINVAL;
   if (c->outer_rule != RP_RULE_GK15 && c->outer_rule != RP_RULE_SIMPSON) return RP_EINVAL;
   if (c->interp != RP_INTERP_TSC && c->interp != RP_INTERP_LAGRANGE3) return RP_EINVAL;
   return RP_OK;

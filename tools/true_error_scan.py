@@ -25,6 +25,8 @@ from paper_conf_icpp_arumugamrztgi17_b200.sim import Simulation  # noqa: E402
 cfgn = int(sys.argv[1]) if len(sys.argv) > 1 else 2
 steps = int(sys.argv[2]) if len(sys.argv) > 2 else 5
 cfg = W.config(cfgn)
+if len(sys.argv) > 3:  # canonical roots (R-12b): 1, 2 or 4 equal pieces of the support
+    cfg.n_root = int(sys.argv[3])
 sim = Simulation(cfg)
 npts = cfg.nx * cfg.ny
 ref = rp.rp_create(cfg.nx, cfg.ny, cfg.hx, cfg.hy, cfg.kappa_max, cfg.c, cfg.dt, cfg.tau / 100,
@@ -33,9 +35,13 @@ f64 = dict(dtype=torch.float64, device="cuda")
 out = [torch.zeros(npts, **f64) for _ in range(4)]
 nseg = torch.zeros(npts, dtype=torch.int32, device="cuda")
 ring = torch.zeros(cfg.H * npts * 4, **f64)
+rp.rp_profile_enable(sim.ctx, True)
+last_ms = 0.0
 for s in range(steps):
-    sim.step()
+    own = sim.step(info=True)
     torch.cuda.synchronize()
+    prof = rp.rp_profile_read(sim.ctx)
+    own_ms, last_ms = prof.integrate_ms - last_ms, prof.integrate_ms
     k, frames = rp.rp_save_state(sim.ctx, ring, cfg.H)
     rp.rp_load_state(ref, k, cfg.n_pre, frames, ring)
     info = rp.rp_compute_potentials(ref, *out, nseg, info=True)
@@ -52,7 +58,9 @@ for s in range(steps):
                       "median_dphi_over_tau": float(np.median(dphi)),
                       "worst_point": worst,
                       "worst_eps_over_tau": float(sim.err[worst].item() / cfg.tau),
-                      "ref_capped": int(info.capped), "ref_segments": int(info.segments)}),
+                      "ref_capped": int(info.capped), "ref_segments": int(info.segments),
+                      "n_root": cfg.n_root, "segments": int(own.segments), "evals": int(own.evals),
+                      "integrate_ms": own_ms}),
           flush=True)
 rp.rp_destroy(ref)
 sim.close()
