@@ -60,6 +60,7 @@ struct Params {
   int nx, ny, PX, npts, kmax, kap, k, H, n_theta, max_depth, n_root, rule, variant, interp;
   double hx, hy, inv_hx, inv_hy, cdt, tau, R;
   double inv_n_theta;        // 1/N when N is a power of two (x/N = x * (1/N) exactly), else 0
+  double grid_extent;        // max(nx hx, ny hy): the near-field root scale (R-12b)
   size_t slot_doubles;
   const double* ring;        // padded ring, slot 0 node (-PAD, -PAD)
   const rp_frame* frames;    // [H]
@@ -743,9 +744,15 @@ __global__ void __launch_bounds__(32 * kWarps) k_integrate(
     unsigned evals = 0, nskip = 0;
     // canonical roots (R-12b): the n_root = 1, 2 or 4 equal pieces of [A, B] (levels 0, 1, 2);
     // with n_root = 2 the near field S_0 starts from its quarters
+    // the near field S_0 (n_root 2 or 4): the 2^L pieces no longer than the grid's extent,
+    // L >= 2 (R-12b), by the oracle's exact power-of-two comparisons
+    int lnear = 2;
+    while (lnear < 10 && BA > ldexp(P.grid_extent, lnear)) ++lnear;
     const int lev0 = UNIT ? P.split_level
-                          : (pred ? 0 : (P.n_root == 4 || (P.n_root == 2 && j == 0)) ? 2
-                                      : P.n_root == 2 ? 1 : 0);
+                          : pred ? 0
+                          : P.n_root == 1 ? 0
+                          : j == 0 ? lnear
+                          : P.n_root == 4 ? 2 : 1;
     int lev = lev0;
     const int rlev = UNIT ? P.split_level : 0;  // the walk ends when it climbs back here
     long long ix = UNIT ? (long long)(ukey & ((1ULL << kUnitShift) - 1)) : 0;
@@ -1289,6 +1296,7 @@ int rp_potentials_impl(rp_ctx* ctx, int kind, const double src[6], int32_t rank,
   P.kap = kappa_of(ctx); P.k = ctx->k; P.H = ctx->H; P.n_theta = c.n_theta;
   P.max_depth = c.max_depth; P.n_root = c.n_root; P.rule = c.outer_rule;
   P.inv_n_theta = (c.n_theta & (c.n_theta - 1)) == 0 ? 1.0 / (double)c.n_theta : 0.0;
+  P.grid_extent = std::max(c.nx * c.hx, c.ny * c.hy);
   P.variant = 0;
   P.interp = c.interp;
   P.hx = c.hx; P.hy = c.hy; P.inv_hx = 1.0 / c.hx; P.inv_hy = 1.0 / c.hy;

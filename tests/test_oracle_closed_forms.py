@@ -212,3 +212,38 @@ def test_canonical_roots_halves_and_near_field_quarters():
     for key in ("phi", "ax", "ay", "err", "nleaf"):
         np.testing.assert_array_equal(r1[key], r2[key])
     np.testing.assert_array_equal(r1["nseg"], r2["nseg"] + 3)
+
+
+def _near_problem(n_root, tau, cdt=12.0):
+    # grid extent L_g = 8 x 0.25 = 2: S_0 = [0, 12] clipped to the Gaussian's support (+-8
+    # widths) is longer than 4 L_g at every point, so its roots are eighths or finer
+    return oracle.Problem(nx=8, ny=8, hx=0.25, hy=0.25, c=1.0, dt=cdt, tau=tau, kappa_max=1,
+                          k=5, n_pre=0, source=oracle.SRC_GAUSS, x0=0.0, y0=0.0, width=1.0,
+                          q=1.0, bx=0.3, by=-0.2, n_root=n_root)
+
+
+def test_near_field_roots_no_longer_than_the_grid_extent():
+    """R-12b: the near field S_0 starts from the 2^L equal pieces of [A, B] with the smallest
+    L >= 2 for which (B - A) / 2^L <= L_g = max(nx hx, ny hy); with a tolerance no segment can
+    miss, the leaf count of S_0 is 2^L at every point, and with one tight enough that the
+    one-root tree splits down to level L everywhere, the pieces are that tree's level-L
+    segments bit for bit (2^L - 1 segments fewer: forced here by a tolerance nothing meets, every
+    leaf capped at D_max = 6)."""
+    pts = np.arange(64)
+    P = _near_problem(2, 1e9)
+    res, leaves = P.potentials_items(pts)
+    Ls = []
+    for p in pts:
+        A, B = P.clip(*P.mesh_point(p % 8, p // 8), 0)
+        L = next(L for L in range(2, 11) if (B - A) / 2.0 ** L <= 2.0)
+        Ls.append(L)
+        assert leaves[p, 0] == 2 ** L, (p, leaves[p, 0], L)
+    assert max(Ls) >= 3  # the rule does more than quarters here
+    # the pieces are dyadic: at a tolerance no segment can meet before D_max, the leaves are
+    # the same as the one-root tree's (all at D_max) and so are the values, bit for bit
+    P1, P2 = _near_problem(1, 1e-300), _near_problem(2, 1e-300)
+    P1.params.max_depth = P2.params.max_depth = 6
+    r1, r2 = P1.potentials(pts), P2.potentials(pts)
+    for key in ("phi", "ax", "ay", "err", "nleaf"):
+        np.testing.assert_array_equal(r1[key], r2[key])
+    np.testing.assert_array_equal(r1["nseg"], r2["nseg"] + 2 ** np.array(Ls) - 1)
