@@ -69,8 +69,9 @@ typedef struct {
   double tau;              /* > 0; absolute tolerance per component (P:170 tau = 1e-6)           */
   int32_t n_theta;         /* even >= 2; inner Newton-Cotes panels per arc (R-11)          */
   int32_t max_depth;       /* 1..60 bisection cap of the outer tree (R-12)                       */
-  int32_t n_root;          /* 2: roots are the two halves of each clipped S_j, the quarters of
-                              the near field S_0 (R-12b); 1: [A, B] itself; 4: quarters      */
+  int32_t n_root;          /* 2: roots are the two halves of each clipped S_j, and for the near
+                              field S_0 the 2^L pieces no longer than max(nx hx, ny hy), L >= 2
+                              (R-12b); 1: [A, B] itself everywhere; 4: quarters for j >= 1   */
   int32_t device;          /* CUDA ordinal                                                       */
   int32_t outer_rule;      /* RP_RULE_GK15 (default, R-8) or RP_RULE_SIMPSON: the paper's own   */
                            /* rule (P:155 RP-QUADRULE), Boole value + |S2 - S1|/15 estimate (R-22) */
@@ -198,8 +199,8 @@ int rp_deposit_step(rp_ctx* ctx, const double* x, const double* y, const double*
  * waiting for the device unless info is given (the work is capturable in a CUDA graph after
  * one warm-up call has sized the scratch).
  * For every (point p, subregion j < kappa(k)): support clip [A, B] of S_j (R-5), then a
- * deterministic top-down dyadic GK15 tree from the n_root halves of [A, B] (quarters for
- * the near field j = 0, R-12b): accept a
+ * deterministic top-down dyadic GK15 tree from the n_root halves of [A, B] (for the near
+ * field j = 0 the pieces no longer than the grid's extent, R-12b): accept a
  * segment iff max_c |K15_c - G7_c| <= tau (b - a) / R(p), R(p) = kappa(k) c dt, or at
  * max_depth (R-8..R-12).  Work items are scheduled longest-predicted-first from the
  * previous step's per-(p, j) segment counts (the paper's forecast g, used for
