@@ -701,12 +701,12 @@ static void point_lab_ex(const orc_params* P, const orc_hist* Hh, const orc_sour
       for (int64_t q = 0; q < 4; ++q) tree(&X, A, B, R, 2, q, res);
     } else if (j == 0) {
       /* R-12b: the near field S_0 (r' from 0) starts from the 2^L equal pieces of [A, B] no
-       * longer than the grid's extent L_g = max(nx hx, ny hy) -- the scale of the comoving
-       * bunch's structure that the first r' of the light cone sweep -- with L >= 2:
-       * the smallest such L, by exact power-of-two comparisons */
+       * longer than an eighth of the grid's extent L_g = max(nx hx, ny hy) -- the scale of the
+       * comoving bunch's structure that the first r' of the light cone sweep -- with
+       * 2 <= L <= 7: the smallest such L, by exact power-of-two comparisons */
       const double Lg = P->nx * P->hx > P->ny * P->hy ? P->nx * P->hx : P->ny * P->hy;
       int32_t L = 2;
-      while (L < 10 && B - A > ldexp(Lg, L)) ++L;
+      while (L < 7 && B - A > ldexp(Lg, L - 3)) ++L;
       for (int64_t q = 0; q < ((int64_t)1 << L); ++q) tree(&X, A, B, R, L, q, res);
     } else {
       tree(&X, A, B, R, 1, 0, res);

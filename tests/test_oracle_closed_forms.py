@@ -202,12 +202,14 @@ def test_canonical_roots_halves_and_near_field_quarters():
         assert (leaves[:, 0][has[:, 0]] == want0).all()
         assert (leaves[:, 1:][has[:, 1:]] == want).all()
         assert (res["nseg"] == leaves.sum(axis=1)).all()
-    # the quarters are the exact level-2 pieces of the one-root tree: with a tolerance tight
-    # enough that [A, B] and both its halves always split (kappa = 1: the near field only),
-    # the near-field quarters (n_root = 2) give the one-root tree's leaves and values bit for
-    # bit with three segments fewer -- a wrong level, index or endpoint would not
-    P1 = gauss_problem(kap=1, k=5, cdt=8.0, n_root=1, tau=1e-13 * SQ)
-    P2 = gauss_problem(kap=1, k=5, cdt=8.0, n_root=2, tau=1e-13 * SQ)
+    # the quarters are the exact level-2 pieces of the one-root tree: with a negative tolerance
+    # meets, [A, B] and both its halves always split (kappa = 1: the near field only, whose
+    # pieces are quarters here), so the near-field quarters (n_root = 2) give the one-root
+    # tree's leaves and values bit for bit with three segments fewer -- a wrong level, index
+    # or endpoint would not
+    P1 = gauss_problem(kap=1, k=5, cdt=1.6, n_root=1, tau=-1.0)
+    P2 = gauss_problem(kap=1, k=5, cdt=1.6, n_root=2, tau=-1.0)
+    P1.params.max_depth = P2.params.max_depth = 5  # every leaf capped at D_max
     r1, r2 = P1.potentials(pts), P2.potentials(pts)
     for key in ("phi", "ax", "ay", "err", "nleaf"):
         np.testing.assert_array_equal(r1[key], r2[key])
@@ -216,7 +218,7 @@ def test_canonical_roots_halves_and_near_field_quarters():
 
 def _near_problem(n_root, tau, cdt=12.0):
     # grid extent L_g = 8 x 0.25 = 2: S_0 = [0, 12] clipped to the Gaussian's support (+-8
-    # widths) is longer than 4 L_g at every point, so its roots are eighths or finer
+    # widths) is longer than L_g / 2 at every point, so its roots are eighths or finer
     return oracle.Problem(nx=8, ny=8, hx=0.25, hy=0.25, c=1.0, dt=cdt, tau=tau, kappa_max=1,
                           k=5, n_pre=0, source=oracle.SRC_GAUSS, x0=0.0, y0=0.0, width=1.0,
                           q=1.0, bx=0.3, by=-0.2, n_root=n_root)
@@ -224,25 +226,25 @@ def _near_problem(n_root, tau, cdt=12.0):
 
 def test_near_field_roots_no_longer_than_the_grid_extent():
     """R-12b: the near field S_0 starts from the 2^L equal pieces of [A, B] with the smallest
-    L >= 2 for which (B - A) / 2^L <= L_g = max(nx hx, ny hy); with a tolerance no segment can
+    2 <= L <= 7 for which (B - A) / 2^L <= L_g / 8, L_g = max(nx hx, ny hy); with a tolerance no segment can
     miss, the leaf count of S_0 is 2^L at every point, and with one tight enough that the
     one-root tree splits down to level L everywhere, the pieces are that tree's level-L
     segments bit for bit (2^L - 1 segments fewer: forced here by a tolerance nothing meets, every
-    leaf capped at D_max = 6)."""
+    leaf capped at D_max = 8)."""
     pts = np.arange(64)
     P = _near_problem(2, 1e9)
     res, leaves = P.potentials_items(pts)
     Ls = []
     for p in pts:
         A, B = P.clip(*P.mesh_point(p % 8, p // 8), 0)
-        L = next(L for L in range(2, 11) if (B - A) / 2.0 ** L <= 2.0)
+        L = next((L for L in range(2, 7) if (B - A) / 2.0 ** L <= 2.0 / 8), 7)
         Ls.append(L)
         assert leaves[p, 0] == 2 ** L, (p, leaves[p, 0], L)
     assert max(Ls) >= 3  # the rule does more than quarters here
     # the pieces are dyadic: at a tolerance no segment can meet before D_max, the leaves are
     # the same as the one-root tree's (all at D_max) and so are the values, bit for bit
-    P1, P2 = _near_problem(1, 1e-300), _near_problem(2, 1e-300)
-    P1.params.max_depth = P2.params.max_depth = 6
+    P1, P2 = _near_problem(1, -1.0), _near_problem(2, -1.0)
+    P1.params.max_depth = P2.params.max_depth = 8
     r1, r2 = P1.potentials(pts), P2.potentials(pts)
     for key in ("phi", "ax", "ay", "err", "nleaf"):
         np.testing.assert_array_equal(r1[key], r2[key])
