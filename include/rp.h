@@ -70,8 +70,9 @@ typedef struct {
   int32_t n_theta;         /* even >= 2; inner Newton-Cotes panels per arc (R-11)          */
   int32_t max_depth;       /* 1..60 bisection cap of the outer tree (R-12)                       */
   int32_t n_root;          /* 2: roots are the two halves of each clipped S_j, and for the near
-                              field S_0 the 2^L pieces no longer than max(nx hx, ny hy), L >= 2
-                              (R-12b); 1: [A, B] itself everywhere; 4: quarters for j >= 1   */
+                              field S_0 the 2^L pieces no longer than max(nx hx, ny hy) / 8,
+                              2 <= L <= 7 (R-12b); 1: [A, B] itself everywhere; 4: quarters
+                              for j >= 1                                                      */
   int32_t device;          /* CUDA ordinal                                                       */
   int32_t outer_rule;      /* RP_RULE_GK15 (default, R-8) or RP_RULE_SIMPSON: the paper's own   */
                            /* rule (P:155 RP-QUADRULE), Boole value + |S2 - S1|/15 estimate (R-22) */
@@ -200,7 +201,7 @@ int rp_deposit_step(rp_ctx* ctx, const double* x, const double* y, const double*
  * one warm-up call has sized the scratch).
  * For every (point p, subregion j < kappa(k)): support clip [A, B] of S_j (R-5), then a
  * deterministic top-down dyadic GK15 tree from the n_root halves of [A, B] (for the near
- * field j = 0 the pieces no longer than the grid's extent, R-12b): accept a
+ * field j = 0 the pieces no longer than an eighth of the grid's extent, R-12b): accept a
  * segment iff max_c |K15_c - G7_c| <= tau (b - a) / R(p), R(p) = kappa(k) c dt, or at
  * max_depth (R-8..R-12).  Work items are scheduled longest-predicted-first from the
  * previous step's per-(p, j) segment counts (the paper's forecast g, used for

@@ -744,10 +744,10 @@ __global__ void __launch_bounds__(32 * kWarps) k_integrate(
     unsigned evals = 0, nskip = 0;
     // canonical roots (R-12b): the n_root = 1, 2 or 4 equal pieces of [A, B] (levels 0, 1, 2);
     // with n_root = 2 the near field S_0 starts from its quarters
-    // the near field S_0 (n_root 2 or 4): the 2^L pieces no longer than the grid's extent,
-    // L >= 2 (R-12b), by the oracle's exact power-of-two comparisons
+    // the near field S_0 (n_root 2 or 4): the 2^L pieces no longer than an eighth of the
+    // grid's extent, 2 <= L <= 7 (R-12b), by the oracle's exact power-of-two comparisons
     int lnear = 2;
-    while (lnear < 10 && BA > ldexp(P.grid_extent, lnear)) ++lnear;
+    while (lnear < 7 && BA > ldexp(P.grid_extent, lnear - 3)) ++lnear;
     const int lev0 = UNIT ? P.split_level
                           : pred ? 0
                           : P.n_root == 1 ? 0
